@@ -1,0 +1,407 @@
+"""Benchmark of the matchmaking hot path on B200 (driver contract: one JSON line).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--app stream|stream-loop|hotspot|stencil|blackscholes|sgemm]
+
+Workload (default): BASELINE.json configs[1] — MK-Seq STREAM copy/scale/add/
+triad on 2^28 FP32 elements, one STREAM-Seq pass per step.  A step is the whole
+hot path: classify -> rank (Table I) -> split -> run the best-ranked strategy
+(SP-Unified for MK-Seq without sync).  Profiling (Glinda's probes, the DP
+warm-up) is excluded from timing as in the paper (P311).  Inputs are 1 GiB per
+array (> 126 MB L2), generated in place; no L2 flush is needed.
+
+value = algorithmic bytes of the step (40 B/element/pass) / device time, summed
+over all ranks' work and divided by the max-over-ranks time (whole job).
+Under torchrun (N>1) every rank owns one GPU = one logical device; exchanges
+go through the library's NCCL communicator.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "per-app exec time & speedup vs 1 GPU per strategy at 1/2/4/8 B200; HBM % peak"
+
+APPS = {
+    # name: (builtin id, iparam, algorithmic bytes per step as fn(iparam), description)
+    "stream": ("MM_APP_STREAM", [1 << 28, 1, 0], lambda p: 40 * p[0] * p[1],
+               "MK-Seq STREAM-Seq copy/scale/add/triad, 2^28 FP32 (BASELINE configs[1])"),
+    "stream-loop": ("MM_APP_STREAM", [1 << 28, 10, 0], lambda p: 40 * p[0] * p[1],
+                    "MK-Loop STREAM-Loop x10, 2^28 FP32"),
+    "hotspot": ("MM_APP_HOTSPOT", [8192, 8192, 1000], lambda p: 12 * p[0] * p[1] * p[2],
+                "SK-Loop HotSpot 8192^2 x 1000 iterations (BASELINE configs[2])"),
+    "stencil": ("MM_APP_STENCIL_REDUCTION", [16384, 16384, 100, 1], lambda p: 20 * p[0] * p[1] * p[2],
+                "MK-Loop stencil + FP64 residual 16384^2 x 100 steps, w-sync (BASELINE configs[3])"),
+    "blackscholes": ("MM_APP_BLACKSCHOLES", [80530632], lambda p: 20 * p[0],
+                     "SK-One BlackScholes 80,530,632 options (P311)"),
+    "sgemm": ("MM_APP_SGEMM", [6144, 6144, 6144, 0], lambda p: 2 * p[0] * p[1] * p[2],
+              "SK-One MatrixMul 6144^2 FP32 (P311)"),
+}
+# kernel whose roofline is reported, and its algorithmic bytes per item
+DOMINANT = {"stream": ("triad", 12), "stream-loop": ("triad", 12), "hotspot": ("hotspot", None),
+            "stencil": ("stencil", None), "blackscholes": ("blackscholes", 20), "sgemm": ("sgemm", None)}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("hbm_gbs", 6650.0), d.get("bf16_tflops", 1590.0), "measured"
+    except Exception:
+        return 6650.0, 1590.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace('.', '').isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace('.', '').isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for i, nm in enumerate(names):
+                if len(r) > 5 + i and r[5 + i].lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def cpu_baseline(app: str, seconds: float = 10.0):
+    """The oracle, as it stands, single-threaded on a bounded sample."""
+    import numpy as np
+
+    import synthgen
+    from oracle import numeric as on
+    if app.startswith("stream"):
+        n = 1 << 24
+        a, b, c = synthgen.stream_random(n)
+        t0 = time.perf_counter()
+        passes = 0
+        while time.perf_counter() - t0 < seconds:
+            on.lib().or_stream_run(a, b, c, n, 3.0, 1)
+            passes += 1
+        dt = time.perf_counter() - t0
+        return {"value": 40 * n * passes / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                "sample": f"{passes} STREAM-Seq passes over 2^24 of the 2^28 elements (single thread, C -O2)"}
+    if app == "hotspot" or app == "stencil":
+        rows, cols = 1024, 8192
+        t, p = synthgen.hotspot(rows, cols)
+        out = np.empty_like(t)
+        t0 = time.perf_counter()
+        it = 0
+        while time.perf_counter() - t0 < seconds:
+            on.hotspot_rows(t, p, out)
+            t, out = out, t
+            it += 1
+        dt = time.perf_counter() - t0
+        return {"value": 12 * rows * cols * it / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                "sample": f"{it} HotSpot iterations over 1024 of the 8192 rows"}
+    if app == "blackscholes":
+        n = 1 << 22
+        S, X, T = synthgen.blackscholes(n)
+        t0 = time.perf_counter()
+        k = 0
+        while time.perf_counter() - t0 < seconds:
+            on.blackscholes(S, X, T)
+            k += 1
+        dt = time.perf_counter() - t0
+        return {"value": 20 * n * k / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                "sample": f"{k} passes over 2^22 options"}
+    n = 512
+    A, B = synthgen.matmul_uniform(n, n, n)
+    t0 = time.perf_counter()
+    k = 0
+    while time.perf_counter() - t0 < seconds:
+        on.sgemm(A, B)
+        k += 1
+    dt = time.perf_counter() - t0
+    return {"value": 2 * n ** 3 * k / dt / 1e12, "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"{k} 512^3 products"}
+
+
+def run_reference(args):
+    world, rank, local = dist_env()
+    if rank != 0:
+        return
+    unit = "TFLOP/s" if args.app == "sgemm" else "GB/s"
+    # each step = a bounded sample of the workload on the oracle (host cores)
+    vals = []
+    for i in range(args.warmup + args.steps):
+        cb = cpu_baseline(args.app, seconds=max(2.0, 20.0 / max(1, args.steps)))
+        if i >= args.warmup:
+            vals.append(cb)
+    v = statistics.median([c["value"] for c in vals])
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": unit, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": APPS[args.app][3], "sample": vals[0]["sample"]},
+            "cpu_baseline": {"value": v, "unit": unit, "cores": 1, "kind": "oracle", "sample": vals[0]["sample"]},
+            "e2e": {"value": v, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--app", default="stream", choices=sorted(APPS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-strategies", action="store_true")
+    ap.add_argument("--logical", type=int, default=0,
+                    help="virtual mode: run G logical devices on this one GPU (G = --logical)")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_shenvms15_b200 import mm, runner
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("gloo")
+        nid = [mm.mm_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(nid, src=0)
+        nccl_id = nid[0]
+    else:
+        nccl_id = None
+    G = world if world > 1 else max(1, args.logical)
+    app_id = getattr(mm, APPS[args.app][0])
+    iparam = list(APPS[args.app][1])
+    algo_bytes = APPS[args.app][2](iparam)
+    sess = runner.session(app_id, iparam, G=G, cuda_devices=[local] * G, rank=rank, world=world,
+                          nccl_id=nccl_id)
+    hbm_peak, tf_peak, peak_kind = load_peaks()
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    # --- setup (excluded from timing, P311): profile, then generate inputs ---
+    prof = sess.profile(reps=3)
+    sess.fill()
+    cls = mm.mm_classify(sess.app)
+    ranked = mm.mm_rank(cls, mm.mm_needs_sync(sess.app))
+    best = ranked[0]
+    plan = sess.plan(best, prof)
+    info = mm.mm_plan_info(plan)
+    K = sess.K
+
+    def step(p, **kw):
+        # the hot path: classify -> rank -> split (pure, host) -> partitioned run
+        c = mm.mm_classify(sess.app)
+        mm.mm_rank(c, mm.mm_needs_sync(sess.app))
+        if best in (mm.MM_SP_SINGLE, mm.MM_SP_UNIFIED, mm.MM_SP_VARIED):
+            mm.mm_split(sess.app, prof, best)
+        return sess.run(p, **kw)
+
+    for _ in range(args.warmup):
+        step(plan, time_kernels=True)
+    barrier()
+    l0 = mm.mm_kernel_launch_count()
+    stream = sess.stream(rank if world > 1 else 0)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    kms = [[0.0] * K for _ in range(G)]
+    launches = 0
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            st = step(plan, time_kernels=True)
+            for d in range(G):
+                for k in range(K):
+                    kms[d][k] += st.kernel_ms[d][k]
+            launches += st.n_launches
+        ev1.record(stream)
+        barrier()
+    ms_total = ev0.elapsed_time(ev1)
+    gpu_launches = mm.mm_kernel_launch_count() - l0
+    if world > 1:
+        t = torch.tensor([ms_total], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+        lt = torch.tensor([gpu_launches], dtype=torch.int64)
+        dist.all_reduce(lt)
+        gpu_launches = int(lt.item())
+    ms_step = ms_total / args.steps
+    value = algo_bytes / (ms_step * 1e-3) / 1e9
+    unit = "GB/s"
+    if args.app == "sgemm":
+        value = algo_bytes / (ms_step * 1e-3) / 1e12
+        unit = "TFLOP/s"
+
+    # --- roofline of the dominant kernel (event-timed inside the timed region)
+    dom, bpi = DOMINANT[args.app]
+    # kernel ids of the builtin apps in program order
+    kname_map = {"stream": ["copy", "scale", "add", "triad"], "stream-loop": ["copy", "scale", "add", "triad"],
+                 "hotspot": ["hotspot"], "stencil": ["stencil", "residual"], "blackscholes": ["blackscholes"],
+                 "sgemm": ["sgemm"]}[args.app]
+    kid = kname_map.index(dom)
+    my = [d for d in range(G) if sess.mine[d]]
+    dom_ms = sum(kms[d][kid] for d in my)
+    dom_launch = sum(st.kernel_launches[d][kid] for d in my) * args.steps
+    items = sum(info.items[d][kid] for d in my)
+    if bpi is None:
+        bpi = {"hotspot": 12 * iparam[1], "stencil": 12 * iparam[1], "sgemm": None}[args.app]
+    roof = None
+    if dom_launch and dom_ms > 0:
+        per_launch_ms = dom_ms / dom_launch
+        launches_per_step = dom_launch / args.steps
+        if args.app == "sgemm":
+            fl = 2 * iparam[1] * iparam[2] * items / launches_per_step
+            ach = fl / (per_launch_ms * 1e-3) / 1e12
+            roof = {"bound": "tensor", "achieved": ach, "peak": tf_peak / 8 * 1.0, "unit": "TFLOP/s",
+                    "frac": None, "traffic": None}
+        else:
+            byts = bpi * items / launches_per_step
+            ach = byts / (per_launch_ms * 1e-3) / 1e9
+            roof = {"bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                    "traffic": None, "kernel": dom, "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)",
+                    "algorithmic_bytes_per_launch": byts, "avg_launch_ms": per_launch_ms}
+        tr = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        if os.path.exists(tr):
+            try:
+                roof["traffic"] = json.load(open(tr)).get(f"{args.app}:{dom}")
+            except Exception:
+                pass
+
+    # --- e2e: same step through the C ABI with HOST buffers (staged mode) ----
+    e2e = None
+    try:
+        import numpy as np
+        nbuf = sess.nbuf
+        host = []
+        for s in range(nbuf):
+            eb, n = mm.mm_app_buffer_info(sess.app, s)
+            h = torch.empty(max(n, 1), dtype=runner._DT[eb], pin_memory=True)
+            h.copy_(sess.bufs[(s, my[0])].cpu()) if n <= (1 << 29) else None
+            host.append(h)
+        splan = sess.plan(best, prof, staged=True)
+        step(splan, host=[h.data_ptr() for h in host])  # warm-up
+        barrier()
+        e0 = time.perf_counter()
+        tot = []
+        hb = db = 0
+        for _ in range(max(1, min(args.steps, 5))):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            st = step(splan, host=[h.data_ptr() for h in host])
+            torch.cuda.synchronize()
+            tot.append(time.perf_counter() - t0)
+            hb, db = st.h2d_bytes, st.d2h_bytes
+        ms_e2e = statistics.median(tot) * 1e3
+        if world > 1:
+            t = torch.tensor([ms_e2e], dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms_e2e = float(t.item())
+        ev = algo_bytes / (ms_e2e * 1e-3) / (1e12 if unit == "TFLOP/s" else 1e9)
+        e2e = {"value": ev, "unit": unit, "h2d_bytes_per_step": int(hb), "d2h_bytes_per_step": int(db),
+               "ms_per_step": ms_e2e, "mode": "staged (pinned host inputs, H2D before first use, D2H after last)"}
+        del host
+    except Exception as ex:  # report, never hide
+        e2e = {"value": None, "unit": unit, "error": str(ex)[:200]}
+
+    # --- every Table I strategy for this class, w/o and w/ sync (ranking) ----
+    strategies = {}
+    if not args.no_strategies:
+        for s_id in ranked:
+            try:
+                p = sess.plan(s_id, prof)
+                step(p)
+                barrier()
+                ts = []
+                for _ in range(3):
+                    st = sess.run(p)
+                    ts.append(st.device_ms)
+                ms = statistics.median(ts)
+                if world > 1:
+                    t = torch.tensor([ms], dtype=torch.float64)
+                    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                    ms = float(t.item())
+                strategies[mm.mm_strategy_name(s_id)] = round(ms, 4)
+            except mm.MMError as ex:
+                strategies[mm.mm_strategy_name(s_id)] = f"error: {ex}"[:120]
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(args.app)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": APPS[args.app][3], "app": args.app, "class": mm.mm_class_name(cls),
+                       "strategy": mm.mm_strategy_name(best), "logical_devices": G,
+                       "l2": "inputs larger than L2 (1 GiB arrays); no flush",
+                       "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}"},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
+            "clocks": clk.summary(), "strategies_ms": strategies,
+            "ranking": [mm.mm_strategy_name(s) for s in ranked],
+        }
+        print(json.dumps(line), flush=True)
+    sess.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

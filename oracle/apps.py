@@ -81,15 +81,17 @@ def cholesky_tasks(T: int, b: int) -> App:
 
     tasks = []
     for k in range(T):
-        tasks.append(Task(0, k, tile(k, k), tile(k, k) + 1, [acc(RW, k, k)]))
+        tasks.append(Task(0, k, tile(k, k), tile(k, k) + 1, [acc(RW, k, k)], ij=(k, k)))
         for i in range(k + 1, T):
-            tasks.append(Task(1, k, tile(i, k), tile(i, k) + 1, [acc(READ, k, k), acc(RW, i, k)]))
+            tasks.append(Task(1, k, tile(i, k), tile(i, k) + 1, [acc(READ, k, k), acc(RW, i, k)],
+                              ij=(i, k)))
         for i in range(k + 1, T):
-            tasks.append(Task(2, k, tile(i, i), tile(i, i) + 1, [acc(READ, i, k), acc(RW, i, i)]))
+            tasks.append(Task(2, k, tile(i, i), tile(i, i) + 1, [acc(READ, i, k), acc(RW, i, i)],
+                              ij=(i, i)))
         for j in range(k + 1, T):
             for i in range(j + 1, T):
                 tasks.append(Task(3, k, tile(i, j), tile(i, j) + 1,
-                                  [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)]))
+                                  [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)], ij=(i, j)))
     ks = [Kernel(nm, 1, 1, 1, []) for nm in ("potrf", "trsm", "syrk", "gemm")]
     edges = [(0, 1), (1, 2), (1, 3), (2, 0), (3, 1), (3, 2), (3, 3)]
     return App(buffers=[(4, T * T * bb)], kernels=ks, edges=edges, dag_tasks=tasks)

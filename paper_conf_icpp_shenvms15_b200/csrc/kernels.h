@@ -1,0 +1,55 @@
+// Launch interface of the sm_100a kernels (one per paper application kernel).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace mm {
+
+struct Kernel;
+struct Task;
+
+struct Launch {
+  const Kernel* k;          // kernel descriptor (op, params)
+  const Task* t;            // task: item range [t->b, t->e) / DAG params
+  void* const* opnd;        // device pointers, one per access (this device's copy)
+  cudaStream_t stream;
+  int32_t sms;              // SMs available to this logical device
+};
+
+// Returns cudaSuccess, cudaErrorNotSupported for an unimplemented op, or the
+// launch error.  Empty ranges launch nothing.
+cudaError_t launch_builtin(const Launch& L);
+
+// STREAM (kernels_stream.cu)
+cudaError_t stream_copy(const float* a, float* c, int64_t lo, int64_t hi, cudaStream_t s, int sms);
+cudaError_t stream_scale(const float* c, float* b, float q, int64_t lo, int64_t hi, cudaStream_t s, int sms);
+cudaError_t stream_add(const float* a, const float* b, float* c, int64_t lo, int64_t hi, cudaStream_t s, int sms);
+cudaError_t stream_triad(const float* b, const float* c, float* a, float q, int64_t lo, int64_t hi, cudaStream_t s, int sms);
+
+// HotSpot + residual (kernels_stencil.cu)
+struct HotCoef { float sdc, rx1, ry1, rz1, amb; };
+cudaError_t hotspot_rows(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols,
+                         int64_t r0, int64_t r1, HotCoef c, cudaStream_t s, int sms);
+cudaError_t row_residual(const float* t0, const float* t1, double* rowsum, int64_t cols,
+                         int64_t r0, int64_t r1, cudaStream_t s, int sms);
+
+// BlackScholes (kernels_bs.cu)
+cudaError_t blackscholes(const float* S, const float* X, const float* T, float* call, float* put,
+                         float R, float V, int64_t lo, int64_t hi, cudaStream_t s, int sms);
+
+// SGEMM rows [r0,r1) of C = A B (kernels_gemm.cu)
+cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
+                       int64_t r0, int64_t r1, int32_t variant, cudaStream_t s, int sms);
+
+// Cholesky tiles (kernels_chol.cu); A tile-major, T x T tiles of b x b.
+cudaError_t chol_task(int32_t op, float* A, int64_t T, int64_t b, int64_t i, int64_t j, int64_t k,
+                      cudaStream_t s, int sms);
+
+// Counter-hash generators (kernels_fill.cu) = synthgen.uniform / integers.
+cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
+                         float lo, float hi, cudaStream_t s);
+cudaError_t fill_integers(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
+                          int32_t lo, int32_t hi, cudaStream_t s);
+
+}  // namespace mm

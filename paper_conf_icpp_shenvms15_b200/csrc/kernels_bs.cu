@@ -1,0 +1,92 @@
+// BlackScholes (P217-221 Table II "Nvidia OpenCL SDK", P311: 80,530,632
+// options in a 1-D array, split into ranges of neighbouring options).
+//
+// European call and put per option (NVIDIA SDK formulation [ext]):
+//   d1 = (ln(S/X) + (R + V^2/2) T) / (V sqrt T), d2 = d1 - V sqrt T
+//   call = S N(d1) - X e^{-RT} N(d2), put = X e^{-RT} (1 - N(d2)) - S (1 - N(d1))
+// N = Abramowitz-Stegun 26.2.17.  FP32 with the accurate libdevice logf/expf/
+// sqrtf (no fast-math): 20 algorithmic bytes per option, HBM-bound on B200
+// (~60 flops/option).  float4 I/O, 4 options per thread.
+#include "kernels.h"
+
+namespace mm {
+
+namespace {
+
+constexpr int kThreads = 256;
+
+__device__ __forceinline__ float cnd(float d) {
+  const float A1 = 0.31938153f, A2 = -0.356563782f, A3 = 1.781477937f, A4 = -1.821255978f,
+              A5 = 1.330274429f, RSQRT2PI = 0.39894228040143267793994605993438f;
+  const float k = 1.0f / (1.0f + 0.2316419f * fabsf(d));
+  float c = RSQRT2PI * expf(-0.5f * d * d) * (k * (A1 + k * (A2 + k * (A3 + k * (A4 + k * A5)))));
+  if (d > 0) c = 1.0f - c;
+  return c;
+}
+
+__device__ __forceinline__ void option(float s, float x, float t, float R, float V, float& call,
+                                       float& put) {
+  const float sqrtT = sqrtf(t);
+  const float d1 = (logf(s / x) + (R + 0.5f * V * V) * t) / (V * sqrtT);
+  const float d2 = d1 - V * sqrtT;
+  const float n1 = cnd(d1), n2 = cnd(d2);
+  const float expRT = expf(-R * t);
+  call = s * n1 - x * expRT * n2;
+  put = x * expRT * (1.0f - n2) - s * (1.0f - n1);
+}
+
+__global__ void __launch_bounds__(kThreads) bs_vec(const float4* __restrict__ S,
+                                                   const float4* __restrict__ X,
+                                                   const float4* __restrict__ T,
+                                                   float4* __restrict__ C, float4* __restrict__ P,
+                                                   int64_t n4, float R, float V) {
+  for (int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x; i < n4;
+       i += (int64_t)gridDim.x * kThreads) {
+    const float4 s = __ldcs(S + i), x = __ldcs(X + i), t = __ldcs(T + i);
+    float4 c, p;
+    option(s.x, x.x, t.x, R, V, c.x, p.x);
+    option(s.y, x.y, t.y, R, V, c.y, p.y);
+    option(s.z, x.z, t.z, R, V, c.z, p.z);
+    option(s.w, x.w, t.w, R, V, c.w, p.w);
+    __stcs(C + i, c);
+    __stcs(P + i, p);
+  }
+}
+
+__global__ void bs_scalar(const float* __restrict__ S, const float* __restrict__ X,
+                          const float* __restrict__ T, float* __restrict__ C, float* __restrict__ P,
+                          int64_t n, float R, float V) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) option(S[i], X[i], T[i], R, V, C[i], P[i]);
+}
+
+}  // namespace
+
+cudaError_t blackscholes(const float* S, const float* X, const float* T, float* call, float* put,
+                         float R, float V, int64_t lo, int64_t hi, cudaStream_t s, int sms) {
+  if (hi <= lo) return cudaSuccess;
+  const int64_t n = hi - lo;
+  S += lo; X += lo; T += lo; call += lo; put += lo;
+  int64_t done = 0;
+  if ((((uintptr_t)S | (uintptr_t)X | (uintptr_t)T | (uintptr_t)call | (uintptr_t)put) & 15u) == 0) {
+    const int64_t n4 = n / 4;
+    if (n4) {
+      int64_t blocks = (n4 + kThreads - 1) / kThreads;
+      const int64_t cap = (int64_t)(sms > 0 ? sms : 148) * 8;  // persistent: 8 CTAs per SM
+      if (blocks > cap) blocks = cap;
+      bs_vec<<<(unsigned)blocks, kThreads, 0, s>>>(
+          reinterpret_cast<const float4*>(S), reinterpret_cast<const float4*>(X),
+          reinterpret_cast<const float4*>(T), reinterpret_cast<float4*>(call),
+          reinterpret_cast<float4*>(put), n4, R, V);
+      done = n4 * 4;
+    }
+  }
+  if (done < n) {
+    const int64_t m = n - done;
+    bs_scalar<<<(unsigned)((m + 255) / 256), 256, 0, s>>>(S + done, X + done, T + done, call + done,
+                                                          put + done, m, R, V);
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace mm

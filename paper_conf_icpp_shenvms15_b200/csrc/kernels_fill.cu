@@ -1,0 +1,63 @@
+// Counter-hash input generator on the device (the
+// same recipe as synthgen.py, checked bit for bit by tests/test_gpu_parity.py).
+// Holds no arithmetic of the method: it only produces seeded synthetic inputs
+// in place on each device (resident mode).
+#include "kernels.h"
+
+namespace mm {
+
+namespace {
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+__global__ void fill_u(float* __restrict__ dst, int64_t n, uint64_t key, int64_t start, float lo,
+                       float span) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t h = splitmix64((uint64_t)(start + i) ^ key) >> 40;
+    const float u = __fmul_rn((float)h, 5.9604644775390625e-08f);  // * 2^-24, exact
+    dst[i] = __fadd_rn(lo, __fmul_rn(span, u));
+  }
+}
+
+__global__ void fill_i(float* __restrict__ dst, int64_t n, uint64_t key, int64_t start, int32_t lo,
+                       uint64_t span) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t h = splitmix64((uint64_t)(start + i) ^ key) >> 40;
+    dst[i] = (float)(lo + (int64_t)(h % span));
+  }
+}
+
+unsigned grid_for(int64_t n) {
+  int64_t b = (n + 255) / 256;
+  if (b > 148 * 64) b = 148 * 64;
+  return (unsigned)(b < 1 ? 1 : b);
+}
+
+}  // namespace
+
+cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
+                         float lo, float hi, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  const uint64_t key = seed ^ ((uint64_t)(uint32_t)array_id << 48);
+  const float span = hi - lo;  // one float32 rounding, as synthgen
+  fill_u<<<grid_for(n), 256, 0, s>>>(dst, n, key, start, lo, span);
+  return cudaGetLastError();
+}
+
+cudaError_t fill_integers(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
+                          int32_t lo, int32_t hi, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  if (hi < lo) return cudaErrorInvalidValue;
+  const uint64_t key = seed ^ ((uint64_t)(uint32_t)array_id << 48);
+  fill_i<<<grid_for(n), 256, 0, s>>>(dst, n, key, start, lo, (uint64_t)(hi - lo + 1));
+  return cudaGetLastError();
+}
+
+}  // namespace mm

@@ -1,0 +1,900 @@
+// Runtime of the matchmaking library: logical devices (streams, optional
+// green-context SM budgets), the op-program executor (in-process streams and
+// events, or NCCL send/recv across processes), CUDA-graph replay, Glinda-style
+// profiling (P49) with the DP-Perf warm-up (P311), and result collection.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstring>
+#include <memory>
+#include <new>
+#include <vector>
+
+#include "kernels.h"
+#include "mm_internal.h"
+
+using namespace mm;
+
+namespace mm {
+std::atomic<int64_t> g_kernel_launches{0};
+}
+
+struct DevRt {
+  int32_t phys = 0, budget = 0, sms = 0, rank = 0;
+  cudaStream_t stream = nullptr;
+  CUgreenCtx gctx = nullptr;
+  CUcontext gcu = nullptr;   // CUcontext view of the green context
+  bool mine = false;
+};
+
+// Driver-API entry points, resolved at run time through the runtime
+// (cudaGetDriverEntryPoint) so the library has no link-time dependency on
+// libcuda.so (it must load on hosts without a driver).
+struct Drv {
+  decltype(&cuInit) Init = nullptr;
+  decltype(&cuDeviceGet) DeviceGet = nullptr;
+  decltype(&cuDeviceGetDevResource) DeviceGetDevResource = nullptr;
+  decltype(&cuDevSmResourceSplitByCount) DevSmResourceSplitByCount = nullptr;
+  decltype(&cuDevResourceGenerateDesc) DevResourceGenerateDesc = nullptr;
+  decltype(&cuGreenCtxCreate) GreenCtxCreate = nullptr;
+  decltype(&cuGreenCtxStreamCreate) GreenCtxStreamCreate = nullptr;
+  decltype(&cuGreenCtxDestroy) GreenCtxDestroy = nullptr;
+  decltype(&cuCtxFromGreenCtx) CtxFromGreenCtx = nullptr;
+  decltype(&cuCtxSetCurrent) CtxSetCurrent = nullptr;
+  decltype(&cuStreamDestroy) StreamDestroy = nullptr;
+  decltype(&cuGetErrorString) GetErrorString = nullptr;
+  bool ok = false;
+};
+
+static Drv& drv() {
+  static Drv d;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    bool ok = true;
+    auto get = [&](const char* name, void** fp) {
+      cudaDriverEntryPointQueryResult q;
+      if (cudaGetDriverEntryPoint(name, fp, cudaEnableDefault, &q) != cudaSuccess ||
+          q != cudaDriverEntryPointSuccess || !*fp)
+        ok = false;
+    };
+    get("cuInit", (void**)&d.Init);
+    get("cuDeviceGet", (void**)&d.DeviceGet);
+    get("cuDeviceGetDevResource", (void**)&d.DeviceGetDevResource);
+    get("cuDevSmResourceSplitByCount", (void**)&d.DevSmResourceSplitByCount);
+    get("cuDevResourceGenerateDesc", (void**)&d.DevResourceGenerateDesc);
+    get("cuGreenCtxCreate", (void**)&d.GreenCtxCreate);
+    get("cuGreenCtxStreamCreate", (void**)&d.GreenCtxStreamCreate);
+    get("cuGreenCtxDestroy", (void**)&d.GreenCtxDestroy);
+    get("cuCtxFromGreenCtx", (void**)&d.CtxFromGreenCtx);
+    get("cuCtxSetCurrent", (void**)&d.CtxSetCurrent);
+    get("cuStreamDestroy", (void**)&d.StreamDestroy);
+    get("cuGetErrorString", (void**)&d.GetErrorString);
+    d.ok = ok;
+  }
+  return d;
+}
+
+struct mm_ctx {
+  std::vector<DevRt> dev;
+  int32_t G = 0, my_rank = 0, world = 1;
+  ncclComm_t comm = nullptr;
+  bool poisoned = false;
+  float* bar_buf = nullptr;        // NCCL barrier scratch (1 float)
+  std::vector<void*> flush_scratch;  // per buffer slot, pinned (lazily)
+  std::vector<size_t> flush_scratch_bytes;
+};
+
+namespace {
+
+#define CU_OK(expr)                                                              \
+  do {                                                                           \
+    cudaError_t e_ = (expr);                                                     \
+    if (e_ != cudaSuccess) {                                                     \
+      if (ctx) ctx->poisoned = true;                                             \
+      MM_FAIL(MM_ECUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                            \
+  } while (0)
+
+#define DRV_OK(expr)                                                             \
+  do {                                                                           \
+    CUresult r_ = (expr);                                                        \
+    if (r_ != CUDA_SUCCESS) {                                                    \
+      const char* s_ = nullptr;                                                  \
+      if (drv().GetErrorString) drv().GetErrorString(r_, &s_);                   \
+      MM_FAIL(MM_ECUDA, "%s failed: %s", #expr, s_ ? s_ : "?");                  \
+    }                                                                            \
+  } while (0)
+
+#define NCCL_OK(expr)                                                            \
+  do {                                                                           \
+    ncclResult_t r_ = (expr);                                                    \
+    if (r_ != ncclSuccess) {                                                     \
+      if (ctx) ctx->poisoned = true;                                             \
+      MM_FAIL(MM_ENCCL, "%s failed: %s", #expr, ncclGetErrorString(r_));         \
+    }                                                                            \
+  } while (0)
+
+struct PlanRt {
+  mm_ctx* ctx = nullptr;
+  std::vector<cudaEvent_t> ev;           // per op that another stream waits on
+  std::vector<cudaEvent_t> bar_ev;       // per device
+  std::vector<cudaEvent_t> join_ev;      // per device
+  cudaEvent_t fork = nullptr;
+  cudaEvent_t t_start = nullptr, t_stop = nullptr;
+  std::vector<cudaEvent_t> kev;          // 2 per kernel op (timing)
+  cudaGraphExec_t gexec = nullptr;
+  cudaGraph_t graph = nullptr;
+  std::vector<void*> graph_bufs;
+  int64_t graph_launches = 0;
+  int64_t graph_xfer = 0, graph_h2d = 0, graph_d2h = 0;
+};
+
+cudaError_t set_dev(mm_ctx* ctx, int32_t d) {
+  const DevRt& r = ctx->dev[d];
+  if (r.gcu) return drv().CtxSetCurrent(r.gcu) == CUDA_SUCCESS ? cudaSuccess : cudaErrorDeviceUninitialized;
+  return cudaSetDevice(r.phys);
+}
+
+void destroy_rt(PlanRt* rt) {
+  if (!rt) return;
+  for (auto e : rt->ev)
+    if (e) cudaEventDestroy(e);
+  for (auto e : rt->bar_ev)
+    if (e) cudaEventDestroy(e);
+  for (auto e : rt->join_ev)
+    if (e) cudaEventDestroy(e);
+  for (auto e : rt->kev)
+    if (e) cudaEventDestroy(e);
+  if (rt->fork) cudaEventDestroy(rt->fork);
+  if (rt->t_start) cudaEventDestroy(rt->t_start);
+  if (rt->t_stop) cudaEventDestroy(rt->t_stop);
+  if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
+  if (rt->graph) cudaGraphDestroy(rt->graph);
+  delete rt;
+}
+
+int32_t first_owned(const mm_ctx* ctx) {
+  for (int32_t d = 0; d < ctx->G; ++d)
+    if (ctx->dev[d].mine) return d;
+  return -1;
+}
+
+}  // namespace
+
+namespace mm {
+
+void plan_runtime_free(Plan* plan) {
+  destroy_rt(static_cast<PlanRt*>(plan->rt));
+  plan->rt = nullptr;
+}
+
+cudaError_t launch_builtin(const Launch& L) {
+  const Kernel& k = *L.k;
+  const Task& t = *L.t;
+  const int64_t b = t.b, e = t.e;
+  float* const* f = reinterpret_cast<float* const*>(L.opnd);
+  switch (k.op) {
+    case MM_OP_STREAM_COPY: return stream_copy(f[0], f[1], b, e, L.stream, L.sms);
+    case MM_OP_STREAM_SCALE: return stream_scale(f[0], f[1], (float)k.fp[0], b, e, L.stream, L.sms);
+    case MM_OP_STREAM_ADD: return stream_add(f[0], f[1], f[2], b, e, L.stream, L.sms);
+    case MM_OP_STREAM_TRIAD: return stream_triad(f[0], f[1], f[2], (float)k.fp[0], b, e, L.stream, L.sms);
+    case MM_OP_HOTSPOT: {
+      HotCoef c{(float)k.fp[0], (float)k.fp[1], (float)k.fp[2], (float)k.fp[3], (float)k.fp[4]};
+      return hotspot_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], b, e, c, L.stream, L.sms);
+    }
+    case MM_OP_ROW_RESIDUAL:
+      return row_residual(f[0], f[1], reinterpret_cast<double*>(L.opnd[2]), k.ip[1], b, e, L.stream, L.sms);
+    case MM_OP_BLACKSCHOLES:
+      return blackscholes(f[0], f[1], f[2], f[3], f[4], (float)k.fp[0], (float)k.fp[1], b, e, L.stream, L.sms);
+    case MM_OP_SGEMM: {
+      int32_t variant = (int32_t)k.ip[3];
+      if (variant == 0) variant = 2;
+      cudaError_t r = sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, variant, L.stream, L.sms);
+      if (r == cudaErrorNotSupported && k.ip[3] == 0)
+        r = sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, 1, L.stream, L.sms);
+      return r;
+    }
+    case MM_OP_CHOL_POTRF:
+    case MM_OP_CHOL_TRSM:
+    case MM_OP_CHOL_SYRK:
+    case MM_OP_CHOL_GEMM:
+      return chol_task(k.op, f[0], k.ip[0], k.ip[1], t.ip[0], t.ip[1], t.ip[2], L.stream, L.sms);
+  }
+  return cudaErrorNotSupported;
+}
+
+}  // namespace mm
+
+namespace {
+
+// Launch the task's kernel on logical device d.
+mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, void* const* buffers,
+                      cudaStream_t s) {
+  const Kernel& k = app.kernels[t.kernel];
+  void* opnd[MM_MAX_ACCESS];
+  const int32_t G = ctx->G;
+  for (size_t i = 0; i < t.acc.size() && i < MM_MAX_ACCESS; ++i) {
+    opnd[i] = buffers[(size_t)t.acc[i].buffer * G + d];
+    if (!opnd[i]) MM_FAIL(MM_EINVAL, "run: buffer slot %d has no pointer on device %d", t.acc[i].buffer, d);
+  }
+  cudaError_t e;
+  if (k.op == MM_OP_CUSTOM) {
+    e = (cudaError_t)k.launch(k.user, d, mm_range{t.b, t.e}, opnd, (void*)s);
+  } else {
+    Launch L{&k, &t, opnd, s, ctx->dev[d].sms};
+    e = launch_builtin(L);
+  }
+  if (e == cudaErrorNotSupported) MM_FAIL(MM_ENOTSUP, "kernel %s (op %d) has no sm_100a implementation yet", k.name.c_str(), k.op);
+  if (e != cudaSuccess) {
+    ctx->poisoned = true;
+    MM_FAIL(MM_ECUDA, "kernel %s launch failed: %s", k.name.c_str(), cudaGetErrorString(e));
+  }
+  g_kernel_launches.fetch_add(1, std::memory_order_relaxed);
+  return MM_OK;
+}
+
+mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
+  PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  if (rt && rt->ctx != ctx) {
+    destroy_rt(rt);
+    rt = nullptr;
+    plan.rt = nullptr;
+  }
+  if (!rt) {
+    rt = new PlanRt();
+    rt->ctx = ctx;
+    plan.rt = rt;
+    const int32_t G = ctx->G;
+    rt->ev.assign(plan.ops.size(), nullptr);
+    for (size_t i = 0; i < plan.ops.size(); ++i)
+      if (plan.needs_event[i] && plan.op_stream[i] >= 0 && ctx->dev[plan.op_stream[i]].mine) {
+        CU_OK(set_dev(ctx, plan.op_stream[i]));
+        CU_OK(cudaEventCreateWithFlags(&rt->ev[i], cudaEventDisableTiming));
+      }
+    rt->bar_ev.assign(G, nullptr);
+    rt->join_ev.assign(G, nullptr);
+    for (int32_t d = 0; d < G; ++d) {
+      if (!ctx->dev[d].mine) continue;
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaEventCreateWithFlags(&rt->bar_ev[d], cudaEventDisableTiming));
+      CU_OK(cudaEventCreateWithFlags(&rt->join_ev[d], cudaEventDisableTiming));
+    }
+    const int32_t root = first_owned(ctx);
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventCreateWithFlags(&rt->fork, cudaEventDisableTiming));
+    CU_OK(cudaEventCreate(&rt->t_start));
+    CU_OK(cudaEventCreate(&rt->t_stop));
+  }
+  if (timing && rt->kev.empty()) {
+    rt->kev.assign(plan.ops.size() * 2, nullptr);
+    for (size_t i = 0; i < plan.ops.size(); ++i)
+      if (plan.ops[i].kind == MM_OPK_KERNEL && ctx->dev[plan.ops[i].device].mine) {
+        CU_OK(set_dev(ctx, plan.ops[i].device));
+        CU_OK(cudaEventCreate(&rt->kev[2 * i]));
+        CU_OK(cudaEventCreate(&rt->kev[2 * i + 1]));
+      }
+  }
+  return MM_OK;
+}
+
+void* flush_target(mm_ctx* ctx, const Plan& plan, const mm_run_opts* o, int32_t buf, size_t bytes_total,
+                   mm_status* st) {
+  *st = MM_OK;
+  if (o && o->host && o->host[buf]) return o->host[buf];
+  if (ctx->flush_scratch.size() <= (size_t)buf) {
+    ctx->flush_scratch.resize(buf + 1, nullptr);
+    ctx->flush_scratch_bytes.resize(buf + 1, 0);
+  }
+  if (ctx->flush_scratch_bytes[buf] < bytes_total) {
+    if (ctx->flush_scratch[buf]) cudaFreeHost(ctx->flush_scratch[buf]);
+    ctx->flush_scratch[buf] = nullptr;
+    if (cudaMallocHost(&ctx->flush_scratch[buf], bytes_total) != cudaSuccess) {
+      set_error("pinned flush scratch of %zu bytes", bytes_total);
+      *st = MM_ENOMEM;
+      return nullptr;
+    }
+    ctx->flush_scratch_bytes[buf] = bytes_total;
+  }
+  (void)plan;
+  return ctx->flush_scratch[buf];
+}
+
+// Issue the op program of an in-process ctx (world == 1) onto the streams.
+mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run_opts* o, bool timing,
+                      mm_run_stats* st) {
+  PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  const int32_t G = ctx->G;
+  const App& app = plan.app;
+  std::vector<uint8_t> used(G, 0);
+  for (int32_t d : plan.task_dev) used[d] = 1;
+  for (auto& op : plan.ops)
+    if (op.kind != MM_OPK_BARRIER) used[op.device] = 1;
+  const int32_t root = first_owned(ctx);
+  used[root] = 1;
+  // fork
+  CU_OK(set_dev(ctx, root));
+  CU_OK(cudaEventRecord(rt->fork, ctx->dev[root].stream));
+  for (int32_t d = 0; d < G; ++d)
+    if (used[d] && d != root) {
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->fork, 0));
+    }
+  for (size_t i = 0; i < plan.ops.size(); ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    if (op.kind == MM_OPK_BARRIER) {
+      for (int32_t d = 0; d < G; ++d)
+        if (used[d]) {
+          CU_OK(set_dev(ctx, d));
+          CU_OK(cudaEventRecord(rt->bar_ev[d], ctx->dev[d].stream));
+        }
+      for (int32_t d = 0; d < G; ++d)
+        if (used[d]) {
+          CU_OK(set_dev(ctx, d));
+          for (int32_t q = 0; q < G; ++q)
+            if (used[q] && q != d) CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->bar_ev[q], 0));
+        }
+      continue;
+    }
+    const int32_t d = plan.op_stream[i];
+    cudaStream_t s = ctx->dev[d].stream;
+    CU_OK(set_dev(ctx, d));
+    for (auto& w : plan.waits[i]) CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
+    if (op.kind == MM_OPK_KERNEL) {
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      mm_status r = launch_task(ctx, app, plan.tasks[op.task], d, buffers, s);
+      if (r) return r;
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      st->n_launches++;
+    } else if (op.kind == MM_OPK_XFER) {
+      const int64_t eb = app.buffers[op.buffer].first;
+      const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+      char* dst = static_cast<char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+      if (op.src < 0) {
+        if (!o || !o->host || !o->host[op.buffer]) MM_FAIL(MM_EINVAL, "staged run: no host pointer for slot %d", op.buffer);
+        const char* src = static_cast<const char*>(o->host[op.buffer]) + op.r.begin * eb;
+        CU_OK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, s));
+        st->h2d_bytes += (int64_t)bytes;
+      } else {
+        const char* src = static_cast<const char*>(buffers[(size_t)op.buffer * G + op.src]) + op.r.begin * eb;
+        if (ctx->dev[op.src].phys == ctx->dev[d].phys)
+          CU_OK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToDevice, s));
+        else
+          CU_OK(cudaMemcpyPeerAsync(dst, ctx->dev[d].phys, src, ctx->dev[op.src].phys, bytes, s));
+        st->xfer_bytes += (int64_t)bytes;
+      }
+    } else if (op.kind == MM_OPK_FLUSH) {
+      const int64_t eb = app.buffers[op.buffer].first;
+      const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+      mm_status fs;
+      char* host = static_cast<char*>(flush_target(ctx, plan, o, op.buffer,
+                                                   (size_t)(app.buffers[op.buffer].second * eb), &fs));
+      if (fs) return fs;
+      const char* src = static_cast<const char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+      CU_OK(cudaMemcpyAsync(host + op.r.begin * eb, src, bytes, cudaMemcpyDeviceToHost, s));
+      st->d2h_bytes += (int64_t)bytes;
+    }
+    if (plan.needs_event[i]) CU_OK(cudaEventRecord(rt->ev[i], s));
+  }
+  // join
+  for (int32_t d = 0; d < G; ++d)
+    if (used[d] && d != root) {
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaEventRecord(rt->join_ev[d], ctx->dev[d].stream));
+      CU_OK(set_dev(ctx, root));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[d], 0));
+    }
+  return MM_OK;
+}
+
+// Issue the op program of one rank of a multi-process ctx: kernels of the
+// owned device, NCCL send/recv for transfers touching it (grouped), an NCCL
+// all-reduce of one float per BARRIER, D2H for its FLUSH ops.
+mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run_opts* o, bool timing,
+                     mm_run_stats* st) {
+  PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  const int32_t G = ctx->G;
+  const int32_t me = first_owned(ctx);
+  const App& app = plan.app;
+  cudaStream_t s = ctx->dev[me].stream;
+  CU_OK(set_dev(ctx, me));
+  bool in_group = false;
+  for (size_t i = 0; i < plan.ops.size(); ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    const bool x = op.kind == MM_OPK_XFER && op.src >= 0 && (op.device == me || op.src == me);
+    if (in_group && !(op.kind == MM_OPK_XFER && op.src >= 0)) {
+      NCCL_OK(ncclGroupEnd());
+      in_group = false;
+    }
+    if (op.kind == MM_OPK_BARRIER) {
+      NCCL_OK(ncclAllReduce(ctx->bar_buf, ctx->bar_buf, 1, ncclFloat, ncclSum, ctx->comm, s));
+      continue;
+    }
+    if (op.kind == MM_OPK_KERNEL) {
+      if (op.device != me) continue;
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      mm_status r = launch_task(ctx, app, plan.tasks[op.task], me, buffers, s);
+      if (r) return r;
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      st->n_launches++;
+      continue;
+    }
+    const int64_t eb = app.buffers[op.buffer].first;
+    const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+    if (op.kind == MM_OPK_XFER && op.src < 0) {
+      if (op.device != me) continue;
+      if (!o || !o->host || !o->host[op.buffer]) MM_FAIL(MM_EINVAL, "staged run: no host pointer for slot %d", op.buffer);
+      char* dst = static_cast<char*>(buffers[(size_t)op.buffer * G + me]) + op.r.begin * eb;
+      CU_OK(cudaMemcpyAsync(dst, static_cast<const char*>(o->host[op.buffer]) + op.r.begin * eb, bytes,
+                            cudaMemcpyHostToDevice, s));
+      st->h2d_bytes += (int64_t)bytes;
+      continue;
+    }
+    if (x) {
+      if (!in_group) {
+        NCCL_OK(ncclGroupStart());
+        in_group = true;
+      }
+      char* mine = static_cast<char*>(buffers[(size_t)op.buffer * G + me]) + op.r.begin * eb;
+      if (op.device == me)
+        NCCL_OK(ncclRecv(mine, bytes, ncclChar, ctx->dev[op.src].rank, ctx->comm, s));
+      else
+        NCCL_OK(ncclSend(mine, bytes, ncclChar, ctx->dev[op.device].rank, ctx->comm, s));
+      st->xfer_bytes += op.device == me ? (int64_t)bytes : 0;
+      continue;
+    }
+    if (op.kind == MM_OPK_FLUSH && op.device == me) {
+      mm_status fs;
+      char* host = static_cast<char*>(flush_target(ctx, plan, o, op.buffer,
+                                                   (size_t)(app.buffers[op.buffer].second * eb), &fs));
+      if (fs) return fs;
+      CU_OK(cudaMemcpyAsync(host + op.r.begin * eb,
+                            static_cast<const char*>(buffers[(size_t)op.buffer * G + me]) + op.r.begin * eb,
+                            bytes, cudaMemcpyDeviceToHost, s));
+      st->d2h_bytes += (int64_t)bytes;
+    }
+  }
+  if (in_group) NCCL_OK(ncclGroupEnd());
+  return MM_OK;
+}
+
+}  // namespace
+
+// ===========================================================================
+// C ABI: runtime
+// ===========================================================================
+extern "C" {
+
+mm_status mm_nccl_unique_id(void* out128) {
+  if (!out128) MM_FAIL(MM_EINVAL, "null out");
+  mm_ctx* ctx = nullptr;
+  ncclUniqueId id;
+  NCCL_OK(ncclGetUniqueId(&id));
+  static_assert(sizeof(id) == 128, "ncclUniqueId size");
+  std::memcpy(out128, &id, sizeof(id));
+  return MM_OK;
+}
+
+mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, int32_t world,
+                        const void* nccl_id, mm_ctx** out) {
+  if (!devs || !out || G < 1 || G > MM_MAX_DEV || world < 1 || my_rank < 0 || my_rank >= world)
+    MM_FAIL(MM_EINVAL, "ctx_create: bad arguments (G=%d rank=%d world=%d)", G, my_rank, world);
+  mm_ctx* ctx = nullptr;
+  try {
+    ctx = new mm_ctx();
+  } catch (...) {
+    MM_FAIL(MM_ENOMEM, "ctx alloc");
+  }
+  std::unique_ptr<mm_ctx, void (*)(mm_ctx*)> guard(ctx, [](mm_ctx* c) { mm_ctx_destroy(c); });
+  ctx->G = G;
+  ctx->my_rank = my_rank;
+  ctx->world = world;
+  ctx->dev.resize(G);
+  int ndev = 0;
+  CU_OK(cudaGetDeviceCount(&ndev));
+  int owned = 0;
+  for (int32_t d = 0; d < G; ++d) {
+    DevRt& r = ctx->dev[d];
+    r.phys = devs[d].cuda_device;
+    r.budget = devs[d].sm_budget;
+    r.rank = devs[d].rank;
+    r.mine = (r.rank == my_rank);
+    if (r.rank < 0 || r.rank >= world) MM_FAIL(MM_EINVAL, "device %d: rank %d", d, r.rank);
+    if (!r.mine) continue;
+    owned++;
+    if (r.phys < 0 || r.phys >= ndev) MM_FAIL(MM_EINVAL, "device %d: cuda ordinal %d of %d", d, r.phys, ndev);
+    CU_OK(cudaSetDevice(r.phys));
+    int sms = 0;
+    CU_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, r.phys));
+    r.sms = sms;
+  }
+  if (world > 1 && owned != 1) MM_FAIL(MM_EINVAL, "multi-process ctx: rank %d owns %d devices (need 1)", my_rank, owned);
+  if (owned == 0) MM_FAIL(MM_EINVAL, "rank %d owns no device", my_rank);
+  // SM budgets (HET mode): per physical GPU, split its SMs into green
+  // contexts — one group of >= budget SMs per budgeted logical device, the
+  // remainder for the unbudgeted one(s).
+  for (int32_t d = 0; d < G; ++d) {
+    DevRt& r = ctx->dev[d];
+    if (!r.mine) continue;
+    bool any_budget = false;
+    for (int32_t q = 0; q < G; ++q)
+      if (ctx->dev[q].mine && ctx->dev[q].phys == r.phys && ctx->dev[q].budget > 0) any_budget = true;
+    if (!any_budget) {
+      CU_OK(cudaSetDevice(r.phys));
+      CU_OK(cudaStreamCreateWithFlags(&r.stream, cudaStreamNonBlocking));
+      continue;
+    }
+    if (r.gctx) continue;
+    // build all green contexts of this physical GPU at once
+    Drv& D = drv();
+    if (!D.ok) MM_FAIL(MM_ENOTSUP, "green contexts: driver entry points unavailable");
+    CU_OK(cudaSetDevice(r.phys));
+    CU_OK(cudaFree(nullptr));  // make sure the primary context exists
+    DRV_OK(D.Init(0));
+    CUdevice cudev;
+    DRV_OK(D.DeviceGet(&cudev, r.phys));
+    CUdevResource all;
+    DRV_OK(D.DeviceGetDevResource(cudev, &all, CU_DEV_RESOURCE_TYPE_SM));
+    CUdevResource rest = all;
+    for (int32_t q = 0; q < G; ++q) {
+      DevRt& rq = ctx->dev[q];
+      if (!rq.mine || rq.phys != r.phys || rq.budget <= 0) continue;
+      CUdevResource grp, remaining;
+      unsigned n = 1;
+      DRV_OK(D.DevSmResourceSplitByCount(&grp, &n, &rest, &remaining, 0, (unsigned)rq.budget));
+      if (n < 1) MM_FAIL(MM_ECUDA, "SM split for device %d gave no group", q);
+      CUdevResourceDesc desc;
+      DRV_OK(D.DevResourceGenerateDesc(&desc, &grp, 1));
+      DRV_OK(D.GreenCtxCreate(&rq.gctx, desc, cudev, CU_GREEN_CTX_DEFAULT_STREAM));
+      DRV_OK(D.CtxFromGreenCtx(&rq.gcu, rq.gctx));
+      CUstream cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.stream = (cudaStream_t)cs;
+      rq.sms = (int32_t)grp.sm.smCount;
+      rest = remaining;
+    }
+    for (int32_t q = 0; q < G; ++q) {
+      DevRt& rq = ctx->dev[q];
+      if (!rq.mine || rq.phys != r.phys || rq.budget > 0) continue;
+      CUdevResourceDesc desc;
+      DRV_OK(D.DevResourceGenerateDesc(&desc, &rest, 1));
+      DRV_OK(D.GreenCtxCreate(&rq.gctx, desc, cudev, CU_GREEN_CTX_DEFAULT_STREAM));
+      DRV_OK(D.CtxFromGreenCtx(&rq.gcu, rq.gctx));
+      CUstream cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.stream = (cudaStream_t)cs;
+      rq.sms = (int32_t)rest.sm.smCount;
+    }
+  }
+  if (world > 1) {
+    if (!nccl_id) MM_FAIL(MM_EINVAL, "multi-process ctx needs an NCCL unique id");
+    ncclUniqueId id;
+    std::memcpy(&id, nccl_id, sizeof(id));
+    const int32_t me = first_owned(ctx);
+    CU_OK(cudaSetDevice(ctx->dev[me].phys));
+    NCCL_OK(ncclCommInitRank(&ctx->comm, world, id, my_rank));
+    CU_OK(cudaMalloc(&ctx->bar_buf, sizeof(float)));
+    CU_OK(cudaMemset(ctx->bar_buf, 0, sizeof(float)));
+  } else {
+    // in-process multi-GPU: enable peer access where possible
+    for (int32_t a = 0; a < G; ++a)
+      for (int32_t b = 0; b < G; ++b) {
+        const int pa = ctx->dev[a].phys, pb = ctx->dev[b].phys;
+        if (pa == pb) continue;
+        int can = 0;
+        cudaDeviceCanAccessPeer(&can, pa, pb);
+        if (can) {
+          cudaSetDevice(pa);
+          cudaError_t e = cudaDeviceEnablePeerAccess(pb, 0);
+          if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+        }
+      }
+  }
+  *out = guard.release();
+  return MM_OK;
+}
+
+void mm_ctx_destroy(mm_ctx* ctx) {
+  if (!ctx) return;
+  for (auto& r : ctx->dev) {
+    if (!r.mine) continue;
+    cudaSetDevice(r.phys);
+    if (r.stream) {
+      if (r.gctx) drv().StreamDestroy((CUstream)r.stream);
+      else cudaStreamDestroy(r.stream);
+    }
+    if (r.gctx) drv().GreenCtxDestroy(r.gctx);
+  }
+  if (ctx->comm) ncclCommDestroy(ctx->comm);
+  if (ctx->bar_buf) cudaFree(ctx->bar_buf);
+  for (auto p : ctx->flush_scratch)
+    if (p) cudaFreeHost(p);
+  delete ctx;
+}
+
+mm_status mm_ctx_stream(mm_ctx* ctx, int32_t d, void** stream) {
+  if (!ctx || !stream || d < 0 || d >= ctx->G) MM_FAIL(MM_EINVAL, "ctx_stream: bad arguments");
+  if (!ctx->dev[d].mine) MM_FAIL(MM_EINVAL, "ctx_stream: device %d not owned by this rank", d);
+  *stream = (void*)ctx->dev[d].stream;
+  return MM_OK;
+}
+
+mm_status mm_ctx_sm_count(mm_ctx* ctx, int32_t d, int32_t* sms) {
+  if (!ctx || !sms || d < 0 || d >= ctx->G) MM_FAIL(MM_EINVAL, "ctx_sm_count: bad arguments");
+  *sms = ctx->dev[d].sms;
+  return MM_OK;
+}
+
+mm_status mm_fill_uniform(mm_ctx* ctx, int32_t d, float* dst, int64_t n, uint64_t seed, int32_t array_id,
+                          int64_t start, float lo, float hi) {
+  if (!ctx || d < 0 || d >= ctx->G || !ctx->dev[d].mine || (n > 0 && !dst) || n < 0)
+    MM_FAIL(MM_EINVAL, "fill_uniform: bad arguments");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  CU_OK(set_dev(ctx, d));
+  CU_OK(fill_uniform(dst, n, seed, array_id, start, lo, hi, ctx->dev[d].stream));
+  CU_OK(cudaStreamSynchronize(ctx->dev[d].stream));
+  return MM_OK;
+}
+
+mm_status mm_fill_integers(mm_ctx* ctx, int32_t d, float* dst, int64_t n, uint64_t seed, int32_t array_id,
+                           int64_t start, int32_t lo, int32_t hi) {
+  if (!ctx || d < 0 || d >= ctx->G || !ctx->dev[d].mine || (n > 0 && !dst) || n < 0 || hi < lo)
+    MM_FAIL(MM_EINVAL, "fill_integers: bad arguments");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  CU_OK(set_dev(ctx, d));
+  CU_OK(fill_integers(dst, n, seed, array_id, start, lo, hi, ctx->dev[d].stream));
+  CU_OK(cudaStreamSynchronize(ctx->dev[d].stream));
+  return MM_OK;
+}
+
+mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_run_opts* o, mm_run_stats* st) {
+  if (!ctx || !plan_h || !buffers) MM_FAIL(MM_EINVAL, "run: null argument");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  Plan& plan = plan_h->p;
+  if (plan.G != ctx->G) MM_FAIL(MM_EINVAL, "run: plan has G=%d, ctx has G=%d", plan.G, ctx->G);
+  mm_run_stats local{};
+  mm_run_stats* S = st ? st : &local;
+  *S = mm_run_stats{};
+  const bool timing = o && o->time_kernels;
+  const bool graph = o && o->use_graph && !timing && ctx->world == 1;
+  mm_status r = ensure_rt(ctx, plan, timing);
+  if (r) return r;
+  PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  const int32_t root = first_owned(ctx);
+  cudaStream_t rs = ctx->dev[root].stream;
+  const size_t nbuf = plan.app.buffers.size() * (size_t)ctx->G;
+  auto t0 = std::chrono::steady_clock::now();
+  if (graph) {
+    std::vector<void*> bufs(buffers, buffers + nbuf);
+    if (!rt->gexec || bufs != rt->graph_bufs) {
+      if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
+      if (rt->graph) cudaGraphDestroy(rt->graph);
+      rt->gexec = nullptr;
+      rt->graph = nullptr;
+      CU_OK(set_dev(ctx, root));
+      CU_OK(cudaStreamBeginCapture(rs, cudaStreamCaptureModeThreadLocal));
+      mm_run_stats cap{};
+      r = issue_local(ctx, plan, buffers, o, false, &cap);
+      cudaGraph_t g = nullptr;
+      cudaError_t ce = cudaStreamEndCapture(rs, &g);
+      if (r) {
+        if (g) cudaGraphDestroy(g);
+        return r;
+      }
+      CU_OK(ce);
+      rt->graph = g;
+      CU_OK(cudaGraphInstantiate(&rt->gexec, g, 0));
+      rt->graph_bufs = bufs;
+      rt->graph_launches = cap.n_launches;
+      rt->graph_xfer = cap.xfer_bytes;
+      rt->graph_h2d = cap.h2d_bytes;
+      rt->graph_d2h = cap.d2h_bytes;
+    }
+    t0 = std::chrono::steady_clock::now();
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventRecord(rt->t_start, rs));
+    CU_OK(cudaGraphLaunch(rt->gexec, rs));
+    CU_OK(cudaEventRecord(rt->t_stop, rs));
+    S->n_launches = rt->graph_launches;
+    S->xfer_bytes = rt->graph_xfer;
+    S->h2d_bytes = rt->graph_h2d;
+    S->d2h_bytes = rt->graph_d2h;
+    g_kernel_launches.fetch_add(rt->graph_launches, std::memory_order_relaxed);
+  } else {
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventRecord(rt->t_start, rs));
+    if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
+    else r = issue_dist(ctx, plan, buffers, o, timing, S);
+    if (r) return r;
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventRecord(rt->t_stop, rs));
+  }
+  CU_OK(cudaEventSynchronize(rt->t_stop));
+  auto t1 = std::chrono::steady_clock::now();
+  S->wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+  float ms = 0.f;
+  CU_OK(cudaEventElapsedTime(&ms, rt->t_start, rt->t_stop));
+  S->device_ms = ms;
+  for (size_t i = 0; i < plan.ops.size(); ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    if (op.kind != MM_OPK_KERNEL || !ctx->dev[op.device].mine) continue;
+    S->kernel_launches[op.device][op.kernel]++;
+    if (timing) {
+      float k = 0.f;
+      CU_OK(cudaEventElapsedTime(&k, rt->kev[2 * i], rt->kev[2 * i + 1]));
+      S->kernel_ms[op.device][op.kernel] += k;
+    }
+  }
+  return MM_OK;
+}
+
+mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan_h, void* const* buffers, int32_t slot, void* dst,
+                     int32_t dst_device) {
+  if (!ctx || !plan_h || !buffers || !dst) MM_FAIL(MM_EINVAL, "collect: null argument");
+  const Plan& plan = plan_h->p;
+  if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "collect: in-process contexts only");
+  if (slot < 0 || slot >= (int32_t)plan.app.buffers.size()) MM_FAIL(MM_EINVAL, "collect: slot");
+  const int64_t eb = plan.app.buffers[slot].first;
+  for (auto& seg : plan.final_owner[slot]) {
+    const int32_t o = seg.second;
+    if (o < 0) continue;
+    const size_t bytes = (size_t)((seg.first.end - seg.first.begin) * eb);
+    const char* src = static_cast<const char*>(buffers[(size_t)slot * ctx->G + o]) + seg.first.begin * eb;
+    char* d = static_cast<char*>(dst) + seg.first.begin * eb;
+    CU_OK(set_dev(ctx, o));
+    if (dst_device < 0) CU_OK(cudaMemcpy(d, src, bytes, cudaMemcpyDeviceToHost));
+    else if (ctx->dev[dst_device].phys == ctx->dev[o].phys) CU_OK(cudaMemcpy(d, src, bytes, cudaMemcpyDeviceToDevice));
+    else CU_OK(cudaMemcpyPeer(d, ctx->dev[dst_device].phys, src, ctx->dev[o].phys, bytes));
+  }
+  return MM_OK;
+}
+
+// Glinda low-cost profiling (P49) + DP-Perf warm-up of 3 task instances per
+// device (P311).  Excluded from run timings.
+mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers, const mm_profile_opts* po,
+                         mm_profile* out) {
+  if (!ctx || !app_h || !buffers || !out) MM_FAIL(MM_EINVAL, "profile: null argument");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  const App& app = app_h->a;
+  const int32_t G = ctx->G, K = (int32_t)app.kernels.size();
+  if (K < 1 || K > MM_MAX_K) MM_FAIL(MM_EINVAL, "profile: K=%d", K);
+  const int32_t reps = po && po->reps > 0 ? po->reps : 5;
+  const int32_t warm = po && po->dp_warmup_chunks > 0 ? po->dp_warmup_chunks : 3;
+  const int32_t kpd = po && po->chunks_per_dev > 0 ? po->chunks_per_dev : 8;
+  *out = mm_profile{};
+  out->G = G;
+  out->K = K;
+  std::vector<uint64_t> row(2 * MM_MAX_K + 1, 0);
+  try {
+    for (int32_t d = 0; d < G; ++d) {
+      if (!ctx->dev[d].mine) continue;
+      cudaStream_t s = ctx->dev[d].stream;
+      CU_OK(set_dev(ctx, d));
+      cudaEvent_t a, b;
+      CU_OK(cudaEventCreate(&a));
+      CU_OK(cudaEventCreate(&b));
+      auto time_task = [&](const Task& t, float* ms) -> mm_status {
+        mm_status r = launch_task(ctx, app, t, d, buffers, s);  // warm-up
+        if (r) return r;
+        CU_OK(cudaEventRecord(a, s));
+        r = launch_task(ctx, app, t, d, buffers, s);
+        if (r) return r;
+        CU_OK(cudaEventRecord(b, s));
+        CU_OK(cudaEventSynchronize(b));
+        CU_OK(cudaEventElapsedTime(ms, a, b));
+        return MM_OK;
+      };
+      for (int32_t k = 0; k < K; ++k) {
+        const Kernel& kern = app.kernels[k];
+        if (app.is_dag) {
+          const Task* t = nullptr;
+          for (auto& x : app.dag)
+            if (x.kernel == k) {
+              t = &x;
+              break;
+            }
+          if (!t) continue;
+          std::vector<float> v(reps);
+          for (int32_t i = 0; i < reps; ++i) {
+            mm_status r = time_task(*t, &v[i]);
+            if (r) return r;
+          }
+          std::sort(v.begin(), v.end());
+          const uint64_t ns = std::max<uint64_t>(1, (uint64_t)(v[reps / 2] * 1e6));
+          out->chunk_est_ns[d][k] = ns;
+          out->ps_item[d][k] = ns * 1000;
+          continue;
+        }
+        // probe: the even share n/G (>= one wave of the kernel), median of reps
+        int64_t probe = po && po->probe_items > 0 ? po->probe_items : chunk_size(kern.n, kern.granule, G);
+        probe = std::min<int64_t>(std::max<int64_t>(probe, std::min(kern.n, kern.min_items)), kern.n);
+        if (probe <= 0) {
+          out->ps_item[d][k] = 1;
+          out->chunk_est_ns[d][k] = 1;
+          continue;
+        }
+        Task t = range_task(app, k, 0, 0, probe, 0);
+        std::vector<float> v(reps);
+        for (int32_t i = 0; i < reps; ++i) {
+          mm_status r = time_task(t, &v[i]);
+          if (r) return r;
+        }
+        std::sort(v.begin(), v.end());
+        out->ps_item[d][k] = std::max<uint64_t>(1, (uint64_t)((double)v[reps / 2] * 1e9 / (double)probe));
+        // DP-Perf warm-up: `warm` nominal chunks on this device (P311)
+        const int64_t cs = chunk_size(kern.n, kern.granule, (int64_t)kpd * G);
+        double sum = 0.0;
+        int32_t cnt = 0;
+        for (int32_t i = 0; i < warm; ++i) {
+          const int64_t b0 = std::min<int64_t>((int64_t)i * cs, std::max<int64_t>(0, kern.n - cs));
+          Task c = range_task(app, k, 0, b0, std::min(kern.n, b0 + cs), 0);
+          float ms = 0.f;
+          mm_status r = time_task(c, &ms);
+          if (r) return r;
+          sum += ms;
+          cnt++;
+        }
+        out->chunk_est_ns[d][k] = std::max<uint64_t>(1, (uint64_t)(sum / cnt * 1e6));
+      }
+      // link: bytes/s of a 64 MiB device-to-device copy into d
+      {
+        const size_t bytes = 64ull << 20;
+        void *x = nullptr, *y = nullptr;
+        CU_OK(cudaMalloc(&x, bytes));
+        CU_OK(cudaMalloc(&y, bytes));
+        CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
+        CU_OK(cudaEventRecord(a, s));
+        CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
+        CU_OK(cudaEventRecord(b, s));
+        CU_OK(cudaEventSynchronize(b));
+        float ms = 0.f;
+        CU_OK(cudaEventElapsedTime(&ms, a, b));
+        cudaFree(x);
+        cudaFree(y);
+        out->link_Bps[d] = (uint64_t)((double)bytes / (ms * 1e-3));
+      }
+      cudaEventDestroy(a);
+      cudaEventDestroy(b);
+    }
+  } catch (const std::bad_alloc&) {
+    MM_FAIL(MM_ENOMEM, "profile: host memory");
+  }
+  if (ctx->world > 1) {
+    // exchange the per-device rows so every rank holds the same profile
+    const int32_t me = first_owned(ctx);
+    const size_t rowlen = 2 * MM_MAX_K + 1;
+    for (int32_t k = 0; k < MM_MAX_K; ++k) {
+      row[k] = out->ps_item[me][k];
+      row[MM_MAX_K + k] = out->chunk_est_ns[me][k];
+    }
+    row[2 * MM_MAX_K] = out->link_Bps[me];
+    uint64_t *dsend = nullptr, *drecv = nullptr;
+    CU_OK(set_dev(ctx, me));
+    CU_OK(cudaMalloc(&dsend, rowlen * 8));
+    CU_OK(cudaMalloc(&drecv, rowlen * 8 * ctx->world));
+    CU_OK(cudaMemcpy(dsend, row.data(), rowlen * 8, cudaMemcpyHostToDevice));
+    NCCL_OK(ncclAllGather(dsend, drecv, rowlen, ncclUint64, ctx->comm, ctx->dev[me].stream));
+    std::vector<uint64_t> all(rowlen * ctx->world);
+    CU_OK(cudaStreamSynchronize(ctx->dev[me].stream));
+    CU_OK(cudaMemcpy(all.data(), drecv, all.size() * 8, cudaMemcpyDeviceToHost));
+    cudaFree(dsend);
+    cudaFree(drecv);
+    for (int32_t d = 0; d < G; ++d) {
+      const uint64_t* rr = all.data() + (size_t)ctx->dev[d].rank * rowlen;
+      for (int32_t k = 0; k < MM_MAX_K; ++k) {
+        out->ps_item[d][k] = rr[k];
+        out->chunk_est_ns[d][k] = rr[MM_MAX_K + k];
+      }
+      out->link_Bps[d] = rr[2 * MM_MAX_K];
+    }
+  }
+  return MM_OK;
+}
+
+int64_t mm_kernel_launch_count(void) { return g_kernel_launches.load(); }
+
+}  // extern "C"

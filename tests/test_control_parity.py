@@ -1,0 +1,279 @@
+"""The C++ control plane (libmm.so through its C ABI) against the oracle:
+classification, ranking, splits, DP schedules and the op program must be
+bit-identical.  Host-only calls: runs on CPU (no GPU needed)."""
+import random
+
+import pytest
+
+from oracle import apps as oa
+from oracle import control as oc
+
+mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+
+
+# ------------------------------------------------------------ app builders --
+def stream_pair(n, passes=1, sync=0, granule=32, min_items=1):
+    app = mm.mm_app_builtin(mm.MM_APP_STREAM, [n, passes, sync, granule, min_items])
+    return app, oa.stream(n, passes, sync, granule, min_items)
+
+
+def hotspot_pair(rows, cols, iters, granule=1, min_items=1):
+    app = mm.mm_app_builtin(mm.MM_APP_HOTSPOT, [rows, cols, iters, granule, min_items])
+    return app, oa.hotspot(rows, cols, iters, granule, min_items)
+
+
+def stencil_pair(rows, cols, steps, sync=1, granule=1):
+    app = mm.mm_app_builtin(mm.MM_APP_STENCIL_REDUCTION, [rows, cols, steps, sync, granule, 1])
+    return app, oa.stencil_reduction(rows, cols, steps, sync, granule)
+
+
+def bs_pair(n, granule=32):
+    app = mm.mm_app_builtin(mm.MM_APP_BLACKSCHOLES, [n, granule, 1])
+    k = oc.Kernel("bs", n, granule, 1, [oc.Access(0, oc.READ), oc.Access(1, oc.READ), oc.Access(2, oc.READ),
+                                        oc.Access(3, oc.WRITE), oc.Access(4, oc.WRITE)])
+    return app, oc.App(buffers=[(4, n)] * 5, kernels=[k])
+
+
+def sgemm_pair(M, N, K, granule=16):
+    app = mm.mm_app_builtin(mm.MM_APP_SGEMM, [M, N, K, 1, granule, 1])
+    k = oc.Kernel("sgemm", M, granule, 1, [oc.Access(0, oc.READ, K), oc.Access(1, oc.READ, 0),
+                                           oc.Access(2, oc.WRITE, N)])
+    return app, oc.App(buffers=[(4, M * K), (4, K * N), (4, M * N)], kernels=[k])
+
+
+def chol_pair(T, b):
+    app = mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [T * b, b])
+    return app, oa.cholesky_tasks(T, b)
+
+
+def rand_profile(rnd, G, K, equal=False):
+    ps = [[rnd.randint(100, 5000) for _ in range(K)] for _ in range(G)]
+    est = [[rnd.randint(1000, 10 ** 6) for _ in range(K)] for _ in range(G)]
+    link = [rnd.randint(10 ** 8, 10 ** 12) for _ in range(G)]
+    if equal:
+        ps = [ps[0]] * G
+        est = [est[0]] * G
+        link = [link[0]] * G
+    po = oc.Profile(G=G, ps_item=ps, chunk_est_ns=est, link_Bps=link)
+    pc = mm.make_profile(G, ps, est, link)
+    return pc, po
+
+
+def ops_as_tuples(plan):
+    out = []
+    for o in mm.mm_plan_ops(plan):
+        if o.kind == mm.MM_OPK_KERNEL:
+            out.append((oc.OP_KERNEL, o.device, o.kernel, o.iter, o.r.begin, o.r.end))
+        elif o.kind == mm.MM_OPK_XFER:
+            out.append((oc.OP_XFER, o.device, o.src, o.buffer, o.r.begin, o.r.end))
+        elif o.kind == mm.MM_OPK_BARRIER:
+            out.append((oc.OP_BARRIER,))
+        else:
+            out.append((oc.OP_FLUSH, o.device, o.buffer, o.r.begin, o.r.end))
+    return out
+
+
+def oracle_plan(oapp, po, strategy, kpd=8, staged=False):
+    G = po.G
+    if strategy in (oc.SP_SINGLE, oc.SP_UNIFIED, oc.SP_VARIED):
+        ranges = oc.sp_split(oapp, po, strategy)
+        tasks, dev = oc.sp_tasks(oapp, ranges)
+        fin = [0] * len(tasks)
+    elif strategy == oc.DP_PERF:
+        tasks, dev, fin = oc.dp_perf(oapp, po, kpd)
+    elif strategy == oc.DP_DEP:
+        tasks, dev = oc.dp_dep(oapp, G, kpd)
+        fin = [0] * len(tasks)
+    else:
+        tasks, dev = oc.sp_cyclic(oapp, G)
+        fin = [0] * len(tasks)
+    ops = oc.op_program(oapp, G, tasks, dev, strategy, staged)
+    return tasks, dev, fin, ops
+
+
+def check_plan(capp, oapp, pc, po, strategy, kpd=8, staged=False):
+    plan = mm.mm_plan_build(capp, pc, mm.plan_opts(strategy, chunks_per_dev=kpd, staged=staged))
+    try:
+        tasks, dev, fin, ops = oracle_plan(oapp, po, strategy, kpd, staged)
+        ch = mm.mm_plan_chunks(plan)
+        assert len(ch) == len(tasks)
+        assert [c.device for c in ch] == dev
+        assert [c.kernel for c in ch] == [t.kernel for t in tasks]
+        assert [(c.items.begin, c.items.end) for c in ch] == [(t.begin, t.end) for t in tasks]
+        if strategy == oc.DP_PERF:
+            assert [c.finish_ns for c in ch] == fin
+        assert ops_as_tuples(plan) == ops
+        info = mm.mm_plan_info(plan)
+        assert info.xfer_bytes == oc.transfer_bytes(oapp, [o for o in ops if o[0] == oc.OP_XFER and o[2] >= 0])
+    finally:
+        mm.mm_plan_destroy(plan)
+
+
+# ------------------------------------------------------------------ tests --
+def test_abi_struct_sizes_match_header():
+    import ctypes
+    assert mm.mm_abi_sizes() == [ctypes.sizeof(s) for s in mm.ABI_STRUCTS]
+
+
+def test_exports_every_declared_symbol():
+    import re
+    import subprocess
+    hdr = open(mm.LIB_PATH.replace("paper_conf_icpp_shenvms15_b200/libmm.so", "include/mm.h")).read()
+    declared = set(re.findall(r"^(?:mm_status|void|const char\*|int64_t)\s+(mm_[a-z0-9_]+)\(", hdr, re.M))
+    assert len(declared) > 30
+    syms = subprocess.run(["nm", "-D", "--defined-only", mm.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (mm_[a-z0-9_]+)", syms))
+    assert declared <= exported, declared - exported
+    assert set(mm.EXPORTS) <= exported
+
+
+def test_classify_and_rank_builtin_apps():
+    cases = [(stream_pair(100, 1), oc.MK_SEQ), (stream_pair(100, 5), oc.MK_LOOP),
+             (hotspot_pair(8, 8, 10), oc.SK_LOOP), (hotspot_pair(8, 8, 1), oc.SK_ONE),
+             (stencil_pair(8, 8, 3), oc.MK_LOOP), (bs_pair(64), oc.SK_ONE), (sgemm_pair(64, 8, 8), oc.SK_ONE),
+             (chol_pair(3, 2), oc.MK_DAG)]
+    for (capp, oapp), cls in cases:
+        assert mm.mm_classify(capp) == oc.classify(oapp) == cls
+        ns = mm.mm_needs_sync(capp)
+        assert ns == oc.needs_sync(oapp)
+        assert mm.mm_rank(cls, ns) == oc.rank(cls, ns)
+        mm.mm_app_destroy(capp)
+
+
+def test_classify_custom_flows():
+    rnd = random.Random(3)
+    for _ in range(300):
+        k = rnd.randint(1, 4)
+        app = mm.mm_app_create()
+        b = mm.mm_app_add_buffer(app, 4, 16)
+        for i in range(k):
+            mm.mm_app_add_kernel(app, mm.kernel_desc(f"k{i}", mm.MM_OP_STREAM_COPY, 16, [(b, mm.MM_READ, 1, 0)]))
+        edges = [(rnd.randrange(k), rnd.randrange(k)) for _ in range(rnd.randint(0, 4))]
+        for a, c in edges:
+            mm.mm_app_add_edge(app, a, c)
+        loop = None
+        if rnd.random() < 0.5:
+            f = rnd.randrange(k)
+            l = rnd.randrange(f, k)
+            it = rnd.randint(1, 4)
+            mm.mm_app_set_loop(app, f, l, it)
+            loop = (f, l, it) if it > 1 else None
+        unstable = rnd.random() < 0.2
+        mm.mm_app_set_unstable(app, unstable)
+        oapp = oc.App(buffers=[(4, 16)], kernels=[oc.Kernel(f"k{i}", 16) for i in range(k)], edges=edges,
+                      loop=loop, unstable=unstable)
+        assert mm.mm_classify(app) == oc.classify(oapp), (k, edges, loop, unstable)
+        mm.mm_app_destroy(app)
+
+
+def test_split_random_profiles_bit_exact():
+    rnd = random.Random(11)
+    for trial in range(200):
+        G = rnd.randint(1, 8)
+        n = rnd.choice([0, 1, 31, 32, 1000, 4099, 1 << 20, (1 << 28) + 5])
+        g = rnd.choice([1, 4, 32, 128])
+        mn = rnd.choice([1, 1, 64, 100000])
+        capp, oapp = stream_pair(n, 1, 0, g, mn)
+        pc, po = rand_profile(rnd, G, 4, equal=(trial % 5 == 0))
+        for s in (oc.SP_UNIFIED, oc.SP_VARIED):
+            got, _ = mm.mm_split(capp, pc, s)
+            assert got == oc.sp_split(oapp, po, s), (trial, s)
+        mm.mm_app_destroy(capp)
+
+
+def test_split_stream_2_28_over_8():
+    capp, _ = stream_pair(1 << 28, 1, 0, 32, 1)
+    pc = mm.make_profile(8, [[1000] * 4] * 8, [[1] * 4] * 8, [1] * 8)
+    got, used = mm.mm_split(capp, pc, mm.MM_SP_UNIFIED)
+    assert used == 8 and [e - b for b, e in got[0]] == [33554432] * 8
+    mm.mm_app_destroy(capp)
+
+
+def test_matmul_1024_resolves_to_one_gpu():
+    # BASELINE configs[0]: 1024^2 fills less than one wave per device -> 1 GPU (P49 decision)
+    capp = mm.mm_app_builtin(mm.MM_APP_SGEMM, [1024, 1024, 1024])
+    pc = mm.make_profile(8, [[1000]] * 8, [[1]] * 8, [1] * 8)
+    got, used = mm.mm_split(capp, pc, mm.MM_SP_SINGLE)
+    assert used == 1 and got[0][0] == (0, 1024)
+    mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_UNIFIED, oc.SP_VARIED, oc.DP_PERF, oc.DP_DEP])
+@pytest.mark.parametrize("sync", [0, 1, 2])
+def test_plan_stream(strategy, sync):
+    rnd = random.Random(100 + strategy * 7 + sync)
+    for trial in range(6):
+        G = rnd.randint(1, 5)
+        n = rnd.choice([64, 1000, 4099])
+        passes = rnd.choice([1, 2])
+        capp, oapp = stream_pair(n, passes, sync, rnd.choice([1, 32]), 1)
+        pc, po = rand_profile(rnd, G, 4)
+        check_plan(capp, oapp, pc, po, strategy, kpd=rnd.choice([1, 2, 4]))
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_SINGLE, oc.DP_PERF, oc.DP_DEP])
+def test_plan_hotspot(strategy):
+    rnd = random.Random(7 + strategy)
+    for trial in range(5):
+        G = rnd.randint(1, 4)
+        capp, oapp = hotspot_pair(rnd.randint(8, 40), rnd.choice([4, 7]), rnd.randint(1, 4))
+        pc, po = rand_profile(rnd, G, 1)
+        check_plan(capp, oapp, pc, po, strategy, kpd=rnd.choice([1, 2, 3]))
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_UNIFIED, oc.SP_VARIED, oc.DP_PERF, oc.DP_DEP])
+def test_plan_stencil_reduction(strategy):
+    rnd = random.Random(17 + strategy)
+    for trial in range(4):
+        G = rnd.randint(1, 4)
+        capp, oapp = stencil_pair(rnd.randint(8, 30), 5, rnd.randint(1, 3), rnd.choice([0, 1, 2]))
+        pc, po = rand_profile(rnd, G, 2)
+        check_plan(capp, oapp, pc, po, strategy, kpd=2)
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_SINGLE, oc.DP_PERF, oc.DP_DEP])
+def test_plan_blackscholes_sgemm(strategy):
+    rnd = random.Random(5 + strategy)
+    for mk in (lambda: bs_pair(rnd.randint(50, 500)), lambda: sgemm_pair(rnd.randint(20, 90), 6, 5)):
+        G = rnd.randint(1, 4)
+        capp, oapp = mk()
+        pc, po = rand_profile(rnd, G, 1)
+        check_plan(capp, oapp, pc, po, strategy, kpd=2)
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.DP_PERF, oc.DP_DEP, oc.SP_CYCLIC])
+def test_plan_cholesky(strategy):
+    rnd = random.Random(23 + strategy)
+    for G in (1, 2, 4, 6):
+        capp, oapp = chol_pair(rnd.randint(2, 5), 2)
+        pc, po = rand_profile(rnd, G, 4)
+        check_plan(capp, oapp, pc, po, strategy)
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_UNIFIED, oc.SP_VARIED, oc.DP_PERF])
+def test_plan_staged(strategy):
+    rnd = random.Random(31 + strategy)
+    for trial in range(4):
+        G = rnd.randint(1, 4)
+        capp, oapp = stream_pair(rnd.choice([100, 777]), rnd.choice([1, 2]), rnd.choice([0, 1]), 32, 1)
+        pc, po = rand_profile(rnd, G, 4)
+        check_plan(capp, oapp, pc, po, strategy, kpd=2, staged=True)
+        mm.mm_app_destroy(capp)
+
+
+def test_errors_are_status_codes():
+    with pytest.raises(mm.MMError) as e:
+        mm.mm_rank(99, 0)
+    assert e.value.status == mm.MM_EINVAL
+    capp, _ = stream_pair(100, 1)
+    pc = mm.make_profile(2, [[0] * 4] * 2, [[1] * 4] * 2, [1, 1])
+    with pytest.raises(mm.MMError):
+        mm.mm_split(capp, pc, mm.MM_SP_UNIFIED)   # zero cost
+    with pytest.raises(mm.MMError):
+        mm.mm_split(capp, mm.make_profile(2, [[1] * 4] * 2), mm.MM_SP_SINGLE)  # 4 kernels
+    mm.mm_app_destroy(capp)

@@ -1,0 +1,209 @@
+"""GPU parity: the CUDA path (libmm.so through its C ABI) against the oracle,
+element by element, on the same seeded inputs.  Several logical devices are
+mapped onto GPU 0 (separate streams and full-size buffer copies), so every
+partitioning strategy, re-sync, halo and sync path runs on one B200.
+
+Tolerances (BASELINE north_star): bit-exact for STREAM, HotSpot and
+integer-input MatrixMul (FP32 with a fixed operation order, R13/R16); <= 1e-5
+for BlackScholes (FP32 vs the FP64 oracle, R19); <= 1e-4 relative for
+MatrixMul on U[0,1) data; rowsum within 1e-12 relative (FP64)."""
+import numpy as np
+import pytest
+
+import synthgen
+from oracle import numeric as on
+
+pytestmark = pytest.mark.gpu
+
+SP = {1: "SP-Single", 2: "SP-Unified", 3: "SP-Varied", 4: "DP-Perf", 5: "DP-Dep"}
+
+
+@pytest.fixture(scope="module")
+def R(gpu):
+    from paper_conf_icpp_shenvms15_b200 import mm, runner
+    return mm, runner
+
+
+def rand_profile(mm, G, K, seed):
+    rnd = np.random.default_rng(seed)
+    ps = rnd.integers(500, 3000, size=(G, K)).tolist()
+    est = rnd.integers(10 ** 4, 10 ** 6, size=(G, K)).tolist()
+    link = rnd.integers(10 ** 9, 10 ** 12, size=G).tolist()
+    return mm.make_profile(G, ps, est, link)
+
+
+def test_device_generator_matches_synthgen(R):
+    mm, runner = R
+    with runner.session(mm.MM_APP_STREAM, [100003, 1, 0, 32, 1], G=1) as s:
+        s.fill()
+        for slot, aid in ((0, synthgen.AID_STREAM_A), (1, synthgen.AID_STREAM_B)):
+            got = s.bufs[(slot, 0)].cpu().numpy()
+            assert np.array_equal(got, synthgen.uniform(100003, aid, -1.0, 1.0))
+        t = s.bufs[(2, 0)]
+        mm.mm_fill_integers(s.ctx, 0, t.data_ptr(), 5000, synthgen.SEED, 31, 17, -4, 4)
+        assert np.array_equal(t[:5000].cpu().numpy(),
+                              synthgen.integers(5000, 31, -4, 4, start=17).astype(np.float32))
+
+
+@pytest.mark.parametrize("strategy", [2, 3, 4, 5])
+@pytest.mark.parametrize("sync", [0, 1, 2])
+@pytest.mark.parametrize("G", [1, 3])
+def test_stream_bit_exact(R, strategy, sync, G):
+    mm, runner = R
+    n, passes = 100003, 3
+    a0, b0, c0 = synthgen.stream_random(n)
+    ra, rb, rc = on.stream_run(a0, b0, c0, passes)
+    with runner.session(mm.MM_APP_STREAM, [n, passes, sync, 32, 1], G=G) as s:
+        s.fill()
+        prof = rand_profile(mm, G, 4, strategy * 10 + sync)
+        plan = s.plan(strategy, prof, chunks_per_dev=3)
+        s.run(plan)
+        for slot, ref in ((0, ra), (1, rb), (2, rc)):
+            got = s.collect(plan, slot)
+            assert np.array_equal(got, ref), (SP[strategy], sync, G, slot)
+
+
+def test_stream_graph_replay_and_staged(R):
+    mm, runner = R
+    n = 65536 + 77
+    a0, b0, c0 = synthgen.stream_random(n)
+    ra, rb, rc = on.stream_run(a0, b0, c0, 2)
+    import torch
+    with runner.session(mm.MM_APP_STREAM, [n, 1, 0, 32, 1], G=2) as s:
+        s.fill()
+        plan = s.plan(4, rand_profile(mm, 2, 4, 5), chunks_per_dev=4)
+        s.run(plan, use_graph=True)
+        s.run(plan, use_graph=True)       # replay: second pass
+        assert np.array_equal(s.collect(plan, 0), ra)
+        # staged mode: host inputs, H2D/D2H inside the run
+        host = [torch.from_numpy(x.copy()).pin_memory() for x in (a0, b0, c0)]
+        splan = s.plan(2, rand_profile(mm, 2, 4, 6), staged=True)
+        st = s.run(splan, host=[h.data_ptr() for h in host])
+        r1 = on.stream_run(a0, b0, c0, 1)
+        assert st.h2d_bytes > 0 and st.d2h_bytes > 0
+        for h, ref in zip(host, r1):
+            assert np.array_equal(h.numpy(), ref)
+
+
+@pytest.mark.parametrize("shape", [(257, 256), (100, 37), (64, 1032)])
+@pytest.mark.parametrize("strategy", [1, 4, 5])
+@pytest.mark.parametrize("G", [1, 3])
+def test_hotspot_bit_exact(R, shape, strategy, G):
+    mm, runner = R
+    rows, cols = shape
+    iters = 7
+    t0, p = synthgen.hotspot(rows, cols)
+    ref = on.hotspot_run(t0, p, iters)
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1], G=G) as s:
+        s.fill()
+        plan = s.plan(strategy, rand_profile(mm, G, 1, rows + strategy), chunks_per_dev=2)
+        s.run(plan)
+        out_slot = 0 if iters % 2 == 0 else 1
+        got = s.collect(plan, out_slot).reshape(rows, cols)
+        assert np.array_equal(got, ref), (SP[strategy], G, shape)
+
+
+@pytest.mark.parametrize("strategy", [2, 3, 4, 5])
+def test_stencil_reduction(R, strategy):
+    mm, runner = R
+    rows, cols, steps = 131, 64, 4
+    t0, p = synthgen.hotspot(rows, cols)
+    tf, rs = on.stencil_reduction_run(t0, p, steps)
+    prev = on.hotspot_run(t0, p, steps - 1)
+    last_rows = on.row_residual(prev, tf)
+    with runner.session(mm.MM_APP_STENCIL_REDUCTION, [rows, cols, steps, 2, 1, 1], G=3) as s:
+        s.fill()
+        plan = s.plan(strategy, rand_profile(mm, 3, 2, strategy), chunks_per_dev=2)
+        s.run(plan)
+        got = s.collect(plan, 0 if steps % 2 == 0 else 1).reshape(rows, cols)
+        assert np.array_equal(got, tf)
+        rowsum = s.collect(plan, 3)
+        assert np.max(np.abs(rowsum - last_rows) / np.maximum(last_rows, 1e-300)) < 1e-12
+        import math
+        assert abs(math.fsum(rowsum) - rs[-1]) <= 1e-12 * rs[-1]
+
+
+@pytest.mark.parametrize("G", [1, 2])
+@pytest.mark.parametrize("strategy", [1, 4, 5])
+def test_blackscholes(R, G, strategy):
+    mm, runner = R
+    n = 100003
+    S, X, T = synthgen.blackscholes(n)
+    rc, rp = on.blackscholes(S, X, T)
+    with runner.session(mm.MM_APP_BLACKSCHOLES, [n, 32, 1], G=G) as s:
+        s.fill()
+        plan = s.plan(strategy, rand_profile(mm, G, 1, 3), chunks_per_dev=2)
+        s.run(plan)
+        c = s.collect(plan, 3).astype(np.float64)
+        p = s.collect(plan, 4).astype(np.float64)
+    err_c = np.max(np.abs(c - rc) / np.maximum(np.abs(rc), 1.0))
+    err_p = np.max(np.abs(p - rp) / np.maximum(np.abs(rp), 1.0))
+    assert err_c <= 1e-5 and err_p <= 1e-5, (err_c, err_p)
+    # put-call parity on the GPU's own outputs (FP32 rounding of ~max(S,X))
+    par = (c - p) - (S - X * np.exp(-on.BS_R * T.astype(np.float64)))
+    assert np.max(np.abs(par) / np.maximum(S, X)) < 4e-6
+
+
+@pytest.mark.parametrize("variant", [1])
+@pytest.mark.parametrize("G", [1, 2])
+def test_sgemm(R, variant, G):
+    mm, runner = R
+    M, N, K = 300, 200, 96
+    Ai, Bi = synthgen.matmul_integer(M, K, N)
+    ref_i = on.sgemm(Ai, Bi)
+    Au, Bu = synthgen.matmul_uniform(M, K, N)
+    ref_u = on.sgemm(Au, Bu)
+    for integer, ref in ((True, ref_i), (False, ref_u)):
+        with runner.session(mm.MM_APP_SGEMM, [M, N, K, variant, 16, 1], G=G) as s:
+            s.fill(integer=integer)
+            plan = s.plan(1, rand_profile(mm, G, 1, 9))
+            s.run(plan)
+            got = s.collect(plan, 2).reshape(M, N)
+        if integer:
+            assert np.array_equal(got, ref)
+        else:
+            assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-4
+
+
+def test_stream_full_size_sampled(R):
+    """BASELINE configs[1] size (2^28) in the bench's launch configuration
+    (1 logical device, SP-Unified, CUDA graph): sampled outputs vs the oracle
+    run on the sampled inputs (STREAM is elementwise)."""
+    mm, runner = R
+    n = 1 << 28
+    idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
+                                    np.random.default_rng(0).integers(0, n, 4096)]))
+    with runner.session(mm.MM_APP_STREAM, [n, 1, 0], G=1) as s:
+        prof = s.profile(reps=3)          # profiling runs the kernels: fill afterwards
+        s.fill()
+        plan = s.plan(2, prof)
+        s.run(plan, use_graph=True)
+        import torch
+        ti = torch.from_numpy(idx).cuda()
+        got = [s.bufs[(k, 0)][ti].cpu().numpy() for k in range(3)]
+    a0 = np.concatenate([synthgen.uniform(1, synthgen.AID_STREAM_A, -1, 1, start=int(i)) for i in idx])
+    b0 = np.concatenate([synthgen.uniform(1, synthgen.AID_STREAM_B, -1, 1, start=int(i)) for i in idx])
+    c0 = np.concatenate([synthgen.uniform(1, synthgen.AID_STREAM_C, -1, 1, start=int(i)) for i in idx])
+    ra, rb, rc = on.stream_run(a0, b0, c0, 1)
+    assert np.array_equal(got[0], ra) and np.array_equal(got[1], rb) and np.array_equal(got[2], rc)
+
+
+def test_hotspot_full_size_sampled_rows(R):
+    """BASELINE configs[2] grid (8192^2) for 6 iterations: sampled rows vs the
+    oracle on a row window (the dependency cone after k steps is k rows)."""
+    mm, runner = R
+    rows = cols = 8192
+    iters = 6
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters], G=1) as s:
+        s.fill()
+        plan = s.plan(1)
+        s.run(plan)
+        out = s.bufs[(0, 0)].view(rows, cols)
+        sample = [0, 1, 4095, 4096, rows - 1]
+        got = {y: out[y].cpu().numpy() for y in sample}
+    t_full, p_full = synthgen.hotspot(rows, cols)
+    for y in sample:
+        lo, hi = max(0, y - iters - 1), min(rows, y + iters + 2)
+        # window rows at the cut are wrong after k steps only within k rows of the cut
+        ref = on.hotspot_run(t_full[lo:hi], p_full[lo:hi], iters)
+        assert np.array_equal(got[y], ref[y - lo]), y
