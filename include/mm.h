@@ -209,6 +209,11 @@ typedef struct {
   int32_t chunks_per_dev;    /* DP: C = chunks_per_dev * G (default 8) */
   int32_t staged;            /* inputs start on the host; outputs end there */
   int32_t grid_rows;         /* SP-Cyclic process grid rows (0 = auto) */
+  int32_t one_shot;          /* resident mode: 1 = program valid only from replicated
+                                inputs (one run); 0 (default) = steady-state program,
+                                planned from the state the program itself leaves, valid
+                                for the first run and every repeated run (R22) */
+  int32_t _pad;
   const mm_range* split;     /* optional SP split override [K*G] */
 } mm_plan_opts;
 
@@ -254,6 +259,11 @@ mm_status mm_plan_info(const mm_plan* plan, mm_plan_info_t* out);
 mm_status mm_plan_ranges(const mm_plan* plan, mm_range* out, int32_t cap, int32_t* count);
 mm_status mm_plan_chunks(const mm_plan* plan, mm_chunk* out, int64_t cap, int64_t* count);
 mm_status mm_plan_ops(const mm_plan* plan, mm_op_rec* out, int64_t cap, int64_t* count);
+/* Final location of buffer `slot` after the program: disjoint element ranges
+ * covering [0, n) and, per range, the device holding its final value (the
+ * last writer, else the lowest device with a valid copy, -1 = host only). */
+mm_status mm_plan_owners(const mm_plan* plan, int32_t slot, mm_range* ranges, int32_t* owners,
+                         int64_t cap, int64_t* count);
 
 /* ------------------------------------------------------------------------
  * Runtime (GPU)

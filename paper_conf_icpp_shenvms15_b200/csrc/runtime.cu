@@ -4,6 +4,7 @@
 // profiling (P49) with the DP-Perf warm-up (P311), and result collection.
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <dlfcn.h>
 #include <nccl.h>
 
 #include <algorithm>
@@ -79,6 +80,52 @@ static Drv& drv() {
   return d;
 }
 
+// NCCL entry points, resolved with dlopen when a multi-process context is
+// created: the library does not link libnccl, so it never pins a second NCCL
+// build into a process that also loads torch's (torch's is reused when present).
+struct Nccl {
+  decltype(&ncclGetUniqueId) GetUniqueId = nullptr;
+  decltype(&ncclCommInitRank) CommInitRank = nullptr;
+  decltype(&ncclCommDestroy) CommDestroy = nullptr;
+  decltype(&ncclGroupStart) GroupStart = nullptr;
+  decltype(&ncclGroupEnd) GroupEnd = nullptr;
+  decltype(&ncclSend) Send = nullptr;
+  decltype(&ncclRecv) Recv = nullptr;
+  decltype(&ncclAllReduce) AllReduce = nullptr;
+  decltype(&ncclAllGather) AllGather = nullptr;
+  decltype(&ncclGetErrorString) GetErrorString = nullptr;
+  bool ok = false;
+};
+
+static Nccl& nccl() {
+  static Nccl n;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);  // already loaded (torch)?
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_LOCAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_LOCAL);
+    if (!h) return n;
+    bool ok = true;
+    auto get = [&](const char* name, void** fp) {
+      *fp = dlsym(h, name);
+      if (!*fp) ok = false;
+    };
+    get("ncclGetUniqueId", (void**)&n.GetUniqueId);
+    get("ncclCommInitRank", (void**)&n.CommInitRank);
+    get("ncclCommDestroy", (void**)&n.CommDestroy);
+    get("ncclGroupStart", (void**)&n.GroupStart);
+    get("ncclGroupEnd", (void**)&n.GroupEnd);
+    get("ncclSend", (void**)&n.Send);
+    get("ncclRecv", (void**)&n.Recv);
+    get("ncclAllReduce", (void**)&n.AllReduce);
+    get("ncclAllGather", (void**)&n.AllGather);
+    get("ncclGetErrorString", (void**)&n.GetErrorString);
+    n.ok = ok;
+  }
+  return n;
+}
+
 struct mm_ctx {
   std::vector<DevRt> dev;
   int32_t G = 0, my_rank = 0, world = 1;
@@ -115,7 +162,7 @@ namespace {
     ncclResult_t r_ = (expr);                                                    \
     if (r_ != ncclSuccess) {                                                     \
       if (ctx) ctx->poisoned = true;                                             \
-      MM_FAIL(MM_ENCCL, "%s failed: %s", #expr, ncclGetErrorString(r_));         \
+      MM_FAIL(MM_ENCCL, "%s failed: %s", #expr, nccl().GetErrorString(r_));      \
     }                                                                            \
   } while (0)
 
@@ -407,11 +454,11 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
     const mm_op_rec& op = plan.ops[i];
     const bool x = op.kind == MM_OPK_XFER && op.src >= 0 && (op.device == me || op.src == me);
     if (in_group && !(op.kind == MM_OPK_XFER && op.src >= 0)) {
-      NCCL_OK(ncclGroupEnd());
+      NCCL_OK(nccl().GroupEnd());
       in_group = false;
     }
     if (op.kind == MM_OPK_BARRIER) {
-      NCCL_OK(ncclAllReduce(ctx->bar_buf, ctx->bar_buf, 1, ncclFloat, ncclSum, ctx->comm, s));
+      NCCL_OK(nccl().AllReduce(ctx->bar_buf, ctx->bar_buf, 1, ncclFloat, ncclSum, ctx->comm, s));
       continue;
     }
     if (op.kind == MM_OPK_KERNEL) {
@@ -436,14 +483,14 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
     }
     if (x) {
       if (!in_group) {
-        NCCL_OK(ncclGroupStart());
+        NCCL_OK(nccl().GroupStart());
         in_group = true;
       }
       char* mine = static_cast<char*>(buffers[(size_t)op.buffer * G + me]) + op.r.begin * eb;
       if (op.device == me)
-        NCCL_OK(ncclRecv(mine, bytes, ncclChar, ctx->dev[op.src].rank, ctx->comm, s));
+        NCCL_OK(nccl().Recv(mine, bytes, ncclChar, ctx->dev[op.src].rank, ctx->comm, s));
       else
-        NCCL_OK(ncclSend(mine, bytes, ncclChar, ctx->dev[op.device].rank, ctx->comm, s));
+        NCCL_OK(nccl().Send(mine, bytes, ncclChar, ctx->dev[op.device].rank, ctx->comm, s));
       st->xfer_bytes += op.device == me ? (int64_t)bytes : 0;
       continue;
     }
@@ -458,7 +505,7 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
       st->d2h_bytes += (int64_t)bytes;
     }
   }
-  if (in_group) NCCL_OK(ncclGroupEnd());
+  if (in_group) NCCL_OK(nccl().GroupEnd());
   return MM_OK;
 }
 
@@ -472,8 +519,9 @@ extern "C" {
 mm_status mm_nccl_unique_id(void* out128) {
   if (!out128) MM_FAIL(MM_EINVAL, "null out");
   mm_ctx* ctx = nullptr;
+  if (!nccl().ok) MM_FAIL(MM_ENCCL, "libnccl.so.2 could not be loaded");
   ncclUniqueId id;
-  NCCL_OK(ncclGetUniqueId(&id));
+  NCCL_OK(nccl().GetUniqueId(&id));
   static_assert(sizeof(id) == 128, "ncclUniqueId size");
   std::memcpy(out128, &id, sizeof(id));
   return MM_OK;
@@ -572,11 +620,12 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
   }
   if (world > 1) {
     if (!nccl_id) MM_FAIL(MM_EINVAL, "multi-process ctx needs an NCCL unique id");
+    if (!nccl().ok) MM_FAIL(MM_ENCCL, "libnccl.so.2 could not be loaded");
     ncclUniqueId id;
     std::memcpy(&id, nccl_id, sizeof(id));
     const int32_t me = first_owned(ctx);
     CU_OK(cudaSetDevice(ctx->dev[me].phys));
-    NCCL_OK(ncclCommInitRank(&ctx->comm, world, id, my_rank));
+    NCCL_OK(nccl().CommInitRank(&ctx->comm, world, id, my_rank));
     CU_OK(cudaMalloc(&ctx->bar_buf, sizeof(float)));
     CU_OK(cudaMemset(ctx->bar_buf, 0, sizeof(float)));
   } else {
@@ -609,7 +658,7 @@ void mm_ctx_destroy(mm_ctx* ctx) {
     }
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);
   }
-  if (ctx->comm) ncclCommDestroy(ctx->comm);
+  if (ctx->comm) nccl().CommDestroy(ctx->comm);
   if (ctx->bar_buf) cudaFree(ctx->bar_buf);
   for (auto p : ctx->flush_scratch)
     if (p) cudaFreeHost(p);
@@ -877,7 +926,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
     CU_OK(cudaMalloc(&dsend, rowlen * 8));
     CU_OK(cudaMalloc(&drecv, rowlen * 8 * ctx->world));
     CU_OK(cudaMemcpy(dsend, row.data(), rowlen * 8, cudaMemcpyHostToDevice));
-    NCCL_OK(ncclAllGather(dsend, drecv, rowlen, ncclUint64, ctx->comm, ctx->dev[me].stream));
+    NCCL_OK(nccl().AllGather(dsend, drecv, rowlen, ncclUint64, ctx->comm, ctx->dev[me].stream));
     std::vector<uint64_t> all(rowlen * ctx->world);
     CU_OK(cudaStreamSynchronize(ctx->dev[me].stream));
     CU_OK(cudaMemcpy(all.data(), drecv, all.size() * 8, cudaMemcpyDeviceToHost));

@@ -84,7 +84,8 @@ class mm_profile(C.Structure):
 
 class mm_plan_opts(C.Structure):
     _fields_ = [("strategy", C.c_int32), ("chunks_per_dev", C.c_int32), ("staged", C.c_int32),
-                ("grid_rows", C.c_int32), ("split", C.POINTER(mm_range))]
+                ("grid_rows", C.c_int32), ("one_shot", C.c_int32), ("_pad", C.c_int32),
+                ("split", C.POINTER(mm_range))]
 
 
 class mm_chunk(C.Structure):
@@ -163,6 +164,8 @@ _SIGS = {
     "mm_plan_ranges": [_P, C.POINTER(mm_range), C.c_int32, C.POINTER(C.c_int32)],
     "mm_plan_chunks": [_P, C.POINTER(mm_chunk), C.c_int64, C.POINTER(C.c_int64)],
     "mm_plan_ops": [_P, C.POINTER(mm_op_rec), C.c_int64, C.POINTER(C.c_int64)],
+    "mm_plan_owners": [_P, C.c_int32, C.POINTER(mm_range), C.POINTER(C.c_int32), C.c_int64,
+                       C.POINTER(C.c_int64)],
     "mm_nccl_unique_id": [C.c_void_p],
     "mm_ctx_create": [C.POINTER(mm_device_spec), C.c_int32, C.c_int32, C.c_int32, C.c_void_p, C.POINTER(_P)],
     "mm_ctx_stream": [_P, C.c_int32, C.POINTER(_P)],
@@ -358,12 +361,13 @@ def mm_split(app: int, prof: mm_profile, strategy: int) -> Tuple[List[List[Tuple
 
 
 def plan_opts(strategy: int, chunks_per_dev: int = 8, staged: bool = False, grid_rows: int = 0,
-              split=None) -> mm_plan_opts:
+              split=None, one_shot: bool = False) -> mm_plan_opts:
     o = mm_plan_opts()
     o.strategy = strategy
     o.chunks_per_dev = chunks_per_dev
     o.staged = int(staged)
     o.grid_rows = grid_rows
+    o.one_shot = int(one_shot)
     if split is not None:
         flat = [r for row in split for r in row]
         arr = (mm_range * len(flat))(*[mm_range(b, e) for b, e in flat])
@@ -420,6 +424,16 @@ def mm_plan_ops(plan: int) -> List[mm_op_rec]:
     out = (mm_op_rec * max(1, n.value))()
     _call("mm_plan_ops", plan, out, n.value, C.byref(n))
     return list(out[:n.value])
+
+
+def mm_plan_owners(plan: int, slot: int) -> List[Tuple[int, int, int]]:
+    """[(begin, end, owner_device)] covering the slot's elements."""
+    n = C.c_int64()
+    lib.mm_plan_owners(plan, slot, None, None, 0, C.byref(n))
+    rr = (mm_range * max(1, n.value))()
+    oo = (C.c_int32 * max(1, n.value))()
+    _call("mm_plan_owners", plan, slot, rr, oo, n.value, C.byref(n))
+    return [(rr[i].begin, rr[i].end, oo[i]) for i in range(n.value)]
 
 
 def mm_nccl_unique_id() -> bytes:

@@ -13,16 +13,19 @@ def pytest_configure(config):
     config.addinivalue_line("markers", "slow: long-running CPU test")
 
 
-def has_gpu() -> bool:
+def gpu_status():
     try:
         import torch
-        return torch.cuda.is_available()
-    except Exception:
-        return False
+        ok = torch.cuda.is_available()
+        return ok, f"torch {torch.__version__} cuda.is_available()={ok} count={torch.cuda.device_count()} " \
+                   f"CUDA_VISIBLE_DEVICES={os.environ.get('CUDA_VISIBLE_DEVICES')}"
+    except Exception as e:  # report the real reason
+        return False, f"{type(e).__name__}: {e}"
 
 
 @pytest.fixture(scope="session")
 def gpu():
-    if not has_gpu():
-        pytest.fail("GPU test collected without a CUDA device (run -m 'not gpu' here)")
+    ok, why = gpu_status()
+    if not ok:
+        pytest.fail(f"GPU test without a usable CUDA device: {why}")
     return 0

@@ -73,7 +73,7 @@ def ops_as_tuples(plan):
     return out
 
 
-def oracle_plan(oapp, po, strategy, kpd=8, staged=False):
+def oracle_plan(oapp, po, strategy, kpd=8, staged=False, one_shot=True):
     G = po.G
     if strategy in (oc.SP_SINGLE, oc.SP_UNIFIED, oc.SP_VARIED):
         ranges = oc.sp_split(oapp, po, strategy)
@@ -87,14 +87,23 @@ def oracle_plan(oapp, po, strategy, kpd=8, staged=False):
     else:
         tasks, dev = oc.sp_cyclic(oapp, G)
         fin = [0] * len(tasks)
-    ops = oc.op_program(oapp, G, tasks, dev, strategy, staged)
+    if staged or one_shot:
+        ops = oc.op_program(oapp, G, tasks, dev, strategy, staged)
+    else:
+        ops = oc.steady_program(oapp, G, tasks, dev, strategy)
     return tasks, dev, fin, ops
 
 
 def check_plan(capp, oapp, pc, po, strategy, kpd=8, staged=False):
-    plan = mm.mm_plan_build(capp, pc, mm.plan_opts(strategy, chunks_per_dev=kpd, staged=staged))
+    for one_shot in (True, False):
+        _check_plan(capp, oapp, pc, po, strategy, kpd, staged, one_shot)
+
+
+def _check_plan(capp, oapp, pc, po, strategy, kpd, staged, one_shot):
+    plan = mm.mm_plan_build(capp, pc, mm.plan_opts(strategy, chunks_per_dev=kpd, staged=staged,
+                                                   one_shot=one_shot))
     try:
-        tasks, dev, fin, ops = oracle_plan(oapp, po, strategy, kpd, staged)
+        tasks, dev, fin, ops = oracle_plan(oapp, po, strategy, kpd, staged, one_shot)
         ch = mm.mm_plan_chunks(plan)
         assert len(ch) == len(tasks)
         assert [c.device for c in ch] == dev
