@@ -306,10 +306,15 @@ def main():
         per_launch_ms = dom_ms / dom_launch
         launches_per_step = dom_launch / args.steps
         if args.app == "sgemm":
+            # 3xTF32: FP32-equivalent flops; peak = measured bf16 x 0.5 (nominal
+            # tf32/bf16 dense ratio) / 3 (three tf32 MMAs per FP32 product)
             fl = 2 * iparam[1] * iparam[2] * items / launches_per_step
             ach = fl / (per_launch_ms * 1e-3) / 1e12
-            roof = {"bound": "tensor", "achieved": ach, "peak": tf_peak / 8 * 1.0, "unit": "TFLOP/s",
-                    "frac": None, "traffic": None}
+            pk = tf_peak * 0.5 / 3.0
+            roof = {"bound": "tensor", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
+                    "traffic": None, "kernel": "sgemm (3xTF32 tcgen05, incl. operand split)",
+                    "peak_kind": peak_kind + " bf16_tflops x 0.5 (tf32) / 3 (3xTF32)",
+                    "avg_launch_ms": per_launch_ms}
         else:
             byts = bpi * items / launches_per_step
             ach = byts / (per_launch_ms * 1e-3) / 1e9

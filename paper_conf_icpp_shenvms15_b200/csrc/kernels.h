@@ -9,13 +9,30 @@ namespace mm {
 struct Kernel;
 struct Task;
 
+// Library-owned device scratch of one logical device, with the cache of the
+// whole-operand split of a 3xTF32 GEMM (B is split once per run and device;
+// `epoch` is bumped by the runtime at every run and every profile launch).
+struct Scratch {
+  void* ptr = nullptr;
+  size_t bytes = 0;
+  const void* b_src = nullptr;
+  int64_t b_K = 0, b_N = 0;
+  uint64_t b_epoch = 0;
+  uint64_t epoch = 1;
+};
+
 struct Launch {
   const Kernel* k;          // kernel descriptor (op, params)
   const Task* t;            // task: item range [t->b, t->e) / DAG params
   void* const* opnd;        // device pointers, one per access (this device's copy)
   cudaStream_t stream;
   int32_t sms;              // SMs available to this logical device
+  Scratch* scr;             // this logical device's scratch
+  uint32_t ro_mask;         // bit i: operand i is never written by the app (cacheable)
 };
+
+// Device scratch a builtin kernel needs for this task (0 if none).
+size_t builtin_scratch_bytes(const Kernel& k, const Task& t);
 
 // Returns cudaSuccess, cudaErrorNotSupported for an unimplemented op, or the
 // launch error.  Empty ranges launch nothing.
@@ -40,7 +57,9 @@ cudaError_t blackscholes(const float* S, const float* X, const float* T, float* 
 
 // SGEMM rows [r0,r1) of C = A B (kernels_gemm.cu)
 cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
-                       int64_t r0, int64_t r1, int32_t variant, cudaStream_t s, int sms);
+                       int64_t r0, int64_t r1, int32_t variant, cudaStream_t s, int sms, Scratch* scr,
+                       bool b_readonly);
+size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows);
 
 // Cholesky tiles (kernels_chol.cu); A tile-major, T x T tiles of b x b.
 cudaError_t chol_task(int32_t op, float* A, int64_t T, int64_t b, int64_t i, int64_t j, int64_t k,

@@ -4,14 +4,15 @@
 //
 // variant 1 (FFMA): classic register-blocked SIMT SGEMM — 128x128 CTA tile,
 // BK = 8, 256 threads x (8x8) outputs, shared-memory double buffering.  It is
-// the FP32-exact correctness baseline (tensor cores only
-// via 3xTF32 or FFMA).  The tcgen05 3xTF32 variant lives in kernels_gemm_tc.cu.
+// the FFMA baseline (tensor cores only via 3xTF32 or
+// FFMA).  variant 2 (default) is the tcgen05 3xTF32 kernel in kernels_gemm_tc.cu.
 #include "kernels.h"
 
 namespace mm {
 
 cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N,
-                              int64_t K, int64_t r0, int64_t r1, cudaStream_t s, int sms);
+                              int64_t K, int64_t r0, int64_t r1, cudaStream_t s, int sms, Scratch* scr,
+                              bool b_readonly);
 
 namespace {
 
@@ -132,10 +133,11 @@ __global__ void __launch_bounds__(NT) sgemm_ffma(const float* __restrict__ A, co
 }  // namespace
 
 cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
-                       int64_t r0, int64_t r1, int32_t variant, cudaStream_t s, int sms) {
+                       int64_t r0, int64_t r1, int32_t variant, cudaStream_t s, int sms, Scratch* scr,
+                       bool b_readonly) {
   (void)M;
   if (r1 <= r0 || N <= 0) return cudaSuccess;
-  if (variant == 2) return sgemm_tf32x3_rows(A, B, C, M, N, K, r0, r1, s, sms);
+  if (variant == 2) return sgemm_tf32x3_rows(A, B, C, M, N, K, r0, r1, s, sms, scr, b_readonly);
   dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((r1 - r0 + BM - 1) / BM));
   sgemm_ffma<<<grid, NT, 0, s>>>(A, B, C, N, K, r0, r1);
   return cudaGetLastError();

@@ -1,11 +1,288 @@
-// tcgen05 3xTF32 SGEMM (placeholder until the tensor-core path lands).
+// MatrixMul on the 5th-generation tensor cores: 3xTF32 SGEMM with tcgen05.mma
+// (P311: C = A x B, FP32, row-wise split; tensor cores only
+// via an FP32-accurate path).
+//
+// x = hi + lo with hi = tf32_rn(x), lo = tf32_rn(x - hi); C = A_lo B_hi +
+// A_hi B_lo + A_hi B_hi accumulated in FP32 in TMEM (the A_lo B_lo term is
+// below FP32 resolution).  Integer inputs |x| <= 2048 have lo = 0, so
+// integer-valued products stay exact.
+//
+// Two phases per launch (all on the caller's stream):
+//  1. split: A rows [r0,r1) -> A_hi, A_lo (row-major, K padded to 32);
+//     B (K x N) -> B_hi^T, B_lo^T (N x K, "K-major") through a 32x32 smem
+//     transpose.  HBM-bound elementwise passes into library scratch.
+//  2. gemm: 128 x 256 output tile per CTA; warp 0 = TMA producer (four 2-D
+//     tensor maps, SWIZZLE_128B boxes of 32 fp32 along K), warp 1 = TMEM
+//     allocator + single-thread tcgen05.mma issuer (kind::tf32, M=128 N=256
+//     K=8, 3 MMAs per K step), warps 2-5 = epilogue (tcgen05.ld 32x32b ->
+//     registers -> global).  mbarrier ring of kStages stages between TMA and
+//     MMA; tcgen05.commit frees a stage and signals the epilogue.
+#include <cuda.h>
+
 #include "kernels.h"
 
 namespace mm {
 
-cudaError_t sgemm_tf32x3_rows(const float*, const float*, float*, int64_t, int64_t, int64_t, int64_t,
-                              int64_t, cudaStream_t, int) {
-  return cudaErrorNotSupported;
+cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                               uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
+
+namespace {
+
+constexpr int BM = 128, BN = 256, BK = 32, kStages = 2;
+constexpr int A_BYTES = BM * BK * 4;                 // 16 KB
+constexpr int B_BYTES = BN * BK * 4;                 // 32 KB
+constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+constexpr int SMEM_BYTES = kStages * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+constexpr int kThreadsGemm = 192;
+
+__device__ __forceinline__ uint32_t saddr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t c) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(saddr(b)), "r"(c));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(saddr(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}\n" ::"r"(saddr(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          saddr(dst)),
+      "l"((uint64_t)map), "r"(x), "r"(y), "r"(saddr(bar))
+      : "memory");
+}
+// UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row groups 1024 B apart.
+__device__ __forceinline__ uint64_t sdesc(const void* p) {
+  const uint64_t a = saddr(p);
+  uint64_t d = (a >> 4) & 0x3FFFull;         // start address
+  d |= 1ull << 16;                           // leading byte offset (unused for SW128 K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;          // stride byte offset
+  d |= 1ull << 46;                           // descriptor version (sm_100)
+  d |= 2ull << 61;                           // SWIZZLE_128B
+  return d;
+}
+__device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(saddr(bar))
+               : "memory");
+}
+
+__global__ void __launch_bounds__(kThreadsGemm, 1)
+    gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
+                const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
+                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(base + kStages * STAGE_BYTES);
+  uint64_t* empty = full + kStages;
+  uint64_t* tfull = empty + kStages;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m_blk = blockIdx.y, n_blk = blockIdx.x;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tAhi) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tAlo) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBhi) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBlo) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)), "n"(BN));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ===== TMA producer
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % kStages;
+        if (kb >= kStages) mbar_wait(&empty[s], (uint32_t)(((kb / kStages) - 1) & 1));
+        uint8_t* st = base + s * STAGE_BYTES;
+        mbar_expect_tx(&full[s], STAGE_BYTES);
+        tma_load_2d(st, &tAhi, kb * BK, m_blk * BM, &full[s]);
+        tma_load_2d(st + A_BYTES, &tAlo, kb * BK, m_blk * BM, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES, &tBhi, kb * BK, n_blk * BN, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kb * BK, n_blk * BN, &full[s]);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0) {  // ===== MMA issuer
+      const uint32_t idesc = (1u << 4)                 // D: fp32
+                             | (2u << 7) | (2u << 10)  // A, B: tf32
+                             | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % kStages;
+        mbar_wait(&full[s], (uint32_t)((kb / kStages) & 1));
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        uint8_t* st = base + s * STAGE_BYTES;
+        const uint64_t ahi = sdesc(st), alo = sdesc(st + A_BYTES);
+        const uint64_t bhi = sdesc(st + 2 * A_BYTES), blo = sdesc(st + 2 * A_BYTES + B_BYTES);
+#pragma unroll
+        for (int kk = 0; kk < BK / 8; ++kk) {
+          const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 fp32 = 32 B along K inside the swizzle atom
+          mma_tf32(tmem, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
+          mma_tf32(tmem, ahi + adv, blo + adv, idesc, 1u);
+          mma_tf32(tmem, ahi + adv, bhi + adv, idesc, 1u);
+        }
+        mma_commit(&empty[s]);
+      }
+      mma_commit(tfull);
+    }
+    __syncwarp();
+  } else {  // ===== epilogue: warps 2..5 -> TMEM lane groups (warp % 4)
+    mbar_wait(tfull, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int g = warp & 3;
+    const int64_t r = (int64_t)m_blk * BM + g * 32 + lane;  // row within [0, mrows)
+    const bool row_ok = r < mrows;
+    float* crow = C + (row0 + r) * N;
+#pragma unroll 1
+    for (int c = 0; c < BN; c += 16) {
+      uint32_t v[16];
+      const uint32_t ta = tmem + ((uint32_t)(g * 32) << 16) + (uint32_t)c;
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+          : "r"(ta));
+      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      const int64_t n0 = (int64_t)n_blk * BN + c;
+      if (row_ok) {
+        if (n0 + 16 <= N && (N & 3) == 0) {
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            *reinterpret_cast<float4*>(crow + n0 + 4 * q) =
+                make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
+                            __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
+        } else {
+#pragma unroll
+          for (int q = 0; q < 16; ++q)
+            if (n0 + q < N) crow[n0 + q] = __uint_as_float(v[q]);
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(BN));
+  }
+}
+
+__device__ __forceinline__ float tf32_rn(float x) {
+  uint32_t r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return __uint_as_float(r);
+}
+
+// A rows [r0, r0+mrows) x K -> hi/lo, row stride Kp (zero padding K..Kp).
+__global__ void split_rows(const float* __restrict__ A, float* __restrict__ hi, float* __restrict__ lo,
+                           int64_t K, int64_t Kp, int64_t r0, int64_t mrows) {
+  const int64_t n = mrows * Kp;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / Kp, k = i % Kp;
+    const float x = k < K ? A[(r0 + r) * K + k] : 0.f;
+    const float h = tf32_rn(x);
+    hi[i] = h;
+    lo[i] = tf32_rn(x - h);
+  }
+}
+
+// B (K x N) -> hi^T/lo^T (N x Kp), 32x32 tiles through shared memory.
+__global__ void split_transpose(const float* __restrict__ B, float* __restrict__ hi, float* __restrict__ lo,
+                                int64_t K, int64_t N, int64_t Kp) {
+  __shared__ float t[32][33];
+  const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
+  for (int j = threadIdx.y; j < 32; j += blockDim.y) {
+    const int64_t k = k0 + j, n = n0 + threadIdx.x;
+    t[j][threadIdx.x] = (k < K && n < N) ? B[k * N + n] : 0.f;
+  }
+  __syncthreads();
+  for (int j = threadIdx.y; j < 32; j += blockDim.y) {
+    const int64_t n = n0 + j, k = k0 + threadIdx.x;
+    if (n < N && k < Kp) {
+      const float x = t[threadIdx.x][j];
+      const float h = tf32_rn(x);
+      hi[n * Kp + k] = h;
+      lo[n * Kp + k] = tf32_rn(x - h);
+    }
+  }
+}
+
+}  // namespace
+
+size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
+  const int64_t Kp = (K + BK - 1) / BK * BK;
+  return (size_t)(2 * mrows * Kp + 2 * N * Kp) * sizeof(float);
+}
+
+cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
+                              int64_t r0, int64_t r1, cudaStream_t s, int sms, Scratch* scr, bool b_readonly) {
+  (void)M;
+  (void)sms;
+  const int64_t mrows = r1 - r0;
+  if (mrows <= 0 || N <= 0) return cudaSuccess;
+  if (!scr || !scr->ptr || scr->bytes < sgemm_tf32x3_scratch(N, K, mrows)) return cudaErrorNotSupported;
+  const int64_t Kp = (K + BK - 1) / BK * BK;
+  // scratch layout: [B_hi^T | B_lo^T] (N x Kp each) then [A_hi | A_lo] (mrows x Kp each)
+  float* bhi = static_cast<float*>(scr->ptr);
+  float* blo = bhi + N * Kp;
+  float* ahi = blo + N * Kp;
+  float* alo = ahi + mrows * Kp;
+  {
+    const int64_t n = mrows * Kp;
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    split_rows<<<(unsigned)blocks, 256, 0, s>>>(A, ahi, alo, K, Kp, r0, mrows);
+    // B is the same whole operand for every row range of this run: split it
+    // once per run on this device (only if the app never writes it).
+    const bool cached = b_readonly && scr->b_src == B && scr->b_K == K && scr->b_N == N && scr->b_epoch == scr->epoch;
+    if (!cached) {
+      dim3 g((unsigned)((N + 31) / 32), (unsigned)((Kp + 31) / 32));
+      split_transpose<<<g, dim3(32, 8), 0, s>>>(B, bhi, blo, K, N, Kp);
+      scr->b_src = b_readonly ? B : nullptr;
+      scr->b_K = K;
+      scr->b_N = N;
+      scr->b_epoch = scr->epoch;
+    }
+  }
+  CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(&ta_hi, ahi, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&ta_lo, alo, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    attr = true;
+  }
+  dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((mrows + BM - 1) / BM));
+  gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows,
+                                                     (int)(Kp / BK));
+  return cudaGetLastError();
 }
 
 }  // namespace mm

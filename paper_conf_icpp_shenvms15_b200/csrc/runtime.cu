@@ -26,6 +26,7 @@ std::atomic<int64_t> g_kernel_launches{0};
 
 struct DevRt {
   int32_t phys = 0, budget = 0, sms = 0, rank = 0;
+  Scratch scr;               // device scratch for builtin kernels (e.g. 3xTF32 operand split)
   cudaStream_t stream = nullptr;
   CUgreenCtx gctx = nullptr;
   CUcontext gcu = nullptr;   // CUcontext view of the green context
@@ -48,6 +49,7 @@ struct Drv {
   decltype(&cuCtxSetCurrent) CtxSetCurrent = nullptr;
   decltype(&cuStreamDestroy) StreamDestroy = nullptr;
   decltype(&cuGetErrorString) GetErrorString = nullptr;
+  decltype(&cuTensorMapEncodeTiled) TensorMapEncodeTiled = nullptr;
   bool ok = false;
 };
 
@@ -76,6 +78,10 @@ static Drv& drv() {
     get("cuStreamDestroy", (void**)&d.StreamDestroy);
     get("cuGetErrorString", (void**)&d.GetErrorString);
     d.ok = ok;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&d.TensorMapEncodeTiled, cudaEnableDefault,
+                                &q) != cudaSuccess || q != cudaDriverEntryPointSuccess)
+      d.TensorMapEncodeTiled = nullptr;
   }
   return d;
 }
@@ -215,6 +221,27 @@ int32_t first_owned(const mm_ctx* ctx) {
 
 namespace mm {
 
+// 2-D fp32 tensor map with a SWIZZLE_128B box (box_inner * 4 must be <= 128 B).
+cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                               uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer) {
+  Drv& D = drv();
+  if (!D.TensorMapEncodeTiled) return cudaErrorNotSupported;
+  const cuuint64_t dims[2] = {inner, outer};
+  const cuuint64_t strides[1] = {row_bytes};
+  const cuuint32_t box[2] = {box_inner, box_outer};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = D.TensorMapEncodeTiled(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides,
+                                      box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+size_t builtin_scratch_bytes(const Kernel& k, const Task& t) {
+  if (k.op == MM_OP_SGEMM && (k.ip[3] == 0 || k.ip[3] == 2))
+    return sgemm_tf32x3_scratch(k.ip[1], k.ip[2], t.e - t.b);
+  return 0;
+}
+
 void plan_runtime_free(Plan* plan) {
   destroy_rt(static_cast<PlanRt*>(plan->rt));
   plan->rt = nullptr;
@@ -239,12 +266,9 @@ cudaError_t launch_builtin(const Launch& L) {
     case MM_OP_BLACKSCHOLES:
       return blackscholes(f[0], f[1], f[2], f[3], f[4], (float)k.fp[0], (float)k.fp[1], b, e, L.stream, L.sms);
     case MM_OP_SGEMM: {
-      int32_t variant = (int32_t)k.ip[3];
-      if (variant == 0) variant = 2;
-      cudaError_t r = sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, variant, L.stream, L.sms);
-      if (r == cudaErrorNotSupported && k.ip[3] == 0)
-        r = sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, 1, L.stream, L.sms);
-      return r;
+      const int32_t variant = k.ip[3] == 0 ? 2 : (int32_t)k.ip[3];
+      return sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, variant, L.stream, L.sms, L.scr,
+                        (L.ro_mask >> 1) & 1u);
     }
     case MM_OP_CHOL_POTRF:
     case MM_OP_CHOL_TRSM:
@@ -260,6 +284,23 @@ cudaError_t launch_builtin(const Launch& L) {
 namespace {
 
 // Launch the task's kernel on logical device d.
+uint32_t readonly_mask(const App& app, const Task& t) {
+  uint32_t m = 0;
+  for (size_t i = 0; i < t.acc.size() && i < 32; ++i) {
+    bool written = false;
+    for (auto& k : app.kernels)
+      for (auto& a : k.acc)
+        if ((a.mode & MM_WRITE) && (a.buffer == t.acc[i].buffer ||
+                                    phys_buffer(app, a.buffer, 1) == t.acc[i].buffer))
+          written = true;
+    for (auto& dt : app.dag)
+      for (auto& a : dt.acc)
+        if ((a.mode & MM_WRITE) && a.buffer == t.acc[i].buffer) written = true;
+    if (!written) m |= 1u << i;
+  }
+  return m;
+}
+
 mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, void* const* buffers,
                       cudaStream_t s) {
   const Kernel& k = app.kernels[t.kernel];
@@ -273,7 +314,21 @@ mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, voi
   if (k.op == MM_OP_CUSTOM) {
     e = (cudaError_t)k.launch(k.user, d, mm_range{t.b, t.e}, opnd, (void*)s);
   } else {
-    Launch L{&k, &t, opnd, s, ctx->dev[d].sms};
+    DevRt& dv = ctx->dev[d];
+    const size_t need = builtin_scratch_bytes(k, t);
+    if (need > dv.scr.bytes) {
+      cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+      cudaStreamIsCapturing(s, &cs);
+      if (cs != cudaStreamCaptureStatusNone) MM_FAIL(MM_ESTATE, "scratch not reserved before graph capture");
+      if (dv.scr.ptr) {
+        cudaStreamSynchronize(s);
+        cudaFree(dv.scr.ptr);
+      }
+      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1};
+      if (cudaMalloc(&dv.scr.ptr, need) != cudaSuccess) MM_FAIL(MM_ENOMEM, "device scratch of %zu bytes", need);
+      dv.scr.bytes = need;
+    }
+    Launch L{&k, &t, opnd, s, dv.sms, &dv.scr, readonly_mask(app, t)};
     e = launch_builtin(L);
   }
   if (e == cudaErrorNotSupported) MM_FAIL(MM_ENOTSUP, "kernel %s (op %d) has no sm_100a implementation yet", k.name.c_str(), k.op);
@@ -316,6 +371,22 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
     CU_OK(cudaEventCreateWithFlags(&rt->fork, cudaEventDisableTiming));
     CU_OK(cudaEventCreate(&rt->t_start));
     CU_OK(cudaEventCreate(&rt->t_stop));
+  }
+  // reserve device scratch for every kernel op before any graph capture
+  for (size_t i = 0; i < plan.ops.size(); ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    if (op.kind != MM_OPK_KERNEL || !ctx->dev[op.device].mine) continue;
+    const Task& t = plan.tasks[op.task];
+    DevRt& dv = ctx->dev[op.device];
+    const size_t need = builtin_scratch_bytes(plan.app.kernels[t.kernel], t);
+    if (need > dv.scr.bytes) {
+      CU_OK(set_dev(ctx, op.device));
+      CU_OK(cudaDeviceSynchronize());
+      if (dv.scr.ptr) cudaFree(dv.scr.ptr);
+      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1};
+      CU_OK(cudaMalloc(&dv.scr.ptr, need));
+      dv.scr.bytes = need;
+    }
   }
   if (timing && rt->kev.empty()) {
     rt->kev.assign(plan.ops.size() * 2, nullptr);
@@ -656,6 +727,7 @@ void mm_ctx_destroy(mm_ctx* ctx) {
       if (r.gctx) drv().StreamDestroy((CUstream)r.stream);
       else cudaStreamDestroy(r.stream);
     }
+    if (r.scr.ptr) cudaFree(r.scr.ptr);
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);
   }
   if (ctx->comm) nccl().CommDestroy(ctx->comm);
@@ -713,6 +785,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   mm_status r = ensure_rt(ctx, plan, timing);
   if (r) return r;
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  for (auto& dv : ctx->dev) dv.scr.epoch++;   // operand-split caches are per run
   const int32_t root = first_owned(ctx);
   cudaStream_t rs = ctx->dev[root].stream;
   const size_t nbuf = plan.app.buffers.size() * (size_t)ctx->G;
@@ -827,8 +900,10 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
       CU_OK(cudaEventCreate(&a));
       CU_OK(cudaEventCreate(&b));
       auto time_task = [&](const Task& t, float* ms) -> mm_status {
+        ctx->dev[d].scr.epoch++;
         mm_status r = launch_task(ctx, app, t, d, buffers, s);  // warm-up
         if (r) return r;
+        ctx->dev[d].scr.epoch++;
         CU_OK(cudaEventRecord(a, s));
         r = launch_task(ctx, app, t, d, buffers, s);
         if (r) return r;

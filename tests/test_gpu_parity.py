@@ -144,11 +144,13 @@ def test_blackscholes(R, G, strategy):
     assert np.max(np.abs(par) / np.maximum(S, X)) < 4e-6
 
 
-@pytest.mark.parametrize("variant", [1])
+@pytest.mark.parametrize("shape", [(300, 200, 96), (257, 520, 77), (1024, 1024, 1024)])
+@pytest.mark.parametrize("variant", [1, 2])
 @pytest.mark.parametrize("G", [1, 2])
-def test_sgemm(R, variant, G):
+def test_sgemm(R, variant, G, shape):
+    """variant 1 = FFMA, 2 = tcgen05 3xTF32 (TMA + TMEM); ragged M, N, K."""
     mm, runner = R
-    M, N, K = 300, 200, 96
+    M, N, K = shape
     Ai, Bi = synthgen.matmul_integer(M, K, N)
     ref_i = on.sgemm(Ai, Bi)
     Au, Bu = synthgen.matmul_uniform(M, K, N)
