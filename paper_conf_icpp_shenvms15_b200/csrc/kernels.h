@@ -62,8 +62,12 @@ cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int6
 size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows);
 
 // Cholesky tiles (kernels_chol.cu); A tile-major, T x T tiles of b x b.
+constexpr int kCholBatch = 128;   // tasks per batched launch
 cudaError_t chol_task(int32_t op, float* A, int64_t T, int64_t b, int64_t i, int64_t j, int64_t k,
                       cudaStream_t s, int sms);
+// n independent tasks of one kernel (ijk = n triples) in one launch.
+cudaError_t chol_batch(int32_t op, float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n,
+                       cudaStream_t s, int sms);
 
 // Counter-hash generators (kernels_fill.cu) = synthgen.uniform / integers.
 cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,

@@ -185,7 +185,64 @@ struct PlanRt {
   std::vector<void*> graph_bufs;
   int64_t graph_launches = 0;
   int64_t graph_xfer = 0, graph_h2d = 0, graph_d2h = 0;
+  // DAG task batching: members[head] = kernel ops launched together with head
+  std::vector<int64_t> batch_head;               // -1: not a member of another op's batch
+  std::vector<std::vector<int64_t>> members;
 };
+
+bool is_batchable_op(int32_t op) {
+  return op == MM_OP_CHOL_TRSM || op == MM_OP_CHOL_SYRK || op == MM_OP_CHOL_GEMM;
+}
+
+// Group consecutive independent kernel ops of one device and one kernel into
+// one launch (MK-DAG steps: all TRSMs / SYRKs / GEMMs of a step on a device).
+// A member joins only if no other op of that device lies between, all of its
+// cross-stream waits point before the head, and it neither reads nor writes
+// what an earlier member writes (nor writes what an earlier member reads).
+void compute_batches(const Plan& plan, PlanRt* rt) {
+  const size_t n = plan.ops.size();
+  rt->batch_head.assign(n, -1);
+  rt->members.assign(n, {});
+  if (!plan.app.is_dag) return;
+  std::vector<int64_t> last_on_dev(plan.G, -1);   // open batch head per device
+  auto overlap = [](const TaskAcc& a, const TaskAcc& b) {
+    return a.buffer == b.buffer && a.lo < b.hi && b.lo < a.hi;
+  };
+  for (size_t i = 0; i < n; ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    if (op.kind == MM_OPK_BARRIER) {
+      std::fill(last_on_dev.begin(), last_on_dev.end(), -1);
+      continue;
+    }
+    const int32_t d = plan.op_stream[i];
+    if (op.kind != MM_OPK_KERNEL || !is_batchable_op(plan.app.kernels[op.kernel].op)) {
+      if (d >= 0) last_on_dev[d] = -1;
+      continue;
+    }
+    int64_t h = last_on_dev[d];
+    bool ok = h >= 0 && plan.ops[h].kernel == op.kernel && (int64_t)rt->members[h].size() + 1 < kCholBatch;
+    if (ok)
+      for (auto& w : plan.waits[i])
+        if (w.op >= h) ok = false;
+    if (ok) {
+      const Task& t = plan.tasks[op.task];
+      std::vector<int64_t> grp = rt->members[h];
+      grp.push_back(h);
+      for (int64_t m : grp) {
+        const Task& u = plan.tasks[plan.ops[m].task];
+        for (auto& a : t.acc)
+          for (auto& c : u.acc)
+            if (overlap(a, c) && ((a.mode & MM_WRITE) || (c.mode & MM_WRITE))) ok = false;
+      }
+    }
+    if (ok) {
+      rt->members[h].push_back((int64_t)i);
+      rt->batch_head[i] = h;
+    } else {
+      last_on_dev[d] = (int64_t)i;
+    }
+  }
+}
 
 cudaError_t set_dev(mm_ctx* ctx, int32_t d) {
   const DevRt& r = ctx->dev[d];
@@ -340,6 +397,32 @@ mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, voi
   return MM_OK;
 }
 
+// Launch a batch head together with its members (one batched kernel).
+mm_status launch_batch(mm_ctx* ctx, const Plan& plan, const PlanRt* rt, int64_t head, int32_t d,
+                       void* const* buffers, cudaStream_t s) {
+  const App& app = plan.app;
+  const Task& t0 = plan.tasks[plan.ops[head].task];
+  const Kernel& k = app.kernels[t0.kernel];
+  std::vector<int32_t> ijk;
+  auto add = [&](int64_t o) {
+    const Task& t = plan.tasks[plan.ops[o].task];
+    ijk.push_back((int32_t)t.ip[0]);
+    ijk.push_back((int32_t)t.ip[1]);
+    ijk.push_back((int32_t)t.ip[2]);
+  };
+  add(head);
+  for (int64_t m : rt->members[head]) add(m);
+  float* A = static_cast<float*>(buffers[(size_t)t0.acc[0].buffer * ctx->G + d]);
+  if (!A) MM_FAIL(MM_EINVAL, "run: buffer slot %d has no pointer on device %d", t0.acc[0].buffer, d);
+  cudaError_t e = chol_batch(k.op, A, k.ip[0], k.ip[1], ijk.data(), (int32_t)(ijk.size() / 3), s, ctx->dev[d].sms);
+  if (e != cudaSuccess) {
+    ctx->poisoned = true;
+    MM_FAIL(MM_ECUDA, "batched %s launch failed: %s", k.name.c_str(), cudaGetErrorString(e));
+  }
+  g_kernel_launches.fetch_add(1, std::memory_order_relaxed);
+  return MM_OK;
+}
+
 mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
   if (rt && rt->ctx != ctx) {
@@ -371,6 +454,7 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
     CU_OK(cudaEventCreateWithFlags(&rt->fork, cudaEventDisableTiming));
     CU_OK(cudaEventCreate(&rt->t_start));
     CU_OK(cudaEventCreate(&rt->t_stop));
+    compute_batches(plan, rt);
   }
   // reserve device scratch for every kernel op before any graph capture
   for (size_t i = 0; i < plan.ops.size(); ++i) {
@@ -460,9 +544,20 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
     }
     const int32_t d = plan.op_stream[i];
     cudaStream_t s = ctx->dev[d].stream;
+    if (op.kind == MM_OPK_KERNEL && rt->batch_head[i] >= 0) continue;  // launched with its head
     CU_OK(set_dev(ctx, d));
     for (auto& w : plan.waits[i]) CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
-    if (op.kind == MM_OPK_KERNEL) {
+    if (op.kind == MM_OPK_KERNEL && !rt->members[i].empty()) {
+      for (int64_t m : rt->members[i])
+        for (auto& w : plan.waits[m]) CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      mm_status r = launch_batch(ctx, plan, rt, (int64_t)i, d, buffers, s);
+      if (r) return r;
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      st->n_launches++;
+      for (int64_t m : rt->members[i])
+        if (plan.needs_event[m]) CU_OK(cudaEventRecord(rt->ev[m], s));
+    } else if (op.kind == MM_OPK_KERNEL) {
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
       mm_status r = launch_task(ctx, app, plan.tasks[op.task], d, buffers, s);
       if (r) return r;
@@ -533,9 +628,10 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
       continue;
     }
     if (op.kind == MM_OPK_KERNEL) {
-      if (op.device != me) continue;
+      if (op.device != me || rt->batch_head[i] >= 0) continue;
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
-      mm_status r = launch_task(ctx, app, plan.tasks[op.task], me, buffers, s);
+      mm_status r = rt->members[i].empty() ? launch_task(ctx, app, plan.tasks[op.task], me, buffers, s)
+                                            : launch_batch(ctx, plan, rt, (int64_t)i, me, buffers, s);
       if (r) return r;
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
       st->n_launches++;
@@ -845,7 +941,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     const mm_op_rec& op = plan.ops[i];
     if (op.kind != MM_OPK_KERNEL || !ctx->dev[op.device].mine) continue;
     S->kernel_launches[op.device][op.kernel]++;
-    if (timing) {
+    if (timing && rt->kev[2 * i]) {
       float k = 0.f;
       CU_OK(cudaEventElapsedTime(&k, rt->kev[2 * i], rt->kev[2 * i + 1]));
       S->kernel_ms[op.device][op.kernel] += k;

@@ -209,3 +209,49 @@ def test_hotspot_full_size_sampled_rows(R):
         # window rows at the cut are wrong after k steps only within k rows of the cut
         ref = on.hotspot_run(t_full[lo:hi], p_full[lo:hi], iters)
         assert np.array_equal(got[y], ref[y - lo]), y
+
+
+def _to_tiles(A, b):
+    n = A.shape[0]
+    T = n // b
+    return A.reshape(T, b, T, b).transpose(0, 2, 1, 3).copy()
+
+
+def _from_tiles(t, n, b):
+    T = n // b
+    return t.reshape(T, T, b, b).transpose(0, 2, 1, 3).reshape(n, n)
+
+
+@pytest.mark.parametrize("strategy", [4, 5, 6])
+@pytest.mark.parametrize("G", [1, 2, 3])
+def test_cholesky_exact_factor(R, strategy, G):
+    """MK-DAG: integer L0 (diag 32..64, band +-1), A = L0 L0^T: every FP32
+    operation is exact, so the factor must be L0 bit for bit for any schedule."""
+    mm, runner = R
+    n, b = 512, 128
+    A, L0 = synthgen.cholesky_exact_factor(n)
+    with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=G) as s:
+        assert s.classify() == mm.MM_MK_DAG
+        s.load(0, _to_tiles(A, b))
+        plan = s.plan(strategy, rand_profile(mm, G, 4, 7))
+        s.run(plan)
+        L = _from_tiles(s.collect(plan, 0), n, b)
+    assert np.array_equal(np.tril(L), L0)
+    T = n // b
+    for k in range(T):   # diagonal tiles: strictly upper part zeroed
+        blk = L[k * b:(k + 1) * b, k * b:(k + 1) * b]
+        assert np.all(np.triu(blk, 1) == 0)
+
+
+@pytest.mark.parametrize("nb", [(512, 128), (1024, 256)])
+def test_cholesky_random_spd(R, nb):
+    mm, runner = R
+    n, b = nb
+    A = synthgen.spd_random(n)
+    ref = on.cholesky(A.astype(np.float64))
+    with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=2) as s:
+        s.load(0, _to_tiles(A, b))
+        plan = s.plan(4, rand_profile(mm, 2, 4, 8))
+        s.run(plan, use_graph=True)
+        L = np.tril(_from_tiles(s.collect(plan, 0), n, b)).astype(np.float64)
+    assert np.max(np.abs(L - ref)) / np.max(np.abs(ref)) <= 1e-4
