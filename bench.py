@@ -45,10 +45,16 @@ APPS = {
                      "SK-One BlackScholes 80,530,632 options (P311)"),
     "sgemm": ("MM_APP_SGEMM", [6144, 6144, 6144, 0], lambda p: 2 * p[0] * p[1] * p[2],
               "SK-One MatrixMul 6144^2 FP32 (P311)"),
+    "matmul1k": ("MM_APP_SGEMM", [1024, 1024, 1024, 0], lambda p: 2 * p[0] * p[1] * p[2],
+                 "SK-One MatrixMul 1024^2 FP32 (BASELINE configs[0])"),
+    "cholesky": ("MM_APP_CHOLESKY", [32768, 1024], lambda p: p[0] ** 3 / 3,
+                 "MK-DAG tiled Cholesky 32768^2 FP32, tile 1024 (BASELINE configs[4])"),
 }
+FLOP_APPS = ("sgemm", "matmul1k", "cholesky")
 # kernel whose roofline is reported, and its algorithmic bytes per item
 DOMINANT = {"stream": ("triad", 12), "stream-loop": ("triad", 12), "hotspot": ("hotspot", None),
-            "stencil": ("stencil", None), "blackscholes": ("blackscholes", 20), "sgemm": ("sgemm", None)}
+            "stencil": ("stencil", None), "blackscholes": ("blackscholes", 20), "sgemm": ("sgemm", None),
+            "matmul1k": ("sgemm", None), "cholesky": ("gemm", None)}
 
 
 def load_peaks():
@@ -284,7 +290,7 @@ def main():
     ms_step = ms_total / args.steps
     value = algo_bytes / (ms_step * 1e-3) / 1e9
     unit = "GB/s"
-    if args.app == "sgemm":
+    if args.app in FLOP_APPS:
         value = algo_bytes / (ms_step * 1e-3) / 1e12
         unit = "TFLOP/s"
 
@@ -293,19 +299,28 @@ def main():
     # kernel ids of the builtin apps in program order
     kname_map = {"stream": ["copy", "scale", "add", "triad"], "stream-loop": ["copy", "scale", "add", "triad"],
                  "hotspot": ["hotspot"], "stencil": ["stencil", "residual"], "blackscholes": ["blackscholes"],
-                 "sgemm": ["sgemm"]}[args.app]
+                 "sgemm": ["sgemm"], "matmul1k": ["sgemm"],
+                 "cholesky": ["potrf", "trsm", "syrk", "gemm"]}[args.app]
     kid = kname_map.index(dom)
     my = [d for d in range(G) if sess.mine[d]]
     dom_ms = sum(kms[d][kid] for d in my)
     dom_launch = sum(st.kernel_launches[d][kid] for d in my) * args.steps
     items = sum(info.items[d][kid] for d in my)
     if bpi is None:
-        bpi = {"hotspot": 12 * iparam[1], "stencil": 12 * iparam[1], "sgemm": None}[args.app]
+        bpi = {"hotspot": 12 * iparam[1], "stencil": 12 * iparam[1]}.get(args.app)
     roof = None
     if dom_launch and dom_ms > 0:
         per_launch_ms = dom_ms / dom_launch
         launches_per_step = dom_launch / args.steps
-        if args.app == "sgemm":
+        if args.app == "cholesky":
+            # FFMA tile update: FP32 FMA pipe peak = 148 SM x 128 lanes x 2 flop x 1.965 GHz
+            b = iparam[1]
+            ach = 2 * b ** 3 * items * args.steps / (dom_ms * 1e-3) / 1e12
+            pk = 148 * 128 * 2 * 1.965e9 / 1e12
+            roof = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
+                    "traffic": None, "kernel": "gemm tile update (FFMA, batched per step)",
+                    "peak_kind": "derived: 148 SMs x 128 FP32 lanes x 2 x 1.965 GHz (B200_PROFILING clocks)"}
+        elif args.app in ("sgemm", "matmul1k"):
             # 3xTF32: FP32-equivalent flops; peak = measured bf16 x 0.5 (nominal
             # tf32/bf16 dense ratio) / 3 (three tf32 MMAs per FP32 product)
             fl = 2 * iparam[1] * iparam[2] * items / launches_per_step
@@ -363,6 +378,8 @@ def main():
         del host
     except Exception as ex:  # report, never hide
         e2e = {"value": None, "unit": unit, "error": str(ex)[:200]}
+    if args.app == "cholesky":
+        ranked = list(ranked) + [mm.MM_SP_CYCLIC]   # static comparator (P201; BASELINE configs[4])
 
     # --- every Table I strategy for this class, w/o and w/ sync (ranking) ----
     strategies = {}

@@ -299,6 +299,11 @@ mm_status mm_fill_uniform(mm_ctx* ctx, int32_t d, float* dst, int64_t n, uint64_
 /* Integer variant (values as float32): lo + (h24 % (hi-lo+1)). */
 mm_status mm_fill_integers(mm_ctx* ctx, int32_t d, float* dst, int64_t n, uint64_t seed,
                            int32_t array_id, int64_t start, int32_t lo, int32_t hi);
+/* = synthgen.spd_random(n) in the Cholesky app's tile-major layout (tile size
+ * b): A = (S + S^T)/2 + n I with S[r][c] = u(seed, array_id, r*n + c),
+ * evaluated in FP64 and rounded once to FP32. */
+mm_status mm_fill_spd_tiles(mm_ctx* ctx, int32_t d, float* dst, int64_t n, int64_t b, uint64_t seed,
+                            int32_t array_id);
 
 typedef struct {
   int64_t probe_items;       /* 0 = per kernel, >= 4 waves */

@@ -74,5 +74,6 @@ cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id,
                          float lo, float hi, cudaStream_t s);
 cudaError_t fill_integers(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
                           int32_t lo, int32_t hi, cudaStream_t s);
+cudaError_t fill_spd_tiles(float* dst, int64_t n, int64_t b, uint64_t seed, int32_t array_id, cudaStream_t s);
 
 }  // namespace mm

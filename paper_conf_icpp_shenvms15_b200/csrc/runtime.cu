@@ -868,6 +868,17 @@ mm_status mm_fill_integers(mm_ctx* ctx, int32_t d, float* dst, int64_t n, uint64
   return MM_OK;
 }
 
+mm_status mm_fill_spd_tiles(mm_ctx* ctx, int32_t d, float* dst, int64_t n, int64_t b, uint64_t seed,
+                            int32_t array_id) {
+  if (!ctx || d < 0 || d >= ctx->G || !ctx->dev[d].mine || !dst || n <= 0 || b <= 0 || n % b)
+    MM_FAIL(MM_EINVAL, "fill_spd_tiles: bad arguments");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  CU_OK(set_dev(ctx, d));
+  CU_OK(fill_spd_tiles(dst, n, b, seed, array_id, ctx->dev[d].stream));
+  CU_OK(cudaStreamSynchronize(ctx->dev[d].stream));
+  return MM_OK;
+}
+
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_run_opts* o, mm_run_stats* st) {
   if (!ctx || !plan_h || !buffers) MM_FAIL(MM_EINVAL, "run: null argument");
   if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
@@ -941,7 +952,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     const mm_op_rec& op = plan.ops[i];
     if (op.kind != MM_OPK_KERNEL || !ctx->dev[op.device].mine) continue;
     S->kernel_launches[op.device][op.kernel]++;
-    if (timing && rt->kev[2 * i]) {
+    if (timing && rt->kev[2 * i] && rt->batch_head[i] < 0) {   // batch members: timed with their head
       float k = 0.f;
       CU_OK(cudaEventElapsedTime(&k, rt->kev[2 * i], rt->kev[2 * i + 1]));
       S->kernel_ms[op.device][op.kernel] += k;

@@ -174,6 +174,7 @@ _SIGS = {
                         C.c_float],
     "mm_fill_integers": [_P, C.c_int32, C.c_void_p, C.c_int64, C.c_uint64, C.c_int32, C.c_int64, C.c_int32,
                          C.c_int32],
+    "mm_fill_spd_tiles": [_P, C.c_int32, C.c_void_p, C.c_int64, C.c_int64, C.c_uint64, C.c_int32],
     "mm_profile_run": [_P, _P, C.POINTER(_P), C.POINTER(mm_profile_opts), C.POINTER(mm_profile)],
     "mm_run": [_P, _P, C.POINTER(_P), C.POINTER(mm_run_opts), C.POINTER(mm_run_stats)],
     "mm_collect": [_P, _P, C.POINTER(_P), C.c_int32, C.c_void_p, C.c_int32],
@@ -477,6 +478,10 @@ def mm_fill_uniform(ctx: int, d: int, ptr: int, n: int, seed: int, array_id: int
 def mm_fill_integers(ctx: int, d: int, ptr: int, n: int, seed: int, array_id: int, start: int,
                      lo: int, hi: int):
     _call("mm_fill_integers", ctx, d, ptr, n, seed, array_id, start, lo, hi)
+
+
+def mm_fill_spd_tiles(ctx: int, d: int, ptr: int, n: int, b: int, seed: int, array_id: int):
+    _call("mm_fill_spd_tiles", ctx, d, ptr, n, b, seed, array_id)
 
 
 def _ptr_array(ptrs: Sequence[int]):

@@ -66,6 +66,7 @@ class Session:
                     self.bufs[(s, d)] = torch.empty(max(n, 1), dtype=_DT[eb],
                                                     device=f"cuda:{cuda_devices[d]}")
         self.plans: List[int] = []
+        self.tile = 0   # Cholesky tile size (set by session())
 
     # -- memory ------------------------------------------------------------
     def ptrs(self) -> List[int]:
@@ -79,6 +80,14 @@ class Session:
     def fill(self, integer: bool = False, seed: int = synthgen.SEED, recipe=None):
         """Generate the app's inputs in place on every owned device (resident
         mode) with the device counter hash (= synthgen)."""
+        if self.app_id == mm.MM_APP_CHOLESKY and recipe is None:
+            _, nn = mm.mm_app_buffer_info(self.app, 0)
+            n = int(round(nn ** 0.5))
+            for d in range(self.G):
+                if self.mine[d]:
+                    mm.mm_fill_spd_tiles(self.ctx, d, self.bufs[(0, d)].data_ptr(), n, self.tile, seed,
+                                         synthgen.AID_CHOL_S)
+            return
         rec = recipe or (RECIPES_INT if integer else RECIPES).get(self.app_id, {})
         for slot, r in rec.items():
             for d in range(self.G):
@@ -156,4 +165,7 @@ def builtin(app_id: int, iparam: Sequence[int] = (), fparam: Sequence[float] = (
 
 
 def session(app_id: int, iparam: Sequence[int] = (), fparam: Sequence[float] = (), **kw) -> Session:
-    return Session(builtin(app_id, iparam, fparam), app_id=app_id, **kw)
+    s = Session(builtin(app_id, iparam, fparam), app_id=app_id, **kw)
+    if app_id == mm.MM_APP_CHOLESKY:
+        s.tile = int(iparam[1]) if len(iparam) > 1 and iparam[1] else 1024
+    return s

@@ -255,3 +255,12 @@ def test_cholesky_random_spd(R, nb):
         s.run(plan, use_graph=True)
         L = np.tril(_from_tiles(s.collect(plan, 0), n, b)).astype(np.float64)
     assert np.max(np.abs(L - ref)) / np.max(np.abs(ref)) <= 1e-4
+
+
+def test_cholesky_device_spd_generator(R):
+    mm, runner = R
+    n, b = 384, 128
+    with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=1) as s:
+        s.fill()
+        got = s.bufs[(0, 0)].cpu().numpy()
+    assert np.array_equal(got, _to_tiles(synthgen.spd_random(n), b).reshape(-1))
