@@ -195,7 +195,7 @@ typedef struct {
   int32_t G, K;
   int32_t staged;                            /* 1: host-resident inputs (R_GD term) */
   int32_t _pad;
-  uint64_t ps_item[MM_MAX_DEV][MM_MAX_K];    /* picoseconds per item (R_GC)   */
+  uint64_t fs_item[MM_MAX_DEV][MM_MAX_K];    /* femtoseconds per item (R_GC)  */
   uint64_t chunk_est_ns[MM_MAX_DEV][MM_MAX_K]; /* DP-Perf estimate per nominal chunk */
   uint64_t link_Bps[MM_MAX_DEV];             /* bytes/s into device d (R_GD)  */
 } mm_profile;

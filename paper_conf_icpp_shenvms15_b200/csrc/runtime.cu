@@ -1037,14 +1037,14 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
           std::sort(v.begin(), v.end());
           const uint64_t ns = std::max<uint64_t>(1, (uint64_t)(v[reps / 2] * 1e6));
           out->chunk_est_ns[d][k] = ns;
-          out->ps_item[d][k] = ns * 1000;
+          out->fs_item[d][k] = ns * 1000000;
           continue;
         }
         // probe: the even share n/G (>= one wave of the kernel), median of reps
         int64_t probe = po && po->probe_items > 0 ? po->probe_items : chunk_size(kern.n, kern.granule, G);
         probe = std::min<int64_t>(std::max<int64_t>(probe, std::min(kern.n, kern.min_items)), kern.n);
         if (probe <= 0) {
-          out->ps_item[d][k] = 1;
+          out->fs_item[d][k] = 1;
           out->chunk_est_ns[d][k] = 1;
           continue;
         }
@@ -1055,21 +1055,31 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
           if (r) return r;
         }
         std::sort(v.begin(), v.end());
-        out->ps_item[d][k] = std::max<uint64_t>(1, (uint64_t)((double)v[reps / 2] * 1e9 / (double)probe));
-        // DP-Perf warm-up: `warm` nominal chunks on this device (P311)
+        out->fs_item[d][k] = std::max<uint64_t>(1, (uint64_t)((double)v[reps / 2] * 1e12 / (double)probe));
+        // DP-Perf warm-up (P311): `warm` nominal chunks on this device, issued
+        // back to back as a dynamic schedule would, timed together (per-chunk
+        // cost at the device's issue rate, launch latency amortised).
         const int64_t cs = chunk_size(kern.n, kern.granule, (int64_t)kpd * G);
-        double sum = 0.0;
-        int32_t cnt = 0;
+        std::vector<Task> ch;
         for (int32_t i = 0; i < warm; ++i) {
           const int64_t b0 = std::min<int64_t>((int64_t)i * cs, std::max<int64_t>(0, kern.n - cs));
-          Task c = range_task(app, k, 0, b0, std::min(kern.n, b0 + cs), 0);
-          float ms = 0.f;
-          mm_status r = time_task(c, &ms);
-          if (r) return r;
-          sum += ms;
-          cnt++;
+          ch.push_back(range_task(app, k, 0, b0, std::min(kern.n, b0 + cs), 0));
         }
-        out->chunk_est_ns[d][k] = std::max<uint64_t>(1, (uint64_t)(sum / cnt * 1e6));
+        {
+          mm_status r = launch_task(ctx, app, ch[0], d, buffers, s);  // warm-up launch
+          if (r) return r;
+          ctx->dev[d].scr.epoch++;
+          CU_OK(cudaEventRecord(a, s));
+          for (auto& c : ch) {
+            r = launch_task(ctx, app, c, d, buffers, s);
+            if (r) return r;
+          }
+          CU_OK(cudaEventRecord(b, s));
+          CU_OK(cudaEventSynchronize(b));
+          float ms = 0.f;
+          CU_OK(cudaEventElapsedTime(&ms, a, b));
+          out->chunk_est_ns[d][k] = std::max<uint64_t>(1, (uint64_t)((double)ms * 1e6 / (double)ch.size()));
+        }
       }
       // link: bytes/s of a 64 MiB device-to-device copy into d
       {
@@ -1099,7 +1109,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
     const int32_t me = first_owned(ctx);
     const size_t rowlen = 2 * MM_MAX_K + 1;
     for (int32_t k = 0; k < MM_MAX_K; ++k) {
-      row[k] = out->ps_item[me][k];
+      row[k] = out->fs_item[me][k];
       row[MM_MAX_K + k] = out->chunk_est_ns[me][k];
     }
     row[2 * MM_MAX_K] = out->link_Bps[me];
@@ -1117,7 +1127,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
     for (int32_t d = 0; d < G; ++d) {
       const uint64_t* rr = all.data() + (size_t)ctx->dev[d].rank * rowlen;
       for (int32_t k = 0; k < MM_MAX_K; ++k) {
-        out->ps_item[d][k] = rr[k];
+        out->fs_item[d][k] = rr[k];
         out->chunk_est_ns[d][k] = rr[MM_MAX_K + k];
       }
       out->link_Bps[d] = rr[2 * MM_MAX_K];

@@ -77,7 +77,7 @@ class mm_app_params(C.Structure):
 
 class mm_profile(C.Structure):
     _fields_ = [("G", C.c_int32), ("K", C.c_int32), ("staged", C.c_int32), ("_pad", C.c_int32),
-                ("ps_item", (C.c_uint64 * MM_MAX_K) * MM_MAX_DEV),
+                ("fs_item", (C.c_uint64 * MM_MAX_K) * MM_MAX_DEV),
                 ("chunk_est_ns", (C.c_uint64 * MM_MAX_K) * MM_MAX_DEV),
                 ("link_Bps", C.c_uint64 * MM_MAX_DEV)]
 
@@ -335,15 +335,15 @@ def mm_rank(cls: int, needs_sync: bool) -> List[int]:
     return list(out[:n.value])
 
 
-def make_profile(G: int, ps_item, chunk_est_ns=None, link_Bps=None, staged: bool = False) -> mm_profile:
-    """Marshal a profile from nested lists ps_item[d][k] (ps), chunk_est_ns[d][k], link_Bps[d]."""
+def make_profile(G: int, fs_item, chunk_est_ns=None, link_Bps=None, staged: bool = False) -> mm_profile:
+    """Marshal a profile from nested lists fs_item[d][k] (fs), chunk_est_ns[d][k], link_Bps[d]."""
     p = mm_profile()
     p.G = G
     p.K = MM_MAX_K
     p.staged = int(staged)
     for d in range(G):
-        for k, v in enumerate(ps_item[d]):
-            p.ps_item[d][k] = int(v)
+        for k, v in enumerate(fs_item[d]):
+            p.fs_item[d][k] = int(v)
         if chunk_est_ns is not None:
             for k, v in enumerate(chunk_est_ns[d]):
                 p.chunk_est_ns[d][k] = int(v)

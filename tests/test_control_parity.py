@@ -54,7 +54,7 @@ def rand_profile(rnd, G, K, equal=False):
         ps = [ps[0]] * G
         est = [est[0]] * G
         link = [link[0]] * G
-    po = oc.Profile(G=G, ps_item=ps, chunk_est_ns=est, link_Bps=link)
+    po = oc.Profile(G=G, fs_item=ps, chunk_est_ns=est, link_Bps=link)
     pc = mm.make_profile(G, ps, est, link)
     return pc, po
 

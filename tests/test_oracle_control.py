@@ -186,7 +186,7 @@ def test_split_decision_drops_slow_device():
 
 def test_sp_unified_vs_varied():
     app = apps.stream(1 << 12, 1)
-    prof = oc.Profile(G=2, ps_item=[[10, 20, 30, 40], [20, 20, 20, 20]],
+    prof = oc.Profile(G=2, fs_item=[[10, 20, 30, 40], [20, 20, 20, 20]],
                       chunk_est_ns=[[1] * 4] * 2, link_Bps=[10 ** 9] * 2)
     u = oc.sp_split(app, prof, oc.SP_UNIFIED)
     assert all(r == u[0] for r in u)
@@ -200,7 +200,7 @@ def test_sp_unified_vs_varied():
 def test_staged_unified_mk_loop_drops_transfer():
     # P549: "the data transfer is not profiled" for MK-Loop SP-Unified.
     seq, loop = apps.stream(1 << 12, 1), apps.stream(1 << 12, 10)
-    prof = oc.Profile(G=2, ps_item=[[10] * 4, [40] * 4], chunk_est_ns=[[1] * 4] * 2,
+    prof = oc.Profile(G=2, fs_item=[[10] * 4, [40] * 4], chunk_est_ns=[[1] * 4] * 2,
                       link_Bps=[10 ** 9, 10 ** 15], staged=True)
     s = oc.sp_split(seq, prof, oc.SP_UNIFIED)[0]
     l = oc.sp_split(loop, prof, oc.SP_UNIFIED)[0]
@@ -210,7 +210,7 @@ def test_staged_unified_mk_loop_drops_transfer():
 # ------------------------------------------------------------- c4 DP-Perf --
 def test_dp_perf_identical_devices_round_robin():
     app = apps.single("bs", 1 << 14)
-    prof = oc.Profile(G=4, ps_item=[[1]] * 4, chunk_est_ns=[[1000]] * 4, link_Bps=[10 ** 9] * 4)
+    prof = oc.Profile(G=4, fs_item=[[1]] * 4, chunk_est_ns=[[1000]] * 4, link_Bps=[10 ** 9] * 4)
     tasks, dev, _ = oc.dp_perf(app, prof, 8)
     assert len(tasks) == 32
     assert dev == [i % 4 for i in range(32)]
@@ -219,7 +219,7 @@ def test_dp_perf_identical_devices_round_robin():
 def test_dp_perf_slow_device_gets_nothing():
     # P329: DP-Perf assigns all MatrixMul task instances to the (much faster) GPU.
     app = apps.single("mm", 6144, granule=1)
-    prof = oc.Profile(G=2, ps_item=[[1], [1]], chunk_est_ns=[[1000], [10 ** 9]], link_Bps=[1] * 2)
+    prof = oc.Profile(G=2, fs_item=[[1], [1]], chunk_est_ns=[[1000], [10 ** 9]], link_Bps=[1] * 2)
     _, dev, _ = oc.dp_perf(app, prof, 8)
     assert set(dev) == {0}
 
@@ -229,7 +229,7 @@ def test_dp_perf_ratio_matches_sp_single():
     n, k = 1 << 16, 16
     for ratio in (2, 3, 5):
         app = apps.single("bs", n)
-        prof = oc.Profile(G=2, ps_item=[[100], [100 * ratio]],
+        prof = oc.Profile(G=2, fs_item=[[100], [100 * ratio]],
                           chunk_est_ns=[[1000], [1000 * ratio]], link_Bps=[10 ** 9] * 2)
         _, dev, _ = oc.dp_perf(app, prof, k)
         cs = oc.chunk_size(n, 32, 2 * k)
@@ -241,7 +241,7 @@ def test_dp_perf_respects_dependencies_hand_schedule():
     # 2 devices, STREAM with 2 chunks per kernel (k=1); est 10 ns per chunk,
     # link so slow that moving data never pays: each chain stays put.
     app = apps.stream(64, 1)
-    prof = oc.Profile(G=2, ps_item=[[1] * 4] * 2, chunk_est_ns=[[10] * 4] * 2, link_Bps=[1, 1])
+    prof = oc.Profile(G=2, fs_item=[[1] * 4] * 2, chunk_est_ns=[[10] * 4] * 2, link_Bps=[1, 1])
     tasks, dev, fin = oc.dp_perf(app, prof, 1)
     assert dev == [0, 1] * 4
     assert fin == [10, 10, 20, 20, 30, 30, 40, 40]
@@ -306,7 +306,7 @@ def _interval_resync(P, Q, halo, nb):
 def test_sp_varied_resync_matches_interval_formula():
     n = 1000
     app = apps.stream(n, 1)
-    prof = oc.Profile(G=3, ps_item=[[10, 30, 20, 10], [20, 10, 20, 30], [30, 20, 10, 20]],
+    prof = oc.Profile(G=3, fs_item=[[10, 30, 20, 10], [20, 10, 20, 30], [30, 20, 10, 20]],
                       chunk_est_ns=[[1] * 4] * 3, link_Bps=[10 ** 9] * 3)
     ranges = oc.sp_split(app, prof, oc.SP_VARIED)
     tasks, dev = oc.sp_tasks(app, ranges)
@@ -321,7 +321,7 @@ def test_sp_varied_resync_matches_interval_formula():
 
 def test_sp_unified_no_transfers():
     app = apps.stream(1000, 3)
-    prof = oc.Profile(G=4, ps_item=[[7, 9, 11, 13]] * 4, chunk_est_ns=[[1] * 4] * 4,
+    prof = oc.Profile(G=4, fs_item=[[7, 9, 11, 13]] * 4, chunk_est_ns=[[1] * 4] * 4,
                       link_Bps=[10 ** 9] * 4)
     ranges = oc.sp_split(app, prof, oc.SP_UNIFIED)
     tasks, dev = oc.sp_tasks(app, ranges)
@@ -333,7 +333,7 @@ def test_sp_unified_no_transfers():
 def test_hotspot_halo_rows():
     rows, cols, iters, G = 40, 8, 5, 4
     app = apps.hotspot(rows, cols, iters)
-    prof = oc.Profile(G=G, ps_item=[[5]] * G, chunk_est_ns=[[1]] * G, link_Bps=[10 ** 9] * G)
+    prof = oc.Profile(G=G, fs_item=[[5]] * G, chunk_est_ns=[[1]] * G, link_Bps=[10 ** 9] * G)
     ranges = oc.sp_split(app, prof, oc.SP_SINGLE)
     assert [e - b for b, e in ranges[0]] == [10] * 4
     tasks, dev = oc.sp_tasks(app, ranges)

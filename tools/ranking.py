@@ -1,0 +1,144 @@
+"""E6: does the paper's Table I ranking hold on B200?  (PAPER.md P549, P565)
+
+Runs every Table I strategy of each application class on
+  * HET-2: two logical devices on one B200, a "GPU" of 132 SMs and a "CPU" of
+    16 SMs (CUDA green contexts) — 148/16 = 9.25, the K20m/E5-2620 SP peak
+    ratio of Table III is 3519.3/384 = 9.16 (P277-281);
+  * HOMO-2: two logical devices of the whole GPU each (identical processors),
+in resident mode (inputs in HBM) and, for the transfer-dominated MK apps,
+staged mode (inputs on the host, P119 H2D/D2H in the run; the paper's regime).
+
+Writes one JSON document (default profiles/r1_ranking.json): per config the
+median device time of every strategy, the devices' item shares, and whether
+the measured order satisfies Propositions 1-3 (ties within 3% count as "=").
+
+    python tools/ranking.py [--out FILE] [--reps 3] [--quick]
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_icpp_shenvms15_b200 import mm, runner  # noqa: E402
+
+TOL = 0.03
+
+# (name, builtin id, iparam) — paper sizes where they fit (P311, P319, P473)
+APPS = [
+    ("MatrixMul 6144^2 (SK-One)", mm.MM_APP_SGEMM, [6144, 6144, 6144, 0, 128, 128]),
+    ("BlackScholes 80,530,632 (SK-One)", mm.MM_APP_BLACKSCHOLES, [80530632, 32, 4096]),
+    ("HotSpot 8192^2 x 100 (SK-Loop)", mm.MM_APP_HOTSPOT, [8192, 8192, 100, 1, 64]),
+    ("STREAM-Seq 62,914,560 w/o sync (MK-Seq)", mm.MM_APP_STREAM, [62914560, 1, 0, 32, 4096]),
+    ("STREAM-Seq 62,914,560 w sync (MK-Seq)", mm.MM_APP_STREAM, [62914560, 1, 1, 32, 4096]),
+    ("STREAM-Loop x10 w/o sync (MK-Loop)", mm.MM_APP_STREAM, [62914560, 10, 0, 32, 4096]),
+    ("STREAM-Loop x10 w sync (MK-Loop)", mm.MM_APP_STREAM, [62914560, 10, 1, 32, 4096]),
+    ("stencil+reduction 8192^2 x 20 w sync (MK-Loop)", mm.MM_APP_STENCIL_REDUCTION, [8192, 8192, 20, 2, 1, 64]),
+    ("Cholesky 8192^2 tile 512 (MK-DAG)", mm.MM_APP_CHOLESKY, [8192, 512]),
+]
+
+
+def expected_order(cls, sync):
+    return mm.mm_rank(cls, sync)
+
+
+def verdict(order, times):
+    """Every adjacent pair of the expected order must satisfy t[a] <= t[b]*(1+TOL)."""
+    ok = True
+    pairs = []
+    for a, b in zip(order, order[1:]):
+        ta, tb = times.get(a), times.get(b)
+        if ta is None or tb is None:
+            continue
+        holds = ta <= tb * (1 + TOL)
+        pairs.append({"better": mm.mm_strategy_name(a), "worse": mm.mm_strategy_name(b),
+                      "ms": [round(ta, 4), round(tb, 4)], "holds": holds})
+        ok &= holds
+    return ok, pairs
+
+
+def run_config(name, app_id, ip, budgets, staged, reps):
+    s = runner.session(app_id, ip, G=2, sm_budgets=budgets)
+    try:
+        cls = s.classify()
+        ns = mm.mm_needs_sync(s.app)
+        order = expected_order(cls, ns)
+        prof = s.profile(reps=3)
+        if staged:
+            prof.staged = 1
+        s.fill()
+        host = None
+        if staged:
+            host = []
+            for slot in range(s.nbuf):
+                eb, n = mm.mm_app_buffer_info(s.app, slot)
+                h = torch.empty(max(n, 1), dtype=runner._DT[eb], pin_memory=True)
+                h.copy_(s.bufs[(slot, 0)].cpu())
+                host.append(h)
+        times, shares = {}, {}
+        strategies = list(order) + ([mm.MM_SP_CYCLIC] if cls == mm.MM_MK_DAG else [])
+        for st in strategies:
+            p = s.plan(st, prof, staged=staged)
+            kw = {"host": [h.data_ptr() for h in host]} if staged else {}
+            s.run(p, **kw)
+            ts = []
+            for _ in range(reps):
+                r = s.run(p, **kw)
+                ts.append(r.device_ms)
+            times[st] = statistics.median(ts)
+            info = mm.mm_plan_info(p)
+            tot = [sum(info.items[d][k] for k in range(s.K)) for d in range(2)]
+            shares[mm.mm_strategy_name(st)] = [round(x / max(1, sum(tot)), 4) for x in tot]
+        ok, pairs = verdict(order, times)
+        return {"app": name, "class": mm.mm_class_name(cls), "needs_sync": ns, "mode": "staged" if staged else "resident",
+                "sms": [mm.mm_ctx_sm_count(s.ctx, 0), mm.mm_ctx_sm_count(s.ctx, 1)],
+                "expected_order": [mm.mm_strategy_name(x) for x in order],
+                "ms": {mm.mm_strategy_name(k): round(v, 4) for k, v in times.items()},
+                "measured_order": [mm.mm_strategy_name(k) for k, _ in sorted(times.items(), key=lambda kv: kv[1])],
+                "share_per_device": shares, "ranking_holds": ok, "pairs": pairs,
+                "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(2)],
+                "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(2)]}
+    finally:
+        s.close()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r1_ranking.json"))
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--quick", action="store_true")
+    args = ap.parse_args()
+    torch.cuda.set_device(0)
+    res = {"platforms": {"HET-2": [0, 16], "HOMO-2": None}, "tolerance": TOL, "configs": []}
+    t0 = time.time()
+    for pname, budgets in (("HET-2", [0, 16]), ("HOMO-2", [0, 0])):
+        for name, app_id, ip in APPS:
+            modes = [False]
+            if app_id == mm.MM_APP_STREAM and not args.quick:
+                modes.append(True)
+            for staged in modes:
+                try:
+                    r = run_config(name, app_id, ip, budgets, staged, args.reps)
+                except Exception as e:  # report, never hide
+                    r = {"app": name, "mode": "staged" if staged else "resident", "error": str(e)[:300]}
+                r["platform"] = pname
+                res["configs"].append(r)
+                print(json.dumps({k: r.get(k) for k in ("platform", "app", "mode", "ms", "ranking_holds",
+                                                         "share_per_device", "error")}), flush=True)
+    res["wall_s"] = round(time.time() - t0, 1)
+    held = [c.get("ranking_holds") for c in res["configs"] if "ranking_holds" in c]
+    res["summary"] = {"configs": len(res["configs"]), "ranking_holds": sum(bool(h) for h in held),
+                      "ranking_violated": sum(not h for h in held)}
+    with open(args.out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps(res["summary"]))
+
+
+if __name__ == "__main__":
+    main()
