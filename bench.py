@@ -313,13 +313,14 @@ def main():
         per_launch_ms = dom_ms / dom_launch
         launches_per_step = dom_launch / args.steps
         if args.app == "cholesky":
-            # FFMA tile update: FP32 FMA pipe peak = 148 SM x 128 lanes x 2 flop x 1.965 GHz
+            # trailing GEMM updates on tcgen05 (3xTF32): FP32-equivalent flops vs
+            # measured bf16 x 0.5 (tf32) / 3
             b = iparam[1]
             ach = 2 * b ** 3 * items * args.steps / (dom_ms * 1e-3) / 1e12
-            pk = 148 * 128 * 2 * 1.965e9 / 1e12
-            roof = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
-                    "traffic": None, "kernel": "gemm tile update (FFMA, batched per step)",
-                    "peak_kind": "derived: 148 SMs x 128 FP32 lanes x 2 x 1.965 GHz (B200_PROFILING clocks)"}
+            pk = tf_peak * 0.5 / 3.0
+            roof = {"bound": "tensor", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
+                    "traffic": None, "kernel": "gemm tile updates (3xTF32 tcgen05, batched per step)",
+                    "peak_kind": peak_kind + " bf16_tflops x 0.5 (tf32) / 3 (3xTF32)"}
         elif args.app in ("sgemm", "matmul1k"):
             # 3xTF32: FP32-equivalent flops; peak = measured bf16 x 0.5 (nominal
             # tf32/bf16 dense ratio) / 3 (three tf32 MMAs per FP32 product)
@@ -417,6 +418,8 @@ def main():
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}"},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
             "clocks": clk.summary(), "strategies_ms": strategies,
+            "kernel_ms_per_step": {kname_map[k]: round(sum(kms[d][k] for d in my) / args.steps, 4)
+                                   for k in range(K)},
             "ranking": [mm.mm_strategy_name(s) for s in ranked],
         }
         print(json.dumps(line), flush=True)

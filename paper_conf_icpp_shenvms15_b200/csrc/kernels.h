@@ -3,6 +3,7 @@
 
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <vector>
 
 namespace mm {
 
@@ -19,6 +20,7 @@ struct Scratch {
   int64_t b_K = 0, b_N = 0;
   uint64_t b_epoch = 0;
   uint64_t epoch = 1;
+  std::vector<uint64_t> panel;   // Cholesky: split tag (epoch, step) per panel slot
 };
 
 struct Launch {
@@ -67,7 +69,11 @@ cudaError_t chol_task(int32_t op, float* A, int64_t T, int64_t b, int64_t i, int
                       cudaStream_t s, int sms);
 // n independent tasks of one kernel (ijk = n triples) in one launch.
 cudaError_t chol_batch(int32_t op, float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n,
-                       cudaStream_t s, int sms);
+                       cudaStream_t s, int sms, Scratch* scr);
+// 3xTF32 tcgen05 trailing update (kernels_gemm_tc.cu); b % 256 == 0
+size_t chol_tc_scratch(int64_t T, int64_t b);
+cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n, cudaStream_t s,
+                           Scratch* scr);
 
 // Counter-hash generators (kernels_fill.cu) = synthgen.uniform / integers.
 cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,

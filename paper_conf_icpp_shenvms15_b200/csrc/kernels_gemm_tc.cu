@@ -19,6 +19,8 @@
 //     MMA; tcgen05.commit frees a stage and signals the epilogue.
 #include <cuda.h>
 
+#include <algorithm>
+
 #include "kernels.h"
 
 namespace mm {
@@ -34,6 +36,16 @@ constexpr int B_BYTES = BN * BK * 4;                 // 32 KB
 constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
 constexpr int SMEM_BYTES = kStages * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 constexpr int kThreadsGemm = 192;
+
+// Batched Cholesky trailing update (mode 1): task z updates tile (ti, tj) of a
+// tile-major matrix, C_tile -= P_i P_j^T, with the split panel tiles at rows
+// slot*b of the hi/lo panel buffers.
+struct GemmJob {
+  int32_t mode;            // 0: rows of a plain SGEMM, 1: Cholesky tile batch
+  int32_t n;
+  int64_t T, b;
+  int32_t ti[kCholBatch], tj[kCholBatch];
+};
 
 __device__ __forceinline__ uint32_t saddr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -81,7 +93,8 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
 __global__ void __launch_bounds__(kThreadsGemm, 1)
     gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
                 const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
-                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb) {
+                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb,
+                const __grid_constant__ GemmJob job) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full = reinterpret_cast<uint64_t*>(base + kStages * STAGE_BYTES);
@@ -90,6 +103,14 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int m_blk = blockIdx.y, n_blk = blockIdx.x;
+  // operand row coordinates in the tensor maps, and the output tile
+  int32_t ya = m_blk * BM, yb = n_blk * BN;
+  if (job.mode == 1) {
+    const int z = blockIdx.z;
+    ya += (int32_t)(job.ti[z] * job.b);
+    yb += (int32_t)(job.tj[z] * job.b);
+    C += ((int64_t)job.ti[z] * job.T + job.tj[z]) * job.b * job.b;
+  }
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < kStages; ++s) {
@@ -119,10 +140,10 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
         if (kb >= kStages) mbar_wait(&empty[s], (uint32_t)(((kb / kStages) - 1) & 1));
         uint8_t* st = base + s * STAGE_BYTES;
         mbar_expect_tx(&full[s], STAGE_BYTES);
-        tma_load_2d(st, &tAhi, kb * BK, m_blk * BM, &full[s]);
-        tma_load_2d(st + A_BYTES, &tAlo, kb * BK, m_blk * BM, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES, &tBhi, kb * BK, n_blk * BN, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kb * BK, n_blk * BN, &full[s]);
+        tma_load_2d(st, &tAhi, kb * BK, ya, &full[s]);
+        tma_load_2d(st + A_BYTES, &tAlo, kb * BK, ya, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES, &tBhi, kb * BK, yb, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kb * BK, yb, &full[s]);
       }
     }
     __syncwarp();
@@ -156,7 +177,7 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     const int g = warp & 3;
     const int64_t r = (int64_t)m_blk * BM + g * 32 + lane;  // row within [0, mrows)
     const bool row_ok = r < mrows;
-    float* crow = C + (row0 + r) * N;
+    float* crow = job.mode == 1 ? C + r * job.b : C + (row0 + r) * N;
 #pragma unroll 1
     for (int c = 0; c < BN; c += 16) {
       uint32_t v[16];
@@ -168,7 +189,18 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
           : "r"(ta));
       asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
       const int64_t n0 = (int64_t)n_blk * BN + c;
-      if (row_ok) {
+      if (job.mode == 1) {   // C_tile -= acc (tile row r, ldc = b)
+        float4* p = reinterpret_cast<float4*>(crow + n0);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          float4 o = p[q];
+          o.x -= __uint_as_float(v[4 * q]);
+          o.y -= __uint_as_float(v[4 * q + 1]);
+          o.z -= __uint_as_float(v[4 * q + 2]);
+          o.w -= __uint_as_float(v[4 * q + 3]);
+          p[q] = o;
+        }
+      } else if (row_ok) {
         if (n0 + 16 <= N && (N & 3) == 0) {
 #pragma unroll
           for (int q = 0; q < 4; ++q)
@@ -231,7 +263,90 @@ __global__ void split_transpose(const float* __restrict__ B, float* __restrict__
   }
 }
 
+// Split panel tiles: tile (list[t].i, k) of the tile-major matrix -> slot i of
+// the hi/lo panel buffers (b x b each, row-major = K-major rows).
+__global__ void split_tiles(const float* __restrict__ A, float* __restrict__ hi, float* __restrict__ lo,
+                            int64_t T, int64_t b, const __grid_constant__ GemmJob list, int32_t k) {
+  const int t = blockIdx.y;
+  const int64_t i = list.ti[t];
+  const float* src = A + (i * T + k) * b * b;
+  float* h = hi + i * b * b;
+  float* l = lo + i * b * b;
+  const int64_t n = b * b / 4;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+    const float4 x = reinterpret_cast<const float4*>(src)[e];
+    float4 hv, lv;
+    hv.x = tf32_rn(x.x); lv.x = tf32_rn(x.x - hv.x);
+    hv.y = tf32_rn(x.y); lv.y = tf32_rn(x.y - hv.y);
+    hv.z = tf32_rn(x.z); lv.z = tf32_rn(x.z - hv.z);
+    hv.w = tf32_rn(x.w); lv.w = tf32_rn(x.w - hv.w);
+    reinterpret_cast<float4*>(h)[e] = hv;
+    reinterpret_cast<float4*>(l)[e] = lv;
+  }
+}
+
 }  // namespace
+
+size_t chol_tc_scratch(int64_t T, int64_t b) {
+  return (b % BN == 0) ? (size_t)(2 * T * b * b) * sizeof(float) : 0;
+}
+
+// Batched C(i,j) -= A(i,k) A(j,k)^T with 3xTF32 tcgen05 (b % 256 == 0).
+cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n, cudaStream_t s,
+                           Scratch* scr) {
+  if (n <= 0) return cudaSuccess;
+  if (b % BN != 0 || !scr || !scr->ptr || scr->bytes < chol_tc_scratch(T, b)) return cudaErrorNotSupported;
+  float* hi = static_cast<float*>(scr->ptr);
+  float* lo = hi + T * b * b;
+  if (scr->panel.size() != (size_t)T) scr->panel.assign(T, 0);
+  const int32_t k = ijk[2];
+  const uint64_t tag = (scr->epoch << 20) | (uint64_t)(k + 1);
+  // 1. split the panel tiles this batch needs that are not split for step k yet
+  GemmJob sl;
+  sl.mode = 1;
+  sl.n = 0;
+  sl.T = T;
+  sl.b = b;
+  auto need = [&](int32_t i) {
+    if (scr->panel[i] != tag && sl.n < kCholBatch) {
+      scr->panel[i] = tag;
+      sl.ti[sl.n++] = i;
+    }
+  };
+  for (int32_t q = 0; q < n; ++q) {
+    if (ijk[3 * q + 2] != k) return cudaErrorInvalidValue;  // one step per batch
+    need(ijk[3 * q]);
+    need(ijk[3 * q + 1]);
+  }
+  if (sl.n) split_tiles<<<dim3((unsigned)std::min<int64_t>(b * b / 4 / 256, 64), (unsigned)sl.n), 256, 0, s>>>(
+      A, hi, lo, T, b, sl, k);
+  // 2. one batched GEMM launch over all tasks
+  CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(&ta_hi, hi, b, T * b, b * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&ta_lo, lo, b, T * b, b * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_hi, hi, b, T * b, b * 4, BK, BN)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_lo, lo, b, T * b, b * 4, BK, BN)) != cudaSuccess) return e;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    attr = true;
+  }
+  for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
+    GemmJob job;
+    job.mode = 1;
+    job.n = std::min<int32_t>(kCholBatch, n - q0);
+    job.T = T;
+    job.b = b;
+    for (int32_t q = 0; q < job.n; ++q) {
+      job.ti[q] = ijk[3 * (q0 + q)];
+      job.tj[q] = ijk[3 * (q0 + q) + 1];
+    }
+    dim3 grid((unsigned)(b / BN), (unsigned)(b / BM), (unsigned)job.n);
+    gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job);
+  }
+  return cudaGetLastError();
+}
 
 size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
   const int64_t Kp = (K + BK - 1) / BK * BK;
@@ -280,8 +395,12 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
     attr = true;
   }
   dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((mrows + BM - 1) / BM));
+  GemmJob job;
+  job.mode = 0;
+  job.n = 0;
+  job.T = job.b = 0;
   gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows,
-                                                     (int)(Kp / BK));
+                                                     (int)(Kp / BK), job);
   return cudaGetLastError();
 }
 

@@ -296,6 +296,7 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
 size_t builtin_scratch_bytes(const Kernel& k, const Task& t) {
   if (k.op == MM_OP_SGEMM && (k.ip[3] == 0 || k.ip[3] == 2))
     return sgemm_tf32x3_scratch(k.ip[1], k.ip[2], t.e - t.b);
+  if (k.op == MM_OP_CHOL_SYRK || k.op == MM_OP_CHOL_GEMM) return chol_tc_scratch(k.ip[0], k.ip[1]);
   return 0;
 }
 
@@ -330,8 +331,10 @@ cudaError_t launch_builtin(const Launch& L) {
     case MM_OP_CHOL_POTRF:
     case MM_OP_CHOL_TRSM:
     case MM_OP_CHOL_SYRK:
-    case MM_OP_CHOL_GEMM:
-      return chol_task(k.op, f[0], k.ip[0], k.ip[1], t.ip[0], t.ip[1], t.ip[2], L.stream, L.sms);
+    case MM_OP_CHOL_GEMM: {
+      const int32_t ijk[3] = {(int32_t)t.ip[0], (int32_t)t.ip[1], (int32_t)t.ip[2]};
+      return chol_batch(k.op, f[0], k.ip[0], k.ip[1], ijk, 1, L.stream, L.sms, L.scr);
+    }
   }
   return cudaErrorNotSupported;
 }
@@ -381,7 +384,7 @@ mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, voi
         cudaStreamSynchronize(s);
         cudaFree(dv.scr.ptr);
       }
-      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1};
+      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1, {}};
       if (cudaMalloc(&dv.scr.ptr, need) != cudaSuccess) MM_FAIL(MM_ENOMEM, "device scratch of %zu bytes", need);
       dv.scr.bytes = need;
     }
@@ -414,7 +417,16 @@ mm_status launch_batch(mm_ctx* ctx, const Plan& plan, const PlanRt* rt, int64_t 
   for (int64_t m : rt->members[head]) add(m);
   float* A = static_cast<float*>(buffers[(size_t)t0.acc[0].buffer * ctx->G + d]);
   if (!A) MM_FAIL(MM_EINVAL, "run: buffer slot %d has no pointer on device %d", t0.acc[0].buffer, d);
-  cudaError_t e = chol_batch(k.op, A, k.ip[0], k.ip[1], ijk.data(), (int32_t)(ijk.size() / 3), s, ctx->dev[d].sms);
+  DevRt& dv = ctx->dev[d];
+  const size_t need = builtin_scratch_bytes(k, t0);
+  if (need > dv.scr.bytes) {  // reserved by ensure_rt; only profile paths get here
+    cudaStreamSynchronize(s);
+    if (dv.scr.ptr) cudaFree(dv.scr.ptr);
+    dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1, {}};
+    if (cudaMalloc(&dv.scr.ptr, need) != cudaSuccess) MM_FAIL(MM_ENOMEM, "device scratch of %zu bytes", need);
+    dv.scr.bytes = need;
+  }
+  cudaError_t e = chol_batch(k.op, A, k.ip[0], k.ip[1], ijk.data(), (int32_t)(ijk.size() / 3), s, dv.sms, &dv.scr);
   if (e != cudaSuccess) {
     ctx->poisoned = true;
     MM_FAIL(MM_ECUDA, "batched %s launch failed: %s", k.name.c_str(), cudaGetErrorString(e));
@@ -467,7 +479,7 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
       CU_OK(set_dev(ctx, op.device));
       CU_OK(cudaDeviceSynchronize());
       if (dv.scr.ptr) cudaFree(dv.scr.ptr);
-      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1};
+      dv.scr = Scratch{nullptr, 0, nullptr, 0, 0, 0, dv.scr.epoch + 1, {}};
       CU_OK(cudaMalloc(&dv.scr.ptr, need));
       dv.scr.bytes = need;
     }

@@ -222,13 +222,15 @@ def _from_tiles(t, n, b):
     return t.reshape(T, T, b, b).transpose(0, 2, 1, 3).reshape(n, n)
 
 
+@pytest.mark.parametrize("nb", [(512, 128), (1024, 256)])
 @pytest.mark.parametrize("strategy", [4, 5, 6])
 @pytest.mark.parametrize("G", [1, 2, 3])
-def test_cholesky_exact_factor(R, strategy, G):
+def test_cholesky_exact_factor(R, strategy, G, nb):
     """MK-DAG: integer L0 (diag 32..64, band +-1), A = L0 L0^T: every FP32
-    operation is exact, so the factor must be L0 bit for bit for any schedule."""
+    operation is exact, so the factor must be L0 bit for bit for any schedule.
+    b = 128 runs the FFMA updates, b = 256 the 3xTF32 tcgen05 updates."""
     mm, runner = R
-    n, b = 512, 128
+    n, b = nb
     A, L0 = synthgen.cholesky_exact_factor(n)
     with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=G) as s:
         assert s.classify() == mm.MM_MK_DAG
