@@ -208,6 +208,7 @@ def main():
     ap.add_argument("--app", default="stream", choices=sorted(APPS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
     ap.add_argument("--logical", type=int, default=0,
                     help="virtual mode: run G logical devices on this one GPU (G = --logical)")
     args = ap.parse_args()
@@ -347,6 +348,8 @@ def main():
     # --- e2e: same step through the C ABI with HOST buffers (staged mode) ----
     e2e = None
     try:
+        if args.no_e2e:
+            raise RuntimeError("skipped (--no-e2e)")
         import numpy as np
         nbuf = sess.nbuf
         host = []
