@@ -209,6 +209,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
+    ap.add_argument("--no-profile", action="store_true",
+                    help="use an equal synthetic profile instead of measuring one (ncu runs)")
     ap.add_argument("--logical", type=int, default=0,
                     help="virtual mode: run G logical devices on this one GPU (G = --logical)")
     args = ap.parse_args()
@@ -243,7 +245,7 @@ def main():
             dist.barrier()
 
     # --- setup (excluded from timing, P311): profile, then generate inputs ---
-    prof = sess.profile(reps=3)
+    prof = sess.equal_profile() if args.no_profile else sess.profile(reps=3)
     sess.fill()
     cls = mm.mm_classify(sess.app)
     ranked = mm.mm_rank(cls, mm.mm_needs_sync(sess.app))
