@@ -324,8 +324,28 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app, void* const* buffers,
 typedef struct {
   int32_t use_graph;         /* capture the op program once, replay it (CUDA graph) */
   int32_t time_kernels;      /* CUDA events around every kernel op -> kernel_ms */
+  int32_t adaptive;          /* DP-Perf plans, in-process only: decide each chunk's device
+                                at run time from estimates updated with the measured times
+                                of completed chunks (P119 "kept and updated"); the
+                                decisions are logged (mm_run_decisions) */
+  int32_t max_inflight;      /* adaptive: chunks in flight per device before the scheduler
+                                waits for completions (default 4) */
   void* const* host;         /* staged / flush: host (pinned) pointer per slot, or NULL */
 } mm_run_opts;
+
+/* One adaptive DP-Perf decision: the snapshot it was taken on.  All times in
+ * ns since the start of the run; eft_d = max(busy_d, ready_d) + cost_d and
+ * chosen = argmin eft (ties -> lowest id).  Unused devices hold 0. */
+typedef struct {
+  int64_t task;
+  int32_t chosen;
+  int32_t kernel;
+  uint64_t now_ns;
+  uint64_t busy_ns[MM_MAX_DEV];
+  uint64_t ready_ns[MM_MAX_DEV];
+  uint64_t cost_ns[MM_MAX_DEV];
+  uint64_t eft_ns[MM_MAX_DEV];
+} mm_decision;
 
 typedef struct {
   double wall_ms;                        /* host-observed, start -> all streams done */
@@ -342,6 +362,9 @@ typedef struct {
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan, void* const* buffers, const mm_run_opts* opts,
                  mm_run_stats* stats);
 
+/* Decisions of the last adaptive run of this plan (creation order). */
+mm_status mm_run_decisions(const mm_plan* plan, mm_decision* out, int64_t cap, int64_t* count);
+
 /* Assemble buffer `slot` after a run: every element range is copied from the
  * device that holds its final value into `dst` (device memory of logical
  * device `dst_device`, or host memory if dst_device < 0).  In-process only. */
@@ -355,7 +378,8 @@ int64_t mm_kernel_launch_count(void);
 /* sizeof of every ABI struct, in this order: mm_range, mm_access,
  * mm_kernel_desc, mm_task_access, mm_task_desc, mm_app_params, mm_profile,
  * mm_plan_opts, mm_chunk, mm_op_rec, mm_plan_info_t, mm_device_spec,
- * mm_profile_opts, mm_run_opts, mm_run_stats (bindings check their mirrors). */
+ * mm_profile_opts, mm_run_opts, mm_run_stats, mm_decision (bindings check
+ * their mirrors). */
 mm_status mm_abi_sizes(int64_t* out, int32_t cap, int32_t* count);
 
 /* Thread-local message describing the last error on this thread. */

@@ -69,6 +69,8 @@ struct Wait { int32_t dev; int64_t op; };
 
 struct Plan {
   App app;                  // copy of the app (plans outlive apps)
+  mm_profile prof{};        // the profile the plan was built from
+  int32_t chunks_per_dev = 8;
   int32_t cls = 0, strategy = 0, G = 1, devices_used = 0;
   int32_t staged = 0;
   std::vector<mm_range> ranges;       // SP: [K*G]
@@ -99,6 +101,16 @@ mm_status split_items(int64_t n, int64_t granule, const std::vector<uint64_t>& c
 mm_status sp_split(const App& app, const mm_profile& prof, int32_t strategy,
                    std::vector<mm_range>& out);
 mm_status build_plan(const App& app, const mm_profile& prof, const mm_plan_opts& opts, Plan& plan);
+
+// Incremental op-program builder (adaptive DP-Perf): the caller sets
+// plan.task_dev[t] and appends task t's ops with inc_planner_step; the
+// ownership directory persists across begin/end cycles (runs).
+struct IncPlanner;
+IncPlanner* inc_planner_create(const App& app, Plan& plan);
+void inc_planner_begin(IncPlanner* ip);
+mm_status inc_planner_step(IncPlanner* ip, int64_t t);
+mm_status inc_planner_end(IncPlanner* ip);
+void inc_planner_destroy(IncPlanner* ip);
 
 // runtime.cu
 void plan_runtime_free(Plan* plan);

@@ -11,12 +11,14 @@
 #include <atomic>
 #include <chrono>
 #include <cstring>
+#include <deque>
 #include <memory>
 #include <new>
 #include <vector>
 
 #include "kernels.h"
 #include "mm_internal.h"
+#include "segmap.h"
 
 using namespace mm;
 
@@ -172,8 +174,30 @@ namespace {
     }                                                                            \
   } while (0)
 
+// Adaptive DP-Perf state of a plan: the op program built incrementally at run
+// time (its ownership directory persists across runs), one end event per op,
+// a begin event per kernel op, and the decision log of the last run.
+struct AdaptiveState {
+  Plan ap;
+  IncPlanner* inc = nullptr;
+  std::vector<mm_decision> decisions;
+  std::vector<cudaEvent_t> ev_end, ev_beg;
+  std::vector<int32_t> ev_dev;
+  cudaEvent_t t0 = nullptr;
+  ~AdaptiveState() {
+    for (auto e : ev_end)
+      if (e) cudaEventDestroy(e);
+    for (auto e : ev_beg)
+      if (e) cudaEventDestroy(e);
+    if (t0) cudaEventDestroy(t0);
+    if (inc) inc_planner_destroy(inc);
+  }
+};
+
 struct PlanRt {
   mm_ctx* ctx = nullptr;
+  AdaptiveState* ad = nullptr;
+  bool last_adaptive = false;
   std::vector<cudaEvent_t> ev;           // per op that another stream waits on
   std::vector<cudaEvent_t> bar_ev;       // per device
   std::vector<cudaEvent_t> join_ev;      // per device
@@ -265,6 +289,7 @@ void destroy_rt(PlanRt* rt) {
   if (rt->t_stop) cudaEventDestroy(rt->t_stop);
   if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
   if (rt->graph) cudaGraphDestroy(rt->graph);
+  delete rt->ad;
   delete rt;
 }
 
@@ -400,21 +425,17 @@ mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, voi
   return MM_OK;
 }
 
-// Launch a batch head together with its members (one batched kernel).
-mm_status launch_batch(mm_ctx* ctx, const Plan& plan, const PlanRt* rt, int64_t head, int32_t d,
-                       void* const* buffers, cudaStream_t s) {
-  const App& app = plan.app;
-  const Task& t0 = plan.tasks[plan.ops[head].task];
+// Launch independent DAG tasks of one kernel as one batched kernel.
+mm_status launch_task_batch(mm_ctx* ctx, const App& app, const std::vector<const Task*>& ts, int32_t d,
+                            void* const* buffers, cudaStream_t s) {
+  const Task& t0 = *ts[0];
   const Kernel& k = app.kernels[t0.kernel];
   std::vector<int32_t> ijk;
-  auto add = [&](int64_t o) {
-    const Task& t = plan.tasks[plan.ops[o].task];
-    ijk.push_back((int32_t)t.ip[0]);
-    ijk.push_back((int32_t)t.ip[1]);
-    ijk.push_back((int32_t)t.ip[2]);
-  };
-  add(head);
-  for (int64_t m : rt->members[head]) add(m);
+  for (const Task* t : ts) {
+    ijk.push_back((int32_t)t->ip[0]);
+    ijk.push_back((int32_t)t->ip[1]);
+    ijk.push_back((int32_t)t->ip[2]);
+  }
   float* A = static_cast<float*>(buffers[(size_t)t0.acc[0].buffer * ctx->G + d]);
   if (!A) MM_FAIL(MM_EINVAL, "run: buffer slot %d has no pointer on device %d", t0.acc[0].buffer, d);
   DevRt& dv = ctx->dev[d];
@@ -433,6 +454,14 @@ mm_status launch_batch(mm_ctx* ctx, const Plan& plan, const PlanRt* rt, int64_t 
   }
   g_kernel_launches.fetch_add(1, std::memory_order_relaxed);
   return MM_OK;
+}
+
+// Launch a batch head together with its members (one batched kernel).
+mm_status launch_batch(mm_ctx* ctx, const Plan& plan, const PlanRt* rt, int64_t head, int32_t d,
+                       void* const* buffers, cudaStream_t s) {
+  std::vector<const Task*> ts{&plan.tasks[plan.ops[head].task]};
+  for (int64_t m : rt->members[head]) ts.push_back(&plan.tasks[plan.ops[m].task]);
+  return launch_task_batch(ctx, plan.app, ts, d, buffers, s);
 }
 
 mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
@@ -688,6 +717,279 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
   return MM_OK;
 }
 
+// ------------------------------------------------------------------------
+// Adaptive DP-Perf (P119: "the runtime profiles how fast each device
+// processes a partition, and estimates the device busy time ... The
+// information is kept and updated to determine which device will be the
+// earliest executor for the next coming partition").  Tasks are decided in
+// creation order with the frozen rule (R21) on live state: estimates are
+// running means seeded by the warm-up profile (counted as its 3 chunks,
+// P311) and updated with every completed chunk's event-timed duration;
+// busy/ready times come from the device clock (events) and predictions.
+// ------------------------------------------------------------------------
+mm_status adaptive_event(mm_ctx* ctx, AdaptiveState* ad, size_t i, int32_t d) {
+  if (ad->ev_end.size() <= i) {
+    ad->ev_end.resize(i + 1, nullptr);
+    ad->ev_beg.resize(i + 1, nullptr);
+    ad->ev_dev.resize(i + 1, -1);
+  }
+  if (ad->ev_end[i] && ad->ev_dev[i] != ctx->dev[d].phys) {
+    cudaEventDestroy(ad->ev_end[i]);
+    cudaEventDestroy(ad->ev_beg[i]);
+    ad->ev_end[i] = ad->ev_beg[i] = nullptr;
+  }
+  if (!ad->ev_end[i]) {
+    CU_OK(cudaEventCreate(&ad->ev_end[i]));
+    CU_OK(cudaEventCreate(&ad->ev_beg[i]));
+    ad->ev_dev[i] = ctx->dev[d].phys;
+  }
+  return MM_OK;
+}
+
+mm_status adaptive_issue_op(mm_ctx* ctx, AdaptiveState* ad, size_t i, void* const* buffers,
+                            const mm_run_opts* o, mm_run_stats* st) {
+  Plan& ap = ad->ap;
+  const App& app = ap.app;
+  const int32_t G = ctx->G;
+  const mm_op_rec& op = ap.ops[i];
+  if (op.kind == MM_OPK_BARRIER) {
+    // every stream waits for every other stream's last op
+    std::vector<cudaEvent_t> evs(G, nullptr);
+    for (int32_t d = 0; d < G; ++d) {
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaEventCreateWithFlags(&evs[d], cudaEventDisableTiming));
+      CU_OK(cudaEventRecord(evs[d], ctx->dev[d].stream));
+    }
+    for (int32_t d = 0; d < G; ++d) {
+      CU_OK(set_dev(ctx, d));
+      for (int32_t q = 0; q < G; ++q)
+        if (q != d) CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, evs[q], 0));
+    }
+    for (auto e : evs) cudaEventDestroy(e);
+    return MM_OK;
+  }
+  const int32_t d = ap.op_stream[i];
+  cudaStream_t s = ctx->dev[d].stream;
+  CU_OK(set_dev(ctx, d));
+  mm_status r = adaptive_event(ctx, ad, i, d);
+  if (r) return r;
+  for (auto& w : ap.waits[i]) CU_OK(cudaStreamWaitEvent(s, ad->ev_end[w.op], 0));
+  if (op.kind == MM_OPK_KERNEL) {
+    CU_OK(cudaEventRecord(ad->ev_beg[i], s));
+    r = launch_task(ctx, app, ap.tasks[op.task], d, buffers, s);
+    if (r) return r;
+    st->n_launches++;
+  } else if (op.kind == MM_OPK_XFER) {
+    const int64_t eb = app.buffers[op.buffer].first;
+    const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+    char* dst = static_cast<char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+    const char* src = static_cast<const char*>(buffers[(size_t)op.buffer * G + op.src]) + op.r.begin * eb;
+    if (ctx->dev[op.src].phys == ctx->dev[d].phys)
+      CU_OK(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToDevice, s));
+    else
+      CU_OK(cudaMemcpyPeerAsync(dst, ctx->dev[d].phys, src, ctx->dev[op.src].phys, bytes, s));
+    st->xfer_bytes += (int64_t)bytes;
+  } else if (op.kind == MM_OPK_FLUSH) {
+    const int64_t eb = app.buffers[op.buffer].first;
+    const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+    mm_status fs;
+    char* host = static_cast<char*>(flush_target(ctx, ap, o, op.buffer,
+                                                 (size_t)(app.buffers[op.buffer].second * eb), &fs));
+    if (fs) return fs;
+    const char* src = static_cast<const char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+    CU_OK(cudaMemcpyAsync(host + op.r.begin * eb, src, bytes, cudaMemcpyDeviceToHost, s));
+    st->d2h_bytes += (int64_t)bytes;
+  }
+  CU_OK(cudaEventRecord(ad->ev_end[i], s));
+  return MM_OK;
+}
+
+mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers, const mm_run_opts* o,
+                       mm_run_stats* st) {
+  const int32_t G = ctx->G;
+  if (!rt->ad) {
+    rt->ad = new AdaptiveState();
+    Plan& ap = rt->ad->ap;
+    ap.app = plan.app;
+    ap.prof = plan.prof;
+    ap.chunks_per_dev = plan.chunks_per_dev;
+    ap.G = G;
+    ap.cls = plan.cls;
+    ap.strategy = MM_DP_PERF;
+    ap.staged = 0;
+    ap.tasks = plan.tasks;
+    ap.task_dev.assign(plan.tasks.size(), 0);
+    ap.task_fin.assign(plan.tasks.size(), 0);
+    rt->ad->inc = inc_planner_create(ap.app, ap);
+  }
+  AdaptiveState* ad = rt->ad;
+  Plan& ap = ad->ap;
+  const App& app = ap.app;
+  const int32_t maxq = o && o->max_inflight > 0 ? o->max_inflight : 4;
+  const int32_t root = first_owned(ctx);
+  inc_planner_begin(ad->inc);
+  ad->decisions.clear();
+  // fork + device time base
+  CU_OK(set_dev(ctx, root));
+  if (!ad->t0) CU_OK(cudaEventCreate(&ad->t0));
+  CU_OK(cudaEventRecord(ad->t0, ctx->dev[root].stream));
+  CU_OK(cudaEventRecord(rt->fork, ctx->dev[root].stream));
+  for (int32_t d = 0; d < G; ++d)
+    if (d != root) {
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->fork, 0));
+    }
+  const auto h0 = std::chrono::steady_clock::now();
+  auto now_ns = [&]() -> uint64_t {
+    return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - h0)
+        .count();
+  };
+  const int64_t C = (int64_t)ap.chunks_per_dev * G;
+  std::vector<int64_t> nominal(app.kernels.size());
+  for (size_t k = 0; k < app.kernels.size(); ++k)
+    nominal[k] = app.is_dag ? 1 : chunk_size(app.kernels[k].n, app.kernels[k].granule, C);
+  std::vector<std::vector<double>> est(G, std::vector<double>(app.kernels.size(), 1.0));
+  std::vector<std::vector<double>> cnt(G, std::vector<double>(app.kernels.size(), 3.0));  // warm-up = 3 chunks
+  for (int32_t d = 0; d < G; ++d)
+    for (size_t k = 0; k < app.kernels.size(); ++k) est[d][k] = (double)std::max<uint64_t>(1, ap.prof.chunk_est_ns[d][k]);
+  std::vector<SegMap<int64_t>> lw(app.buffers.size());
+  for (size_t b = 0; b < app.buffers.size(); ++b) lw[b].reset(app.buffers[b].second, -1);
+  std::vector<uint64_t> fin(ap.tasks.size(), 0);  // predicted, then measured finish (ns, device time)
+  std::vector<uint64_t> pred_fin(G, 0);
+  std::vector<int64_t> last_task(G, -1);
+  struct Out { int64_t t; int32_t d; size_t op; };
+  std::deque<Out> outq;
+  auto complete = [&](const Out& x) -> mm_status {
+    float ms = 0.f, endms = 0.f;
+    CU_OK(cudaEventElapsedTime(&ms, ad->ev_beg[x.op], ad->ev_end[x.op]));
+    CU_OK(cudaEventElapsedTime(&endms, ad->t0, ad->ev_end[x.op]));
+    const Task& t = ap.tasks[x.t];
+    const int64_t items = app.is_dag ? 1 : std::max<int64_t>(1, t.e - t.b);
+    const double meas = (double)ms * 1e6 * (double)nominal[t.kernel] / (double)items;
+    double& e = est[x.d][t.kernel];
+    double& c = cnt[x.d][t.kernel];
+    e = (e * c + meas) / (c + 1.0);
+    c += 1.0;
+    fin[x.t] = (uint64_t)((double)endms * 1e6);
+    if (last_task[x.d] == x.t) pred_fin[x.d] = fin[x.t];
+    return MM_OK;
+  };
+  auto poll = [&](bool block_oldest) -> mm_status {
+    if (block_oldest && !outq.empty()) CU_OK(cudaEventSynchronize(ad->ev_end[outq.front().op]));
+    while (!outq.empty()) {
+      cudaError_t q = cudaEventQuery(ad->ev_end[outq.front().op]);
+      if (q == cudaErrorNotReady) break;
+      CU_OK(q);
+      mm_status r = complete(outq.front());
+      if (r) return r;
+      outq.pop_front();
+    }
+    return MM_OK;
+  };
+  int32_t last_inv = -1;
+  for (size_t t = 0; t < ap.tasks.size(); ++t) {
+    const Task& task = ap.tasks[t];
+    if (!app.is_dag && task.inv != last_inv) {
+      if (last_inv >= 0) {  // R11: a sync point after the previous invocation aligns the devices
+        const int32_t kprev = ap.tasks[t - 1].kernel;
+        auto it = app.sync.find(kprev);
+        if (it != app.sync.end() && it->second != MM_SYNC_NONE) {
+          const uint64_t m = *std::max_element(pred_fin.begin(), pred_fin.end());
+          std::fill(pred_fin.begin(), pred_fin.end(), m);
+        }
+      }
+      last_inv = task.inv;
+    }
+    mm_status r = poll(false);
+    if (r) return r;
+    while ((int64_t)outq.size() >= (int64_t)maxq * G) {
+      r = poll(true);
+      if (r) return r;
+    }
+    // producers of what the task reads (RAW), with bytes
+    std::map<int64_t, int64_t> preds;
+    for (auto& a : task.acc) {
+      if (!(a.mode & MM_READ)) continue;
+      const int64_t eb = app.buffers[a.buffer].first;
+      lw[a.buffer].visit(a.lo, a.hi, [&](int64_t lo, int64_t hi, const int64_t& w) {
+        if (w >= 0) preds[w] += (hi - lo) * eb;
+      });
+    }
+    mm_decision dec;
+    std::memset(&dec, 0, sizeof(dec));
+    dec.task = (int64_t)t;
+    dec.kernel = task.kernel;
+    dec.now_ns = now_ns();
+    const int64_t items = app.is_dag ? 1 : std::max<int64_t>(1, task.e - task.b);
+    int32_t best = -1;
+    for (int32_t d = 0; d < G; ++d) {
+      uint64_t ready = 0;
+      for (auto& p : preds) {
+        uint64_t rr = fin[p.first];
+        if (ap.task_dev[p.first] != d) {
+          const uint64_t link = std::max<uint64_t>(1, ap.prof.link_Bps[d]);
+          rr += (uint64_t)(((unsigned __int128)p.second * 1000000000ull + link - 1) / link);
+        }
+        ready = std::max(ready, rr);
+      }
+      const uint64_t busy = std::max(dec.now_ns, pred_fin[d]);
+      const uint64_t cost = (uint64_t)(est[d][task.kernel] * (double)items / (double)nominal[task.kernel]);
+      dec.busy_ns[d] = busy;
+      dec.ready_ns[d] = ready;
+      dec.cost_ns[d] = cost;
+      dec.eft_ns[d] = std::max(busy, ready) + cost;
+      if (best < 0 || dec.eft_ns[d] < dec.eft_ns[best]) best = d;
+    }
+    dec.chosen = best;
+    ad->decisions.push_back(dec);
+    ap.task_dev[t] = best;
+    fin[t] = dec.eft_ns[best];
+    pred_fin[best] = fin[t];
+    last_task[best] = (int64_t)t;
+    for (auto& a : task.acc)
+      if (a.mode & MM_WRITE) lw[a.buffer].assign(a.core_lo, a.core_hi, (int64_t)t);
+    const size_t n0 = ap.ops.size();
+    r = inc_planner_step(ad->inc, (int64_t)t);
+    if (r) return r;
+    for (size_t i = n0; i < ap.ops.size(); ++i) {
+      r = adaptive_issue_op(ctx, ad, i, buffers, o, st);
+      if (r) return r;
+      if (ap.ops[i].kind == MM_OPK_KERNEL) outq.push_back(Out{(int64_t)t, best, i});
+    }
+  }
+  const size_t n0 = ap.ops.size();
+  mm_status r = inc_planner_end(ad->inc);
+  if (r) return r;
+  for (size_t i = n0; i < ap.ops.size(); ++i) {
+    r = adaptive_issue_op(ctx, ad, i, buffers, o, st);
+    if (r) return r;
+  }
+  // join
+  for (int32_t d = 0; d < G; ++d)
+    if (d != root) {
+      CU_OK(set_dev(ctx, d));
+      CU_OK(cudaEventRecord(rt->join_ev[d], ctx->dev[d].stream));
+      CU_OK(set_dev(ctx, root));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[d], 0));
+    }
+  CU_OK(set_dev(ctx, root));
+  CU_OK(cudaStreamSynchronize(ctx->dev[root].stream));
+  while (!outq.empty()) {
+    r = complete(outq.front());
+    if (r) return r;
+    outq.pop_front();
+  }
+  for (size_t i = 0; i < ap.ops.size(); ++i) {
+    const mm_op_rec& op = ap.ops[i];
+    if (op.kind != MM_OPK_KERNEL) continue;
+    float ms = 0.f;
+    CU_OK(cudaEventElapsedTime(&ms, ad->ev_beg[i], ad->ev_end[i]));
+    st->kernel_ms[op.device][op.kernel] += ms;
+    st->kernel_launches[op.device][op.kernel]++;
+  }
+  return MM_OK;
+}
+
 }  // namespace
 
 // ===========================================================================
@@ -909,6 +1211,25 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   cudaStream_t rs = ctx->dev[root].stream;
   const size_t nbuf = plan.app.buffers.size() * (size_t)ctx->G;
   auto t0 = std::chrono::steady_clock::now();
+  if (o && o->adaptive) {
+    if (plan.strategy != MM_DP_PERF) MM_FAIL(MM_EINVAL, "run: adaptive needs a DP-Perf plan");
+    if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "run: adaptive DP-Perf is in-process only");
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventRecord(rt->t_start, rs));
+    r = run_adaptive(ctx, plan, rt, buffers, o, S);
+    if (r) return r;
+    CU_OK(set_dev(ctx, root));
+    CU_OK(cudaEventRecord(rt->t_stop, rs));
+    CU_OK(cudaEventSynchronize(rt->t_stop));
+    auto t1a = std::chrono::steady_clock::now();
+    S->wall_ms = std::chrono::duration<double, std::milli>(t1a - t0).count();
+    float msa = 0.f;
+    CU_OK(cudaEventElapsedTime(&msa, rt->t_start, rt->t_stop));
+    S->device_ms = msa;
+    rt->last_adaptive = true;
+    return MM_OK;
+  }
+  rt->last_adaptive = false;
   if (graph) {
     std::vector<void*> bufs(buffers, buffers + nbuf);
     if (!rt->gexec || bufs != rt->graph_bufs) {
@@ -976,7 +1297,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
 mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan_h, void* const* buffers, int32_t slot, void* dst,
                      int32_t dst_device) {
   if (!ctx || !plan_h || !buffers || !dst) MM_FAIL(MM_EINVAL, "collect: null argument");
-  const Plan& plan = plan_h->p;
+  const PlanRt* prt = static_cast<const PlanRt*>(plan_h->p.rt);
+  const Plan& plan = (prt && prt->last_adaptive && prt->ad) ? prt->ad->ap : plan_h->p;
   if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "collect: in-process contexts only");
   if (slot < 0 || slot >= (int32_t)plan.app.buffers.size()) MM_FAIL(MM_EINVAL, "collect: slot");
   const int64_t eb = plan.app.buffers[slot].first;
@@ -1034,20 +1356,30 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
       for (int32_t k = 0; k < K; ++k) {
         const Kernel& kern = app.kernels[k];
         if (app.is_dag) {
-          const Task* t = nullptr;
+          // per-task cost at the device's batch capacity: up to 16 independent
+          // tasks of this kernel from its first step, launched as one batch
+          // (how the executor runs them); non-batchable kernels: one task.
+          std::vector<const Task*> ts;
           for (auto& x : app.dag)
-            if (x.kernel == k) {
-              t = &x;
-              break;
+            if (x.kernel == k && (ts.empty() || x.ip[2] == ts[0]->ip[2])) {
+              if (!ts.empty() && !is_batchable_op(kern.op)) break;
+              ts.push_back(&x);
+              if (ts.size() >= 16) break;
             }
-          if (!t) continue;
+          if (ts.empty()) continue;
           std::vector<float> v(reps);
           for (int32_t i = 0; i < reps; ++i) {
-            mm_status r = time_task(*t, &v[i]);
+            mm_status r = launch_task_batch(ctx, app, ts, d, buffers, s);  // warm-up
             if (r) return r;
+            CU_OK(cudaEventRecord(a, s));
+            r = launch_task_batch(ctx, app, ts, d, buffers, s);
+            if (r) return r;
+            CU_OK(cudaEventRecord(b, s));
+            CU_OK(cudaEventSynchronize(b));
+            CU_OK(cudaEventElapsedTime(&v[i], a, b));
           }
           std::sort(v.begin(), v.end());
-          const uint64_t ns = std::max<uint64_t>(1, (uint64_t)(v[reps / 2] * 1e6));
+          const uint64_t ns = std::max<uint64_t>(1, (uint64_t)(v[reps / 2] * 1e6 / (double)ts.size()));
           out->chunk_est_ns[d][k] = ns;
           out->fs_item[d][k] = ns * 1000000;
           continue;
@@ -1149,5 +1481,18 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
 }
 
 int64_t mm_kernel_launch_count(void) { return g_kernel_launches.load(); }
+
+mm_status mm_run_decisions(const mm_plan* plan_h, mm_decision* out, int64_t cap, int64_t* count) {
+  if (!plan_h || !count) MM_FAIL(MM_EINVAL, "decisions: null argument");
+  const PlanRt* rt = static_cast<const PlanRt*>(plan_h->p.rt);
+  if (!rt || !rt->ad) {
+    *count = 0;
+    return MM_OK;
+  }
+  *count = (int64_t)rt->ad->decisions.size();
+  if (cap < *count || (!out && *count)) MM_FAIL(MM_ERANGE, "decisions: cap");
+  std::copy(rt->ad->decisions.begin(), rt->ad->decisions.end(), out);
+  return MM_OK;
+}
 
 }  // extern "C"

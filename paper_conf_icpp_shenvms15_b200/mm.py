@@ -118,7 +118,14 @@ class mm_profile_opts(C.Structure):
 
 
 class mm_run_opts(C.Structure):
-    _fields_ = [("use_graph", C.c_int32), ("time_kernels", C.c_int32), ("host", C.POINTER(C.c_void_p))]
+    _fields_ = [("use_graph", C.c_int32), ("time_kernels", C.c_int32), ("adaptive", C.c_int32),
+                ("max_inflight", C.c_int32), ("host", C.POINTER(C.c_void_p))]
+
+
+class mm_decision(C.Structure):
+    _fields_ = [("task", C.c_int64), ("chosen", C.c_int32), ("kernel", C.c_int32), ("now_ns", C.c_uint64),
+                ("busy_ns", C.c_uint64 * MM_MAX_DEV), ("ready_ns", C.c_uint64 * MM_MAX_DEV),
+                ("cost_ns", C.c_uint64 * MM_MAX_DEV), ("eft_ns", C.c_uint64 * MM_MAX_DEV)]
 
 
 class mm_run_stats(C.Structure):
@@ -131,7 +138,7 @@ class mm_run_stats(C.Structure):
 
 ABI_STRUCTS = [mm_range, mm_access, mm_kernel_desc, mm_task_access, mm_task_desc, mm_app_params,
                mm_profile, mm_plan_opts, mm_chunk, mm_op_rec, mm_plan_info_t, mm_device_spec,
-               mm_profile_opts, mm_run_opts, mm_run_stats]
+               mm_profile_opts, mm_run_opts, mm_run_stats, mm_decision]
 
 # ---------------------------------------------------------------- loading --
 if not os.path.exists(LIB_PATH):
@@ -178,6 +185,7 @@ _SIGS = {
     "mm_profile_run": [_P, _P, C.POINTER(_P), C.POINTER(mm_profile_opts), C.POINTER(mm_profile)],
     "mm_run": [_P, _P, C.POINTER(_P), C.POINTER(mm_run_opts), C.POINTER(mm_run_stats)],
     "mm_collect": [_P, _P, C.POINTER(_P), C.c_int32, C.c_void_p, C.c_int32],
+    "mm_run_decisions": [_P, C.POINTER(mm_decision), C.c_int64, C.POINTER(C.c_int64)],
     "mm_abi_sizes": [C.POINTER(C.c_int64), C.c_int32, C.POINTER(C.c_int32)],
 }
 for _name, _args in _SIGS.items():
@@ -497,16 +505,26 @@ def mm_profile_run(ctx: int, app: int, buffers: Sequence[int], reps: int = 5, dp
 
 
 def mm_run(ctx: int, plan: int, buffers: Sequence[int], use_graph: bool = False, time_kernels: bool = False,
-           host: Optional[Sequence[int]] = None) -> mm_run_stats:
+           host: Optional[Sequence[int]] = None, adaptive: bool = False, max_inflight: int = 0) -> mm_run_stats:
     o = mm_run_opts()
     o.use_graph = int(use_graph)
     o.time_kernels = int(time_kernels)
+    o.adaptive = int(adaptive)
+    o.max_inflight = int(max_inflight)
     if host is not None:
         harr = _ptr_array(host)
         o.host = C.cast(harr, C.POINTER(C.c_void_p))
     st = mm_run_stats()
     _call("mm_run", ctx, plan, _ptr_array(buffers), C.byref(o), C.byref(st))
     return st
+
+
+def mm_run_decisions(plan: int) -> List[mm_decision]:
+    n = C.c_int64()
+    lib.mm_run_decisions(plan, None, 0, C.byref(n))
+    out = (mm_decision * max(1, n.value))()
+    _call("mm_run_decisions", plan, out, n.value, C.byref(n))
+    return list(out[:n.value])
 
 
 def mm_collect(ctx: int, plan: int, buffers: Sequence[int], slot: int, dst: int, dst_device: int = -1):

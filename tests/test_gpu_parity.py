@@ -266,3 +266,42 @@ def test_cholesky_device_spd_generator(R):
         s.fill()
         got = s.bufs[(0, 0)].cpu().numpy()
     assert np.array_equal(got, _to_tiles(synthgen.spd_random(n), b).reshape(-1))
+
+
+@pytest.mark.parametrize("app", ["stream", "hotspot"])
+def test_adaptive_dp_perf(R, app):
+    """Adaptive DP-Perf (P119: estimates kept and updated at run time): results
+    stay bit-exact, and every logged decision is the earliest-finish choice on
+    its own snapshot (replayed by the oracle's rule)."""
+    mm, runner = R
+    from oracle import control as oc
+    if app == "stream":
+        n, passes = 1 << 20, 2
+        ip, G = [n, passes, 1, 32, 1], 3
+        a0, b0, c0 = synthgen.stream_random(n)
+        ref = on.stream_run(a0, b0, c0, 2 * passes)
+        sess = runner.session(mm.MM_APP_STREAM, ip, G=G)
+    else:
+        rows, cols, iters = 512, 256, 6
+        ip, G = [rows, cols, iters, 1, 1], 2
+        t0, p = synthgen.hotspot(rows, cols)
+        ref = on.hotspot_run(t0, p, 2 * iters)
+        sess = runner.session(mm.MM_APP_HOTSPOT, ip, G=G)
+    with sess as s:
+        prof = s.profile(reps=3)
+        s.fill()
+        plan = s.plan(4, prof, chunks_per_dev=4)
+        s.run(plan, adaptive=True, max_inflight=3)
+        s.run(plan, adaptive=True, max_inflight=3)   # continues from the first run's placement
+        if app == "stream":
+            for k in range(3):
+                assert np.array_equal(s.collect(plan, k), ref[k])
+        else:
+            assert np.array_equal(s.collect(plan, 0).reshape(rows, cols), ref)
+        decs = mm.mm_run_decisions(plan)
+        info = mm.mm_plan_info(plan)
+        assert len(decs) == info.n_tasks
+        for dc in decs:
+            busy, ready, cost = list(dc.busy_ns[:G]), list(dc.ready_ns[:G]), list(dc.cost_ns[:G])
+            chosen, eft = oc.replay_decision(busy, ready, cost)
+            assert chosen == dc.chosen and eft == list(dc.eft_ns[:G])

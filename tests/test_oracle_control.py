@@ -342,3 +342,11 @@ def test_hotspot_halo_rows():
     # iterations 1..4 each move one ghost row per internal boundary per direction
     assert len(xs) == (iters - 1) * 2 * (G - 1)
     assert all(o[5] - o[4] == cols for o in xs)
+
+
+def test_replay_decision_rule():
+    # earliest finish wins; a busier device loses; ties go to the lowest id
+    assert oc.replay_decision([0, 0], [0, 0], [10, 5])[0] == 1
+    assert oc.replay_decision([100, 0], [0, 0], [10, 50])[0] == 1
+    assert oc.replay_decision([0, 0], [0, 0], [7, 7])[0] == 0
+    assert oc.replay_decision([0, 0], [30, 0], [10, 25]) == (1, [40, 25])
