@@ -82,6 +82,7 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 h.copy_(s.bufs[(slot, 0)].cpu())
                 host.append(h)
         times, shares = {}, {}
+        adaptive_ms, ad_share = None, None
         strategies = list(order) + ([mm.MM_SP_CYCLIC] if cls == mm.MM_MK_DAG else [])
         for st in strategies:
             p = s.plan(st, prof, staged=staged)
@@ -92,6 +93,13 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 r = s.run(p, **kw)
                 ts.append(r.device_ms)
             times[st] = statistics.median(ts)
+            if st == mm.MM_DP_PERF and not staged:
+                # adaptive DP-Perf (estimates updated at run time) beside the frozen schedule
+                s.run(p, adaptive=True)
+                ta = [s.run(p, adaptive=True).device_ms for _ in range(reps)]
+                adaptive_ms = statistics.median(ta)
+                decs = mm.mm_run_decisions(p)
+                ad_share = [sum(1 for dc in decs if dc.chosen == d) / max(1, len(decs)) for d in range(2)]
             info = mm.mm_plan_info(p)
             tot = [sum(info.items[d][k] for k in range(s.K)) for d in range(2)]
             shares[mm.mm_strategy_name(st)] = [round(x / max(1, sum(tot)), 4) for x in tot]
@@ -102,6 +110,8 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 "ms": {mm.mm_strategy_name(k): round(v, 4) for k, v in times.items()},
                 "measured_order": [mm.mm_strategy_name(k) for k, _ in sorted(times.items(), key=lambda kv: kv[1])],
                 "share_per_device": shares, "ranking_holds": ok, "pairs": pairs,
+                "dp_perf_adaptive_ms": None if adaptive_ms is None else round(adaptive_ms, 4),
+                "dp_perf_adaptive_task_share": ad_share,
                 "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(2)],
                 "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(2)]}
     finally:
@@ -130,7 +140,8 @@ def main():
                 r["platform"] = pname
                 res["configs"].append(r)
                 print(json.dumps({k: r.get(k) for k in ("platform", "app", "mode", "ms", "ranking_holds",
-                                                         "share_per_device", "error")}), flush=True)
+                                                         "dp_perf_adaptive_ms", "share_per_device", "error")}),
+                      flush=True)
     res["wall_s"] = round(time.time() - t0, 1)
     held = [c.get("ranking_holds") for c in res["configs"] if "ranking_holds" in c]
     res["summary"] = {"configs": len(res["configs"]), "ranking_holds": sum(bool(h) for h in held),
