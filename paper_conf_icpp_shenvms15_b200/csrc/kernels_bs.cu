@@ -29,9 +29,9 @@ __device__ __forceinline__ float cnd(float d) {
 
 __device__ __forceinline__ void option(float s, float x, float t, float R, float V, float& call,
                                        float& put) {
-  const float sqrtT = sqrtf(t);
-  const float vst = V * sqrtT;
-  const float d1 = __fdividef(logf(__fdividef(s, x)) + (R + 0.5f * V * V) * t, vst);
+  const float rsT = rsqrtf(t);                     // MUFU.RSQ: 1/sqrt(T)
+  const float vst = V * (t * rsT);                 // V sqrt(T)
+  const float d1 = (logf(__fdividef(s, x)) + (R + 0.5f * V * V) * t) * (rsT * (1.0f / V));
   const float d2 = d1 - vst;
   const float n1 = cnd(d1), n2 = cnd(d2);
   const float expRT = __expf(-R * t);
@@ -44,9 +44,18 @@ __global__ void __launch_bounds__(kThreads) bs_vec(const float4* __restrict__ S,
                                                    const float4* __restrict__ T,
                                                    float4* __restrict__ C, float4* __restrict__ P,
                                                    int64_t n4, float R, float V) {
-  for (int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x; i < n4;
-       i += (int64_t)gridDim.x * kThreads) {
+  // two float4 groups per iteration: all six loads are issued before the math
+  const int64_t stride = (int64_t)gridDim.x * kThreads;
+  for (int64_t i = (int64_t)blockIdx.x * kThreads + threadIdx.x; i < n4; i += 2 * stride) {
+    const int64_t j = i + stride;
+    const bool has_j = j < n4;
     const float4 s = __ldcs(S + i), x = __ldcs(X + i), t = __ldcs(T + i);
+    float4 s2 = s, x2 = x, t2 = t;
+    if (has_j) {
+      s2 = __ldcs(S + j);
+      x2 = __ldcs(X + j);
+      t2 = __ldcs(T + j);
+    }
     float4 c, p;
     option(s.x, x.x, t.x, R, V, c.x, p.x);
     option(s.y, x.y, t.y, R, V, c.y, p.y);
@@ -54,6 +63,14 @@ __global__ void __launch_bounds__(kThreads) bs_vec(const float4* __restrict__ S,
     option(s.w, x.w, t.w, R, V, c.w, p.w);
     __stcs(C + i, c);
     __stcs(P + i, p);
+    if (has_j) {
+      option(s2.x, x2.x, t2.x, R, V, c.x, p.x);
+      option(s2.y, x2.y, t2.y, R, V, c.y, p.y);
+      option(s2.z, x2.z, t2.z, R, V, c.z, p.z);
+      option(s2.w, x2.w, t2.w, R, V, c.w, p.w);
+      __stcs(C + j, c);
+      __stcs(P + j, p);
+    }
   }
 }
 
