@@ -49,12 +49,14 @@ APPS = {
                  "SK-One MatrixMul 1024^2 FP32 (BASELINE configs[0])"),
     "cholesky": ("MM_APP_CHOLESKY", [32768, 1024], lambda p: p[0] ** 3 / 3,
                  "MK-DAG tiled Cholesky 32768^2 FP32, tile 1024 (BASELINE configs[4])"),
+    "nbody": ("MM_APP_NBODY", [1048576, 1], lambda p: 20 * p[0] * p[0] * p[1],
+              "SK-Loop Nbody 1,048,576 bodies, 1 step (P319; 20 flop/interaction)"),
 }
-FLOP_APPS = ("sgemm", "matmul1k", "cholesky")
+FLOP_APPS = ("sgemm", "matmul1k", "cholesky", "nbody")
 # kernel whose roofline is reported, and its algorithmic bytes per item
 DOMINANT = {"stream": ("triad", 12), "stream-loop": ("triad", 12), "hotspot": ("hotspot", None),
             "stencil": ("stencil", None), "blackscholes": ("blackscholes", 20), "sgemm": ("sgemm", None),
-            "matmul1k": ("sgemm", None), "cholesky": ("gemm", None)}
+            "matmul1k": ("sgemm", None), "cholesky": ("gemm", None), "nbody": ("nbody", None)}
 
 
 def load_peaks():
@@ -303,7 +305,7 @@ def main():
     kname_map = {"stream": ["copy", "scale", "add", "triad"], "stream-loop": ["copy", "scale", "add", "triad"],
                  "hotspot": ["hotspot"], "stencil": ["stencil", "residual"], "blackscholes": ["blackscholes"],
                  "sgemm": ["sgemm"], "matmul1k": ["sgemm"],
-                 "cholesky": ["potrf", "trsm", "syrk", "gemm"]}[args.app]
+                 "cholesky": ["potrf", "trsm", "syrk", "gemm"], "nbody": ["nbody"]}[args.app]
     kid = kname_map.index(dom)
     my = [d for d in range(G) if sess.mine[d]]
     dom_ms = sum(kms[d][kid] for d in my)
@@ -315,7 +317,15 @@ def main():
     if dom_launch and dom_ms > 0:
         per_launch_ms = dom_ms / dom_launch
         launches_per_step = dom_launch / args.steps
-        if args.app == "cholesky":
+        if args.app == "nbody":
+            # FFMA/MUFU-bound all-pairs: 20 flop per interaction vs the FP32 FMA peak
+            n_b = iparam[0]
+            ach = 20 * n_b * items * args.steps / (dom_ms * 1e-3) / 1e12
+            pk = 148 * 128 * 2 * 1.965e9 / 1e12
+            roof = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
+                    "traffic": None, "kernel": "nbody (all pairs, smem tiles)",
+                    "peak_kind": "derived: 148 SMs x 128 FP32 lanes x 2 x 1.965 GHz (B200_PROFILING clocks)"}
+        elif args.app == "cholesky":
             # trailing GEMM updates on tcgen05 (3xTF32): FP32-equivalent flops vs
             # measured bf16 x 0.5 (tf32) / 3
             b = iparam[1]

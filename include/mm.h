@@ -98,7 +98,9 @@ typedef enum {
   MM_OP_CHOL_POTRF = 9,      /* DAG task ops [A]; task iparam k; kernel iparam T, b */
   MM_OP_CHOL_TRSM = 10,      /* DAG task iparam i, k                              */
   MM_OP_CHOL_SYRK = 11,      /* DAG task iparam i, k                              */
-  MM_OP_CHOL_GEMM = 12       /* DAG task iparam i, j, k                           */
+  MM_OP_CHOL_GEMM = 12,      /* DAG task iparam i, j, k                           */
+  MM_OP_NBODY = 13           /* ops [pos R (whole), vel R, pos' W, vel' W] float4 bodies;
+                                iparam n; fparam dt, eps2                  (P319)   */
 } mm_op;
 
 /* User kernel callback (MM_OP_CUSTOM): launch the kernel for `items` on
@@ -169,7 +171,8 @@ typedef enum {
   MM_APP_STENCIL_REDUCTION = 3, /* ip0 rows, ip1 cols, ip2 steps, ip3 sync      */
   MM_APP_BLACKSCHOLES = 4,      /* ip0 n; fp0 R, fp1 V                          */
   MM_APP_SGEMM = 5,             /* ip0 M, ip1 N, ip2 K, ip3 variant             */
-  MM_APP_CHOLESKY = 6           /* ip0 n, ip1 tile b                            */
+  MM_APP_CHOLESKY = 6,          /* ip0 n, ip1 tile b                            */
+  MM_APP_NBODY = 7              /* ip0 bodies, ip1 iterations, ip2 granule, ip3 min; fp0 dt, fp1 eps2 */
 } mm_app_id;
 typedef struct { int64_t iparam[MM_MAX_PARAM]; double fparam[MM_MAX_PARAM]; } mm_app_params;
 mm_status mm_app_builtin(int32_t app_id, const mm_app_params* p, mm_app** out);

@@ -95,3 +95,15 @@ def cholesky_tasks(T: int, b: int) -> App:
     ks = [Kernel(nm, 1, 1, 1, []) for nm in ("potrf", "trsm", "syrk", "gemm")]
     edges = [(0, 1), (1, 2), (1, 3), (2, 0), (3, 1), (3, 2), (3, 3)]
     return App(buffers=[(4, T * T * bb)], kernels=ks, edges=edges, dag_tasks=tasks)
+
+
+def nbody(n: int, iters: int, granule: int = 256, min_items: int = 1) -> App:
+    """Nbody (P223-227, P319): one all-pairs kernel iterated (SK-Loop); slots
+    pos_in=0, pos_out=1, vel_in=2, vel_out=3 (float4 bodies = 4 elements per
+    item); every body reads all positions (whole-buffer access, R18)."""
+    k = Kernel("nbody", n, granule, min_items,
+               [Access(0, READ, 0), Access(2, READ, 4), Access(1, WRITE, 4), Access(3, WRITE, 4)])
+    app = App(buffers=[(4, 4 * n)] * 4, kernels=[k], swaps=[(0, 1), (2, 3)])
+    if iters > 1:
+        app.loop = (0, 0, iters)
+    return app

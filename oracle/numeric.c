@@ -180,3 +180,39 @@ int32_t or_cholesky(const double *A, double *L, int64_t n) {
     }
     return 0;
 }
+
+/* ---------------------------------------------------------------------------
+ * Nbody (P223-227 Table II "Mont-Blanc benchmark suite", P319: 1,048,576
+ * bodies, 64 MB, iterated -> SK-Loop).  All-pairs gravitational acceleration
+ * with Plummer softening and a semi-implicit Euler step (the CUDA SDK nbody
+ * integrator [ext]):
+ *   a_i = sum_j m_j (p_j - p_i) / (|p_j - p_i|^2 + eps2)^{3/2}
+ *   v_i' = v_i + a_i dt,   p_i' = p_i + v_i' dt
+ * Bodies are float4 (x, y, z, m) positions and (vx, vy, vz, 0) velocities;
+ * computed in FP64, stored in FP32 (R13).  Bodies [r0, r1) are written.
+ * ------------------------------------------------------------------------- */
+void or_nbody_step(const float *pin, const float *vin, float *pout, float *vout, int64_t n,
+                   int64_t r0, int64_t r1, double dt, double eps2) {
+    for (int64_t i = r0; i < r1; ++i) {
+        const double xi = pin[4 * i], yi = pin[4 * i + 1], zi = pin[4 * i + 2];
+        double ax = 0.0, ay = 0.0, az = 0.0;
+        for (int64_t j = 0; j < n; ++j) {
+            const double dx = (double)pin[4 * j] - xi, dy = (double)pin[4 * j + 1] - yi,
+                         dz = (double)pin[4 * j + 2] - zi;
+            const double d2 = dx * dx + dy * dy + dz * dz + eps2;
+            const double s = (double)pin[4 * j + 3] / (d2 * sqrt(d2));
+            ax += dx * s;
+            ay += dy * s;
+            az += dz * s;
+        }
+        const double vx = vin[4 * i] + ax * dt, vy = vin[4 * i + 1] + ay * dt, vz = vin[4 * i + 2] + az * dt;
+        vout[4 * i] = (float)vx;
+        vout[4 * i + 1] = (float)vy;
+        vout[4 * i + 2] = (float)vz;
+        vout[4 * i + 3] = vin[4 * i + 3];
+        pout[4 * i] = (float)(xi + vx * dt);
+        pout[4 * i + 1] = (float)(yi + vy * dt);
+        pout[4 * i + 2] = (float)(zi + vz * dt);
+        pout[4 * i + 3] = pin[4 * i + 3];
+    }
+}

@@ -173,3 +173,26 @@ def cholesky(A):
     if rc != 0:
         raise ValueError(f"not positive definite at row {-rc - 1}")
     return L
+
+
+# --- Nbody (P223-227, P319; CUDA SDK integrator) ---------------------------
+NBODY_DT, NBODY_EPS2 = 1e-3, 1e-2
+
+
+def nbody_run(pos, vel, iters, dt=NBODY_DT, eps2=NBODY_EPS2):
+    """pos, vel: (n, 4) float32.  Returns (pos, vel) after `iters` steps."""
+    L = lib()
+    if not hasattr(L, "_nbody_ready"):
+        f32p = np.ctypeslib.ndpointer(np.float32, flags="C_CONTIGUOUS")
+        L.or_nbody_step.argtypes = [f32p, f32p, f32p, f32p, C.c_int64, C.c_int64, C.c_int64,
+                                    C.c_double, C.c_double]
+        L._nbody_ready = True
+    n = pos.shape[0]
+    p = np.ascontiguousarray(pos, dtype=np.float32).copy()
+    v = np.ascontiguousarray(vel, dtype=np.float32).copy()
+    p2, v2 = np.empty_like(p), np.empty_like(v)
+    for _ in range(iters):
+        L.or_nbody_step(p.reshape(-1), v.reshape(-1), p2.reshape(-1), v2.reshape(-1), n, 0, n, dt, eps2)
+        p, p2 = p2, p
+        v, v2 = v2, v
+    return p, v

@@ -197,6 +197,32 @@ mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
   return MM_OK;
 }
 
+mm_status nbody_app(const mm_app_params& p, mm_app* app) {
+  // Nbody (P223-227, P319): one all-pairs kernel iterated (SK-Loop); bodies are
+  // float4 (4 elements per item); positions are read whole (every body needs
+  // every position), velocities and outputs per body; ping-pong buffers.
+  const int64_t n = p.iparam[0], iters = std::max<int64_t>(1, p.iparam[1]);
+  const int64_t g = p.iparam[2] > 0 ? p.iparam[2] : 256;
+  const int64_t mn = p.iparam[3] > 0 ? p.iparam[3] : kSMs * 256;
+  if (n <= 0) MM_FAIL(MM_EINVAL, "nbody: n");
+  int32_t p0, p1, v0, v1;
+  mm_app_add_buffer(app, 4, 4 * n, &p0);
+  mm_app_add_buffer(app, 4, 4 * n, &p1);
+  mm_app_add_buffer(app, 4, 4 * n, &v0);
+  mm_app_add_buffer(app, 4, 4 * n, &v1);
+  mm_kernel_desc k = kd("nbody", MM_OP_NBODY, n, g, mn);
+  acc(k, p0, MM_READ, 0); acc(k, v0, MM_READ, 4); acc(k, p1, MM_WRITE, 4); acc(k, v1, MM_WRITE, 4);
+  k.iparam[0] = n;
+  k.fparam[0] = p.fparam[0] != 0.0 ? p.fparam[0] : 1e-3;   // dt
+  k.fparam[1] = p.fparam[1] != 0.0 ? p.fparam[1] : 1e-2;   // softening eps^2
+  mm_status st = mm_app_add_kernel(app, &k, nullptr);
+  if (st) return st;
+  mm_app_set_swap(app, p0, p1);
+  mm_app_set_swap(app, v0, v1);
+  if (iters > 1) mm_app_set_loop(app, 0, 0, iters);
+  return MM_OK;
+}
+
 }  // namespace
 
 extern "C" mm_status mm_app_builtin(int32_t app_id, const mm_app_params* p, mm_app** out) {
@@ -212,6 +238,7 @@ extern "C" mm_status mm_app_builtin(int32_t app_id, const mm_app_params* p, mm_a
       case MM_APP_BLACKSCHOLES: st = bs_app(*p, app); break;
       case MM_APP_SGEMM: st = sgemm_app(*p, app); break;
       case MM_APP_CHOLESKY: st = cholesky_app(*p, app); break;
+      case MM_APP_NBODY: st = nbody_app(*p, app); break;
       default: set_error("unknown builtin app %d", app_id); st = MM_EINVAL;
     }
   } catch (const std::bad_alloc&) {

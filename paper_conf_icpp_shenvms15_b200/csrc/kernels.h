@@ -75,6 +75,10 @@ size_t chol_tc_scratch(int64_t T, int64_t b);
 cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n, cudaStream_t s,
                            Scratch* scr);
 
+// Nbody step for bodies [r0, r1) (kernels_nbody.cu); float4 bodies.
+cudaError_t nbody_rows_launch(const float* pin, const float* vin, float* pout, float* vout, int64_t n, int64_t r0,
+                              int64_t r1, float dt, float eps2, cudaStream_t s);
+
 // Counter-hash generators (kernels_fill.cu) = synthgen.uniform / integers.
 cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id, int64_t start,
                          float lo, float hi, cudaStream_t s);

@@ -353,6 +353,8 @@ cudaError_t launch_builtin(const Launch& L) {
       return sgemm_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], k.ip[2], b, e, variant, L.stream, L.sms, L.scr,
                         (L.ro_mask >> 1) & 1u);
     }
+    case MM_OP_NBODY:
+      return nbody_rows_launch(f[0], f[1], f[2], f[3], k.ip[0], b, e, (float)k.fp[0], (float)k.fp[1], L.stream);
     case MM_OP_CHOL_POTRF:
     case MM_OP_CHOL_TRSM:
     case MM_OP_CHOL_SYRK:

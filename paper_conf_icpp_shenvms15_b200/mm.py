@@ -25,10 +25,10 @@ MM_SYNC_NONE, MM_SYNC_BARRIER, MM_SYNC_FLUSH = 0, 1, 2
 MM_READ, MM_WRITE, MM_RW = 1, 2, 3
 (MM_OP_CUSTOM, MM_OP_STREAM_COPY, MM_OP_STREAM_SCALE, MM_OP_STREAM_ADD, MM_OP_STREAM_TRIAD,
  MM_OP_HOTSPOT, MM_OP_ROW_RESIDUAL, MM_OP_BLACKSCHOLES, MM_OP_SGEMM, MM_OP_CHOL_POTRF,
- MM_OP_CHOL_TRSM, MM_OP_CHOL_SYRK, MM_OP_CHOL_GEMM) = range(13)
+ MM_OP_CHOL_TRSM, MM_OP_CHOL_SYRK, MM_OP_CHOL_GEMM, MM_OP_NBODY) = range(14)
 MM_OPK_KERNEL, MM_OPK_XFER, MM_OPK_BARRIER, MM_OPK_FLUSH = 1, 2, 3, 4
 (MM_APP_STREAM, MM_APP_HOTSPOT, MM_APP_STENCIL_REDUCTION, MM_APP_BLACKSCHOLES, MM_APP_SGEMM,
- MM_APP_CHOLESKY) = 1, 2, 3, 4, 5, 6
+ MM_APP_CHOLESKY, MM_APP_NBODY) = 1, 2, 3, 4, 5, 6, 7
 
 STRATEGY_NAMES = {MM_SP_SINGLE: "SP-Single", MM_SP_UNIFIED: "SP-Unified", MM_SP_VARIED: "SP-Varied",
                   MM_DP_PERF: "DP-Perf", MM_DP_DEP: "DP-Dep", MM_SP_CYCLIC: "SP-Cyclic"}

@@ -80,6 +80,23 @@ class Session:
     def fill(self, integer: bool = False, seed: int = synthgen.SEED, recipe=None):
         """Generate the app's inputs in place on every owned device (resident
         mode) with the device counter hash (= synthgen)."""
+        if self.app_id == mm.MM_APP_NBODY and recipe is None:
+            # synthgen.nbody: positions U[-1,1)^3 with masses U[0.5,1) in w,
+            # velocities U[-0.01,0.01)^3 with w = 0 (strided fills of the float4s)
+            _, n4 = mm.mm_app_buffer_info(self.app, 0)
+            n = n4 // 4
+            for d in range(self.G):
+                if not self.mine[d]:
+                    continue
+                p, v = self.bufs[(0, d)], self.bufs[(2, d)]
+                mm.mm_fill_uniform(self.ctx, d, p.data_ptr(), n4, seed, synthgen.AID_NB_P, 0, -1.0, 1.0)
+                mm.mm_fill_uniform(self.ctx, d, v.data_ptr(), n4, seed, synthgen.AID_NB_V, 0, -0.01, 0.01)
+                m = torch.empty(n, dtype=torch.float32, device=p.device)
+                mm.mm_fill_uniform(self.ctx, d, m.data_ptr(), n, seed, synthgen.AID_NB_P + 100, 0, 0.5, 1.0)
+                p.view(n, 4)[:, 3].copy_(m)
+                v.view(n, 4)[:, 3].zero_()
+            torch.cuda.synchronize()
+            return
         if self.app_id == mm.MM_APP_CHOLESKY and recipe is None:
             _, nn = mm.mm_app_buffer_info(self.app, 0)
             n = int(round(nn ** 0.5))

@@ -140,3 +140,17 @@ def spd_random(n: int, seed: int = SEED):
     s = uniform(n * n, AID_CHOL_S, 0.0, 1.0, seed).reshape(n, n).astype(np.float64)
     a = (s + s.T) * 0.5 + n * np.eye(n)
     return a.astype(np.float32)
+
+
+AID_NB_P, AID_NB_V = 51, 52
+
+
+def nbody(n: int, seed: int = SEED):
+    """Positions U[-1,1)^3 with masses U[0.5,1) (w), velocities U[-0.01,0.01)^3
+    with w = 0; (n, 4) float32 each."""
+    p = uniform(4 * n, AID_NB_P, -1.0, 1.0, seed).reshape(n, 4)
+    m = uniform(n, AID_NB_P + 100, 0.5, 1.0, seed)
+    p[:, 3] = m
+    v = uniform(4 * n, AID_NB_V, -0.01, 0.01, seed).reshape(n, 4)
+    v[:, 3] = 0.0
+    return p, v

@@ -215,3 +215,38 @@ def test_cholesky_random_spd():
 def test_cholesky_rejects_indefinite():
     with pytest.raises(ValueError):
         on.cholesky(np.array([[1.0, 2.0], [2.0, 1.0]]))
+
+
+# ----------------------------------------------------------------- Nbody ---
+def test_nbody_two_body_closed_form():
+    # two bodies on the x axis: a_1 = m_2 r / (r^2 + eps2)^{3/2}, equal and
+    # opposite momentum change; one step of the semi-implicit Euler integrator
+    pos = np.array([[0.0, 0, 0, 2.0], [0.5, 0, 0, 3.0]], np.float32)
+    vel = np.zeros((2, 4), np.float32)
+    dt, eps2 = 1e-3, 1e-2
+    p1, v1 = on.nbody_run(pos, vel, 1, dt, eps2)
+    r = 0.5
+    a0 = 3.0 * r / (r * r + eps2) ** 1.5
+    a1 = -2.0 * r / (r * r + eps2) ** 1.5
+    assert abs(v1[0, 0] - a0 * dt) < 1e-6 * abs(a0 * dt)
+    assert abs(v1[1, 0] - a1 * dt) < 1e-6 * abs(a1 * dt)
+    assert abs(p1[0, 0] - a0 * dt * dt) < 1e-9 and v1[0, 1] == 0 and v1[0, 2] == 0
+    assert abs(2.0 * v1[0, 0] + 3.0 * v1[1, 0]) < 1e-9        # momentum conserved
+    assert p1[0, 3] == 2.0 and p1[1, 3] == 3.0                 # masses carried
+
+
+def test_nbody_single_body_at_rest_and_drift():
+    p, v = on.nbody_run(np.array([[0.3, -0.2, 0.1, 1.0]], np.float32),
+                        np.array([[1.0, 2.0, -1.0, 0.0]], np.float32), 5)
+    # self-interaction contributes 0 (softened): uniform motion
+    assert np.allclose(p[0, :3], [0.3 + 5e-3, -0.2 + 1e-2, 0.1 - 5e-3], atol=1e-7)
+    assert np.array_equal(v, np.array([[1.0, 2.0, -1.0, 0.0]], np.float32))
+
+
+def test_nbody_momentum_conservation_many():
+    pos, vel = synthgen.nbody(300)
+    p1, v1 = on.nbody_run(pos, vel, 1)
+    m = pos[:, 3].astype(np.float64)
+    dp = (m[:, None] * (v1[:, :3].astype(np.float64) - vel[:, :3].astype(np.float64))).sum(0)
+    # sum_i m_i a_i = 0 analytically; FP32 storage of v' rounds each term
+    assert np.max(np.abs(dp)) < 300 * 2.0 * 6e-8 * np.max(np.abs(v1[:, :3]))
