@@ -216,7 +216,11 @@ typedef struct {
                                 inputs (one run); 0 (default) = steady-state program,
                                 planned from the state the program itself leaves, valid
                                 for the first run and every repeated run (R22) */
-  int32_t _pad;
+  int32_t pipeline;          /* staged SP-Single/SP-Unified plans of pointwise apps (no halo,
+                                no whole-buffer operand, no sync): split every device range
+                                into this many sub-chunks run chunk-major, each flushed to
+                                the host as soon as it is final, so H2D, kernels and D2H of
+                                different sub-chunks overlap on separate streams (0/1 = off) */
   const mm_range* split;     /* optional SP split override [K*G] */
 } mm_plan_opts;
 

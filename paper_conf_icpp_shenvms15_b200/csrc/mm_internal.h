@@ -77,6 +77,8 @@ struct Plan {
   std::vector<Task> tasks;            // creation order
   std::vector<int32_t> task_dev;
   std::vector<uint64_t> task_fin;     // DP-Perf model finish (ns)
+  bool pipelined = false;             // staged sub-chunk pipeline (mm_plan_opts.pipeline)
+  std::vector<uint8_t> flush_after;   // pipelined: flush the group's outputs after task t
   std::vector<mm_op_rec> ops;         // global op program
   std::vector<int32_t> op_stream;     // executing logical device (-1 barrier)
   std::vector<std::vector<Wait>> waits;   // per op

@@ -29,7 +29,9 @@ std::atomic<int64_t> g_kernel_launches{0};
 struct DevRt {
   int32_t phys = 0, budget = 0, sms = 0, rank = 0;
   Scratch scr;               // device scratch for builtin kernels (e.g. 3xTF32 operand split)
-  cudaStream_t stream = nullptr;
+  cudaStream_t stream = nullptr;      // compute stream (kernels, device<->device pulls)
+  cudaStream_t h2d = nullptr;         // host->device copies (staged inputs)
+  cudaStream_t d2h = nullptr;         // device->host copies (flushes)
   CUgreenCtx gctx = nullptr;
   CUcontext gcu = nullptr;   // CUcontext view of the green context
   bool mine = false;
@@ -238,7 +240,9 @@ void compute_batches(const Plan& plan, PlanRt* rt) {
       std::fill(last_on_dev.begin(), last_on_dev.end(), -1);
       continue;
     }
-    const int32_t d = plan.op_stream[i];
+    const int32_t sid = plan.op_stream[i];
+    if (sid >= plan.G) continue;  // copy-stream ops do not interrupt a compute-stream batch
+    const int32_t d = sid;
     if (op.kind != MM_OPK_KERNEL || !is_batchable_op(plan.app.kernels[op.kernel].op)) {
       if (d >= 0) last_on_dev[d] = -1;
       continue;
@@ -297,6 +301,14 @@ int32_t first_owned(const mm_ctx* ctx) {
   for (int32_t d = 0; d < ctx->G; ++d)
     if (ctx->dev[d].mine) return d;
   return -1;
+}
+
+// Op stream ids of the planner: sid = kind * G + d (kind 0 compute, 1 H2D, 2 D2H).
+inline int32_t sid_dev(const mm_ctx* ctx, int32_t sid) { return sid % ctx->G; }
+inline cudaStream_t sid_stream(const mm_ctx* ctx, int32_t sid) {
+  const DevRt& r = ctx->dev[sid % ctx->G];
+  const int32_t kind = sid / ctx->G;
+  return kind == 0 ? r.stream : (kind == 1 ? r.h2d : r.d2h);
 }
 
 }  // namespace
@@ -480,17 +492,17 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
     const int32_t G = ctx->G;
     rt->ev.assign(plan.ops.size(), nullptr);
     for (size_t i = 0; i < plan.ops.size(); ++i)
-      if (plan.needs_event[i] && plan.op_stream[i] >= 0 && ctx->dev[plan.op_stream[i]].mine) {
-        CU_OK(set_dev(ctx, plan.op_stream[i]));
+      if (plan.needs_event[i] && plan.op_stream[i] >= 0 && ctx->dev[sid_dev(ctx, plan.op_stream[i])].mine) {
+        CU_OK(set_dev(ctx, sid_dev(ctx, plan.op_stream[i])));
         CU_OK(cudaEventCreateWithFlags(&rt->ev[i], cudaEventDisableTiming));
       }
-    rt->bar_ev.assign(G, nullptr);
-    rt->join_ev.assign(G, nullptr);
-    for (int32_t d = 0; d < G; ++d) {
-      if (!ctx->dev[d].mine) continue;
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaEventCreateWithFlags(&rt->bar_ev[d], cudaEventDisableTiming));
-      CU_OK(cudaEventCreateWithFlags(&rt->join_ev[d], cudaEventDisableTiming));
+    rt->bar_ev.assign(3 * G, nullptr);
+    rt->join_ev.assign(3 * G, nullptr);
+    for (int32_t sid = 0; sid < 3 * G; ++sid) {
+      if (!ctx->dev[sid % G].mine) continue;
+      CU_OK(set_dev(ctx, sid % G));
+      CU_OK(cudaEventCreateWithFlags(&rt->bar_ev[sid], cudaEventDisableTiming));
+      CU_OK(cudaEventCreateWithFlags(&rt->join_ev[sid], cudaEventDisableTiming));
     }
     const int32_t root = first_owned(ctx);
     CU_OK(set_dev(ctx, root));
@@ -555,38 +567,39 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
   const int32_t G = ctx->G;
   const App& app = plan.app;
-  std::vector<uint8_t> used(G, 0);
+  const int32_t NS = 3 * G;
+  std::vector<uint8_t> used(NS, 0);
   for (int32_t d : plan.task_dev) used[d] = 1;
-  for (auto& op : plan.ops)
-    if (op.kind != MM_OPK_BARRIER) used[op.device] = 1;
+  for (size_t i = 0; i < plan.ops.size(); ++i)
+    if (plan.op_stream[i] >= 0) used[plan.op_stream[i]] = 1;
   const int32_t root = first_owned(ctx);
   used[root] = 1;
   // fork
   CU_OK(set_dev(ctx, root));
   CU_OK(cudaEventRecord(rt->fork, ctx->dev[root].stream));
-  for (int32_t d = 0; d < G; ++d)
-    if (used[d] && d != root) {
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->fork, 0));
+  for (int32_t sid = 0; sid < NS; ++sid)
+    if (used[sid] && sid != root) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), rt->fork, 0));
     }
   for (size_t i = 0; i < plan.ops.size(); ++i) {
     const mm_op_rec& op = plan.ops[i];
     if (op.kind == MM_OPK_BARRIER) {
-      for (int32_t d = 0; d < G; ++d)
-        if (used[d]) {
-          CU_OK(set_dev(ctx, d));
-          CU_OK(cudaEventRecord(rt->bar_ev[d], ctx->dev[d].stream));
+      for (int32_t sid = 0; sid < NS; ++sid)
+        if (used[sid]) {
+          CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+          CU_OK(cudaEventRecord(rt->bar_ev[sid], sid_stream(ctx, sid)));
         }
-      for (int32_t d = 0; d < G; ++d)
-        if (used[d]) {
-          CU_OK(set_dev(ctx, d));
-          for (int32_t q = 0; q < G; ++q)
-            if (used[q] && q != d) CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->bar_ev[q], 0));
+      for (int32_t sid = 0; sid < NS; ++sid)
+        if (used[sid]) {
+          CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+          for (int32_t q = 0; q < NS; ++q)
+            if (used[q] && q != sid) CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), rt->bar_ev[q], 0));
         }
       continue;
     }
-    const int32_t d = plan.op_stream[i];
-    cudaStream_t s = ctx->dev[d].stream;
+    const int32_t d = sid_dev(ctx, plan.op_stream[i]);
+    cudaStream_t s = sid_stream(ctx, plan.op_stream[i]);
     if (op.kind == MM_OPK_KERNEL && rt->batch_head[i] >= 0) continue;  // launched with its head
     CU_OK(set_dev(ctx, d));
     for (auto& w : plan.waits[i]) CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
@@ -637,12 +650,12 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
     if (plan.needs_event[i]) CU_OK(cudaEventRecord(rt->ev[i], s));
   }
   // join
-  for (int32_t d = 0; d < G; ++d)
-    if (used[d] && d != root) {
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaEventRecord(rt->join_ev[d], ctx->dev[d].stream));
+  for (int32_t sid = 0; sid < NS; ++sid)
+    if (used[sid] && sid != root) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      CU_OK(cudaEventRecord(rt->join_ev[sid], sid_stream(ctx, sid)));
       CU_OK(set_dev(ctx, root));
-      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[d], 0));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[sid], 0));
     }
   return MM_OK;
 }
@@ -756,22 +769,23 @@ mm_status adaptive_issue_op(mm_ctx* ctx, AdaptiveState* ad, size_t i, void* cons
   const mm_op_rec& op = ap.ops[i];
   if (op.kind == MM_OPK_BARRIER) {
     // every stream waits for every other stream's last op
-    std::vector<cudaEvent_t> evs(G, nullptr);
-    for (int32_t d = 0; d < G; ++d) {
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaEventCreateWithFlags(&evs[d], cudaEventDisableTiming));
-      CU_OK(cudaEventRecord(evs[d], ctx->dev[d].stream));
+    const int32_t NS = 3 * G;
+    std::vector<cudaEvent_t> evs(NS, nullptr);
+    for (int32_t sid = 0; sid < NS; ++sid) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      CU_OK(cudaEventCreateWithFlags(&evs[sid], cudaEventDisableTiming));
+      CU_OK(cudaEventRecord(evs[sid], sid_stream(ctx, sid)));
     }
-    for (int32_t d = 0; d < G; ++d) {
-      CU_OK(set_dev(ctx, d));
-      for (int32_t q = 0; q < G; ++q)
-        if (q != d) CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, evs[q], 0));
+    for (int32_t sid = 0; sid < NS; ++sid) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      for (int32_t q = 0; q < NS; ++q)
+        if (q != sid) CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), evs[q], 0));
     }
     for (auto e : evs) cudaEventDestroy(e);
     return MM_OK;
   }
-  const int32_t d = ap.op_stream[i];
-  cudaStream_t s = ctx->dev[d].stream;
+  const int32_t d = sid_dev(ctx, ap.op_stream[i]);
+  cudaStream_t s = sid_stream(ctx, ap.op_stream[i]);
   CU_OK(set_dev(ctx, d));
   mm_status r = adaptive_event(ctx, ad, i, d);
   if (r) return r;
@@ -836,10 +850,10 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
   if (!ad->t0) CU_OK(cudaEventCreate(&ad->t0));
   CU_OK(cudaEventRecord(ad->t0, ctx->dev[root].stream));
   CU_OK(cudaEventRecord(rt->fork, ctx->dev[root].stream));
-  for (int32_t d = 0; d < G; ++d)
-    if (d != root) {
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaStreamWaitEvent(ctx->dev[d].stream, rt->fork, 0));
+  for (int32_t sid = 0; sid < 3 * G; ++sid)
+    if (sid != root) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), rt->fork, 0));
     }
   const auto h0 = std::chrono::steady_clock::now();
   auto now_ns = [&]() -> uint64_t {
@@ -967,12 +981,12 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
     if (r) return r;
   }
   // join
-  for (int32_t d = 0; d < G; ++d)
-    if (d != root) {
-      CU_OK(set_dev(ctx, d));
-      CU_OK(cudaEventRecord(rt->join_ev[d], ctx->dev[d].stream));
+  for (int32_t sid = 0; sid < 3 * G; ++sid)
+    if (sid != root) {
+      CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
+      CU_OK(cudaEventRecord(rt->join_ev[sid], sid_stream(ctx, sid)));
       CU_OK(set_dev(ctx, root));
-      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[d], 0));
+      CU_OK(cudaStreamWaitEvent(ctx->dev[root].stream, rt->join_ev[sid], 0));
     }
   CU_OK(set_dev(ctx, root));
   CU_OK(cudaStreamSynchronize(ctx->dev[root].stream));
@@ -1057,6 +1071,8 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
     if (!any_budget) {
       CU_OK(cudaSetDevice(r.phys));
       CU_OK(cudaStreamCreateWithFlags(&r.stream, cudaStreamNonBlocking));
+      CU_OK(cudaStreamCreateWithFlags(&r.h2d, cudaStreamNonBlocking));
+      CU_OK(cudaStreamCreateWithFlags(&r.d2h, cudaStreamNonBlocking));
       continue;
     }
     if (r.gctx) continue;
@@ -1085,6 +1101,10 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       CUstream cs;
       DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
       rq.stream = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.h2d = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.d2h = (cudaStream_t)cs;
       rq.sms = (int32_t)grp.sm.smCount;
       rest = remaining;
     }
@@ -1098,6 +1118,10 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       CUstream cs;
       DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
       rq.stream = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.h2d = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.d2h = (cudaStream_t)cs;
       rq.sms = (int32_t)rest.sm.smCount;
     }
   }
@@ -1135,9 +1159,10 @@ void mm_ctx_destroy(mm_ctx* ctx) {
   for (auto& r : ctx->dev) {
     if (!r.mine) continue;
     cudaSetDevice(r.phys);
-    if (r.stream) {
-      if (r.gctx) drv().StreamDestroy((CUstream)r.stream);
-      else cudaStreamDestroy(r.stream);
+    for (cudaStream_t st : {r.stream, r.h2d, r.d2h}) {
+      if (!st) continue;
+      if (r.gctx) drv().StreamDestroy((CUstream)st);
+      else cudaStreamDestroy(st);
     }
     if (r.scr.ptr) cudaFree(r.scr.ptr);
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);

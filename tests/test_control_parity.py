@@ -264,6 +264,28 @@ def test_plan_cholesky(strategy):
         mm.mm_app_destroy(capp)
 
 
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_plan_staged_pipeline(P):
+    rnd = random.Random(90 + P)
+    for trial in range(4):
+        G = rnd.randint(1, 3)
+        capp, oapp = stream_pair(rnd.choice([100, 777, 4099]), rnd.choice([1, 2]), 0, 32, 1)
+        pc, po = rand_profile(rnd, G, 4)
+        plan = mm.mm_plan_build(capp, pc, mm.plan_opts(oc.SP_UNIFIED, staged=True, pipeline=P))
+        ranges = oc.sp_split(oapp, po, oc.SP_UNIFIED)
+        tasks, dev, flush = oc.sp_tasks_pipelined(oapp, ranges, P)
+        ops = oc.op_program(oapp, G, tasks, dev, oc.SP_UNIFIED, True, None, flush)
+        ch = mm.mm_plan_chunks(plan)
+        assert [c.device for c in ch] == dev
+        assert [(c.items.begin, c.items.end) for c in ch] == [(t.begin, t.end) for t in tasks]
+        assert ops_as_tuples(plan) == ops
+        # every written element is flushed exactly once
+        fl = [o for o in ops if o[0] == oc.OP_FLUSH]
+        assert sum(o[4] - o[3] for o in fl) == 3 * oapp.kernels[0].n_items
+        mm.mm_plan_destroy(plan)
+        mm.mm_app_destroy(capp)
+
+
 @pytest.mark.parametrize("strategy", [oc.SP_UNIFIED, oc.SP_VARIED, oc.DP_PERF])
 def test_plan_staged(strategy):
     rnd = random.Random(31 + strategy)
