@@ -159,6 +159,10 @@ mm_status mm_app_set_loop(mm_app* app, int32_t first, int32_t last, int64_t iter
 mm_status mm_app_set_sync(mm_app* app, int32_t kernel, int32_t sync);
 /* Ping-pong: slots a and b exchange roles after each loop iteration. */
 mm_status mm_app_set_swap(mm_app* app, int32_t slot_a, int32_t slot_b);
+/* Execution lane of a kernel's tasks on a device (0 default, 1 second compute
+ * stream): independent tasks of different lanes overlap (e.g. the MK-DAG
+ * critical path POTRF/TRSM of step k+1 under the trailing updates of step k). */
+mm_status mm_app_set_lane(mm_app* app, int32_t kernel, int32_t lane);
 /* SK-Loop with unstable per-iteration performance (P117 -> MK-Seq). */
 mm_status mm_app_set_unstable(mm_app* app, int32_t unstable);
 /* Explicit task (MK-DAG).  Tasks are kept in creation order. */

@@ -170,6 +170,10 @@ mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
   }
   const int32_t e[7][2] = {{0, 1}, {1, 2}, {1, 3}, {2, 0}, {3, 1}, {3, 2}, {3, 3}};
   for (auto& x : e) mm_app_add_edge(app, x[0], x[1]);
+  // critical path (POTRF, TRSM) on lane 1: step k+1's panel overlaps step k's
+  // trailing updates (lookahead)
+  mm_app_set_lane(app, 0, 1);
+  mm_app_set_lane(app, 1, 1);
   auto tile = [&](int64_t i, int64_t j) { return (i * T + j) * bb; };
   auto task = [&](int32_t kern, int64_t i, int64_t j, int64_t k,
                   std::initializer_list<std::pair<int32_t, std::pair<int64_t, int64_t>>> a) {

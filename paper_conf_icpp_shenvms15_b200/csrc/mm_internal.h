@@ -29,6 +29,7 @@ struct Kernel {
   int64_t ip[MM_MAX_PARAM] = {0};
   mm_launch_fn launch = nullptr;
   void* user = nullptr;
+  int32_t lane = 0;          // compute stream of the device its tasks run on
 };
 
 // A task's access in element units of a physical buffer.  Reads cover

@@ -32,6 +32,7 @@ struct DevRt {
   cudaStream_t stream = nullptr;      // compute stream (kernels, device<->device pulls)
   cudaStream_t h2d = nullptr;         // host->device copies (staged inputs)
   cudaStream_t d2h = nullptr;         // device->host copies (flushes)
+  cudaStream_t lane1 = nullptr;       // second compute stream (lane-1 kernels)
   CUgreenCtx gctx = nullptr;
   CUcontext gcu = nullptr;   // CUcontext view of the green context
   bool mine = false;
@@ -176,6 +177,8 @@ namespace {
     }                                                                            \
   } while (0)
 
+constexpr int kKinds = 4;   // streams per logical device (see sid_stream)
+
 // Adaptive DP-Perf state of a plan: the op program built incrementally at run
 // time (its ownership directory persists across runs), one end event per op,
 // a begin event per kernel op, and the decision log of the last run.
@@ -225,35 +228,44 @@ bool is_batchable_op(int32_t op) {
 // A member joins only if no other op of that device lies between, all of its
 // cross-stream waits point before the head, and it neither reads nor writes
 // what an earlier member writes (nor writes what an earlier member reads).
+// Batch key: tasks of one batch must share it.  Cholesky lookahead: GEMM
+// updates are batched per output column j and SYRK(k+1, k) runs alone, so
+// step k+1's POTRF / TRSM (lane 1) wait only for the updates they read.
+int64_t batch_key(const Kernel& k, const Task& t) {
+  if (k.op == MM_OP_CHOL_GEMM) return t.ip[2] * 1000003 + t.ip[1];
+  if (k.op == MM_OP_CHOL_SYRK) return t.ip[2] * 2 + (t.ip[0] == t.ip[2] + 1 ? 1 : 0);
+  return t.ip[2];
+}
+
 void compute_batches(const Plan& plan, PlanRt* rt) {
   const size_t n = plan.ops.size();
   rt->batch_head.assign(n, -1);
   rt->members.assign(n, {});
   if (!plan.app.is_dag) return;
-  std::vector<int64_t> last_on_dev(plan.G, -1);   // open batch head per device
+  std::vector<int64_t> open(kKinds * plan.G, -1);   // open batch head per stream
   auto overlap = [](const TaskAcc& a, const TaskAcc& b) {
     return a.buffer == b.buffer && a.lo < b.hi && b.lo < a.hi;
   };
   for (size_t i = 0; i < n; ++i) {
     const mm_op_rec& op = plan.ops[i];
     if (op.kind == MM_OPK_BARRIER) {
-      std::fill(last_on_dev.begin(), last_on_dev.end(), -1);
+      std::fill(open.begin(), open.end(), -1);
       continue;
     }
     const int32_t sid = plan.op_stream[i];
-    if (sid >= plan.G) continue;  // copy-stream ops do not interrupt a compute-stream batch
-    const int32_t d = sid;
     if (op.kind != MM_OPK_KERNEL || !is_batchable_op(plan.app.kernels[op.kernel].op)) {
-      if (d >= 0) last_on_dev[d] = -1;
+      open[sid] = -1;   // any other op on the stream ends its batch
       continue;
     }
-    int64_t h = last_on_dev[d];
-    bool ok = h >= 0 && plan.ops[h].kernel == op.kernel && (int64_t)rt->members[h].size() + 1 < kCholBatch;
+    const Task& t = plan.tasks[op.task];
+    const Kernel& kern = plan.app.kernels[op.kernel];
+    int64_t h = open[sid];
+    bool ok = h >= 0 && plan.ops[h].kernel == op.kernel && (int64_t)rt->members[h].size() + 1 < kCholBatch &&
+              batch_key(kern, plan.tasks[plan.ops[h].task]) == batch_key(kern, t);
     if (ok)
       for (auto& w : plan.waits[i])
         if (w.op >= h) ok = false;
     if (ok) {
-      const Task& t = plan.tasks[op.task];
       std::vector<int64_t> grp = rt->members[h];
       grp.push_back(h);
       for (int64_t m : grp) {
@@ -267,7 +279,7 @@ void compute_batches(const Plan& plan, PlanRt* rt) {
       rt->members[h].push_back((int64_t)i);
       rt->batch_head[i] = h;
     } else {
-      last_on_dev[d] = (int64_t)i;
+      open[sid] = (int64_t)i;
     }
   }
 }
@@ -303,12 +315,13 @@ int32_t first_owned(const mm_ctx* ctx) {
   return -1;
 }
 
-// Op stream ids of the planner: sid = kind * G + d (kind 0 compute, 1 H2D, 2 D2H).
+// Op stream ids of the planner: sid = kind * G + d (kind 0 compute lane 0,
+// 1 H2D, 2 D2H, 3 compute lane 1); kKinds is defined with PlanRt.
 inline int32_t sid_dev(const mm_ctx* ctx, int32_t sid) { return sid % ctx->G; }
 inline cudaStream_t sid_stream(const mm_ctx* ctx, int32_t sid) {
   const DevRt& r = ctx->dev[sid % ctx->G];
   const int32_t kind = sid / ctx->G;
-  return kind == 0 ? r.stream : (kind == 1 ? r.h2d : r.d2h);
+  return kind == 0 ? r.stream : (kind == 1 ? r.h2d : (kind == 2 ? r.d2h : r.lane1));
 }
 
 }  // namespace
@@ -496,9 +509,9 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
         CU_OK(set_dev(ctx, sid_dev(ctx, plan.op_stream[i])));
         CU_OK(cudaEventCreateWithFlags(&rt->ev[i], cudaEventDisableTiming));
       }
-    rt->bar_ev.assign(3 * G, nullptr);
-    rt->join_ev.assign(3 * G, nullptr);
-    for (int32_t sid = 0; sid < 3 * G; ++sid) {
+    rt->bar_ev.assign(kKinds * G, nullptr);
+    rt->join_ev.assign(kKinds * G, nullptr);
+    for (int32_t sid = 0; sid < kKinds * G; ++sid) {
       if (!ctx->dev[sid % G].mine) continue;
       CU_OK(set_dev(ctx, sid % G));
       CU_OK(cudaEventCreateWithFlags(&rt->bar_ev[sid], cudaEventDisableTiming));
@@ -567,7 +580,7 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
   const int32_t G = ctx->G;
   const App& app = plan.app;
-  const int32_t NS = 3 * G;
+  const int32_t NS = kKinds * G;
   std::vector<uint8_t> used(NS, 0);
   for (int32_t d : plan.task_dev) used[d] = 1;
   for (size_t i = 0; i < plan.ops.size(); ++i)
@@ -769,7 +782,7 @@ mm_status adaptive_issue_op(mm_ctx* ctx, AdaptiveState* ad, size_t i, void* cons
   const mm_op_rec& op = ap.ops[i];
   if (op.kind == MM_OPK_BARRIER) {
     // every stream waits for every other stream's last op
-    const int32_t NS = 3 * G;
+    const int32_t NS = kKinds * G;
     std::vector<cudaEvent_t> evs(NS, nullptr);
     for (int32_t sid = 0; sid < NS; ++sid) {
       CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
@@ -850,7 +863,7 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
   if (!ad->t0) CU_OK(cudaEventCreate(&ad->t0));
   CU_OK(cudaEventRecord(ad->t0, ctx->dev[root].stream));
   CU_OK(cudaEventRecord(rt->fork, ctx->dev[root].stream));
-  for (int32_t sid = 0; sid < 3 * G; ++sid)
+  for (int32_t sid = 0; sid < kKinds * G; ++sid)
     if (sid != root) {
       CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
       CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), rt->fork, 0));
@@ -981,7 +994,7 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
     if (r) return r;
   }
   // join
-  for (int32_t sid = 0; sid < 3 * G; ++sid)
+  for (int32_t sid = 0; sid < kKinds * G; ++sid)
     if (sid != root) {
       CU_OK(set_dev(ctx, sid_dev(ctx, sid)));
       CU_OK(cudaEventRecord(rt->join_ev[sid], sid_stream(ctx, sid)));
@@ -1073,6 +1086,11 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       CU_OK(cudaStreamCreateWithFlags(&r.stream, cudaStreamNonBlocking));
       CU_OK(cudaStreamCreateWithFlags(&r.h2d, cudaStreamNonBlocking));
       CU_OK(cudaStreamCreateWithFlags(&r.d2h, cudaStreamNonBlocking));
+      {  // lane 1 carries the critical path: highest stream priority
+        int lo = 0, hi = 0;
+        CU_OK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        CU_OK(cudaStreamCreateWithPriority(&r.lane1, cudaStreamNonBlocking, hi));
+      }
       continue;
     }
     if (r.gctx) continue;
@@ -1105,6 +1123,8 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       rq.h2d = (cudaStream_t)cs;
       DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
       rq.d2h = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, -1));
+      rq.lane1 = (cudaStream_t)cs;
       rq.sms = (int32_t)grp.sm.smCount;
       rest = remaining;
     }
@@ -1122,6 +1142,8 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       rq.h2d = (cudaStream_t)cs;
       DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
       rq.d2h = (cudaStream_t)cs;
+      DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, 0));
+      rq.lane1 = (cudaStream_t)cs;
       rq.sms = (int32_t)rest.sm.smCount;
     }
   }
@@ -1159,7 +1181,7 @@ void mm_ctx_destroy(mm_ctx* ctx) {
   for (auto& r : ctx->dev) {
     if (!r.mine) continue;
     cudaSetDevice(r.phys);
-    for (cudaStream_t st : {r.stream, r.h2d, r.d2h}) {
+    for (cudaStream_t st : {r.stream, r.h2d, r.d2h, r.lane1}) {
       if (!st) continue;
       if (r.gctx) drv().StreamDestroy((CUstream)st);
       else cudaStreamDestroy(st);

@@ -156,6 +156,7 @@ _SIGS = {
     "mm_app_set_sync": [_P, C.c_int32, C.c_int32],
     "mm_app_set_swap": [_P, C.c_int32, C.c_int32],
     "mm_app_set_unstable": [_P, C.c_int32],
+    "mm_app_set_lane": [_P, C.c_int32, C.c_int32],
     "mm_app_add_task": [_P, C.POINTER(mm_task_desc)],
     "mm_app_builtin": [C.c_int32, C.POINTER(mm_app_params), C.POINTER(_P)],
     "mm_app_info": [_P, C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_int64)],
@@ -287,6 +288,10 @@ def mm_app_set_swap(app: int, a: int, b: int):
 
 def mm_app_set_unstable(app: int, unstable: bool):
     _call("mm_app_set_unstable", app, int(unstable))
+
+
+def mm_app_set_lane(app: int, kernel: int, lane: int):
+    _call("mm_app_set_lane", app, kernel, lane)
 
 
 def mm_app_add_task(app: int, kernel: int, iparam: Sequence[int],
