@@ -318,13 +318,16 @@ def main():
         per_launch_ms = dom_ms / dom_launch
         launches_per_step = dom_launch / args.steps
         if args.app == "nbody":
-            # FFMA/MUFU-bound all-pairs: 20 flop per interaction vs the FP32 FMA peak
+            # FP32-pipe-bound all-pairs: 20 flop per interaction (usual count);
+            # the kernel needs 12 FP32 lane-ops per interaction, so the ceiling
+            # is 148 SMs x 128 lanes x 1.965 GHz / 12 interactions/s x 20 flop
             n_b = iparam[0]
             ach = 20 * n_b * items * args.steps / (dom_ms * 1e-3) / 1e12
-            pk = 148 * 128 * 2 * 1.965e9 / 1e12
+            pk = 148 * 128 * 1.965e9 / 12 * 20 / 1e12
             roof = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
-                    "traffic": None, "kernel": "nbody (all pairs, smem tiles)",
-                    "peak_kind": "derived: 148 SMs x 128 FP32 lanes x 2 x 1.965 GHz (B200_PROFILING clocks)"}
+                    "traffic": None, "kernel": "nbody (all pairs, smem tiles, 2 bodies/thread in f32x2)",
+                    "peak_kind": "derived: 148 SMs x 128 FP32 lanes/clk (measured, tools/pipe_rates.cu) x "
+                                 "1.965 GHz / 12 FP32 lane-ops per interaction x 20 flop"}
         elif args.app == "cholesky":
             # trailing GEMM updates on tcgen05 (3xTF32): FP32-equivalent flops vs
             # measured bf16 x 0.5 (tf32) / 3

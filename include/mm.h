@@ -176,7 +176,8 @@ typedef enum {
   MM_APP_BLACKSCHOLES = 4,      /* ip0 n; fp0 R, fp1 V                          */
   MM_APP_SGEMM = 5,             /* ip0 M, ip1 N, ip2 K, ip3 variant             */
   MM_APP_CHOLESKY = 6,          /* ip0 n, ip1 tile b                            */
-  MM_APP_NBODY = 7              /* ip0 bodies, ip1 iterations, ip2 granule, ip3 min; fp0 dt, fp1 eps2 */
+  MM_APP_NBODY = 7              /* ip0 bodies, ip1 iterations, ip2 granule, ip3 min; fp0 dt, fp1 eps2
+                                   (a normal float > 0, else MM_EINVAL) */
 } mm_app_id;
 typedef struct { int64_t iparam[MM_MAX_PARAM]; double fparam[MM_MAX_PARAM]; } mm_app_params;
 mm_status mm_app_builtin(int32_t app_id, const mm_app_params* p, mm_app** out);

@@ -219,6 +219,7 @@ mm_status nbody_app(const mm_app_params& p, mm_app* app) {
   k.iparam[0] = n;
   k.fparam[0] = p.fparam[0] != 0.0 ? p.fparam[0] : 1e-3;   // dt
   k.fparam[1] = p.fparam[1] != 0.0 ? p.fparam[1] : 1e-2;   // softening eps^2
+  if (!((float)k.fparam[1] >= 1.17549435e-38f)) MM_FAIL(MM_EINVAL, "nbody: eps2 must be a normal float > 0");
   mm_status st = mm_app_add_kernel(app, &k, nullptr);
   if (st) return st;
   mm_app_set_swap(app, p0, p1);

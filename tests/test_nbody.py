@@ -80,3 +80,11 @@ def test_nbody_partition_invariance(gpu):
             outs.append(s.collect(plan, 0))
     for o in outs[1:]:
         assert np.array_equal(o, outs[0])
+
+
+@pytest.mark.parametrize("eps2", [-1.0, 1e-40])
+def test_nbody_rejects_non_normal_softening(eps2):
+    """The kernel's rsqrt.approx.ftz equals rsqrtf only for normal d2 >= eps2
+    (include/mm.h MM_APP_NBODY): a negative or denormal eps^2 is MM_EINVAL."""
+    with pytest.raises(mm.MMError):
+        mm.mm_app_builtin(mm.MM_APP_NBODY, [64, 1, 32, 1], [1e-3, eps2])
