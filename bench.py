@@ -53,6 +53,11 @@ APPS = {
               "SK-Loop Nbody 1,048,576 bodies, 1 step (P319; 20 flop/interaction)"),
 }
 FLOP_APPS = ("sgemm", "matmul1k", "cholesky", "nbody")
+# HotSpot temporal block: iterations per launch in the bench
+# step (1000 % HOTSPOT_TB == 0); the result is bit-identical for every value
+HOTSPOT_TB = 4
+# FP32 lane-ops per HotSpot cell update (R16: 9 add/sub + 5 mul)
+HOT_FLOPS = 14
 # kernel whose roofline is reported, and its algorithmic bytes per item
 DOMINANT = {"stream": ("triad", 12), "stream-loop": ("triad", 12), "hotspot": ("hotspot", None),
             "stencil": ("stencil", None), "blackscholes": ("blackscholes", 20), "sgemm": ("sgemm", None),
@@ -208,6 +213,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--app", default="stream", choices=sorted(APPS))
+    ap.add_argument("--tb", type=int, default=None,
+                    help="HotSpot temporal block h (iterations per launch; default 4 for --app hotspot)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
@@ -236,6 +243,10 @@ def main():
     G = world if world > 1 else max(1, args.logical)
     app_id = getattr(mm, APPS[args.app][0])
     iparam = list(APPS[args.app][1])
+    tb = 1
+    if args.app == "hotspot":
+        tb = args.tb if args.tb is not None else HOTSPOT_TB
+        iparam = iparam + [0, 0, tb]
     algo_bytes = APPS[args.app][2](iparam)
     sess = runner.session(app_id, iparam, G=G, cuda_devices=[local] * G, rank=rank, world=world,
                           nccl_id=nccl_id)
@@ -347,6 +358,29 @@ def main():
                     "traffic": None, "kernel": "sgemm (3xTF32 tcgen05, incl. operand split)",
                     "peak_kind": peak_kind + " bf16_tflops x 0.5 (tf32) / 3 (3xTF32)",
                     "avg_launch_ms": per_launch_ms}
+        elif args.app == "hotspot" and tb > 1:
+            # temporal block: per launch 12 B per cell (read T, read P, write T)
+            # for tb updates per cell.  Two ceilings: HBM (12 B / tb per update)
+            # and the FP32 pipe (14 lane-ops per update, 128 lanes/clk/SM,
+            # tools/pipe_rates.cu); the lower one bounds the kernel
+            byts = bpi * items / launches_per_step
+            upd = tb * items * iparam[1] / launches_per_step
+            ach_gbs = byts / (per_launch_ms * 1e-3) / 1e9
+            alu_peak_upd = 148 * 128 * 1.965e9 / HOT_FLOPS
+            hbm_peak_upd = hbm_peak * 1e9 / (12.0 / tb)
+            if hbm_peak_upd <= alu_peak_upd:
+                roof = {"bound": "hbm", "achieved": ach_gbs, "peak": hbm_peak, "unit": "GB/s",
+                        "frac": ach_gbs / hbm_peak, "traffic": None, "kernel": f"hotspot_tb<{tb}>",
+                        "peak_kind": peak_kind + " (MEASURED_PEAKS.json hbm_gbs)"}
+            else:
+                ach_tf = upd * HOT_FLOPS / (per_launch_ms * 1e-3) / 1e12
+                pk = alu_peak_upd * HOT_FLOPS / 1e12
+                roof = {"bound": "alu", "achieved": ach_tf, "peak": pk, "unit": "TFLOP/s", "frac": ach_tf / pk,
+                        "traffic": None, "kernel": f"hotspot_tb<{tb}>",
+                        "peak_kind": "derived: 148 SMs x 128 FP32 lanes/clk x 1.965 GHz; 14 FP32 ops per cell update"}
+            roof.update({"algorithmic_bytes_per_launch": byts, "avg_launch_ms": per_launch_ms,
+                         "cell_updates_per_s": upd / (per_launch_ms * 1e-3),
+                         "ceilings_updates_per_s": {"hbm": hbm_peak_upd, "fp32": alu_peak_upd}})
         else:
             byts = bpi * items / launches_per_step
             ach = byts / (per_launch_ms * 1e-3) / 1e9
@@ -435,7 +469,8 @@ def main():
             "config": {"workload": APPS[args.app][3], "app": args.app, "class": mm.mm_class_name(cls),
                        "strategy": mm.mm_strategy_name(best), "logical_devices": G,
                        "l2": "inputs larger than L2 (1 GiB arrays); no flush",
-                       "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}"},
+                       "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
+                       **({"temporal_block": tb} if args.app == "hotspot" else {})},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
             "clocks": clk.summary(), "strategies_ms": strategies,
             "kernel_ms_per_step": {kname_map[k]: round(sum(kms[d][k] for d in my) / args.steps, 4)

@@ -89,8 +89,12 @@ typedef enum {
   MM_OP_STREAM_SCALE = 2,    /* ops [c R, b W]        b = s c        fparam0 s */
   MM_OP_STREAM_ADD = 3,      /* ops [a R, b R, c W]   c = a + b                */
   MM_OP_STREAM_TRIAD = 4,    /* ops [b R, c R, a W]   a = fma(s,c,b) fparam0 s */
-  MM_OP_HOTSPOT = 5,         /* ops [Tin R halo1, P R, Tout W]; iparam rows,cols;
-                                fparam sdc, rx1, ry1, rz1, amb        (P319)    */
+  MM_OP_HOTSPOT = 5,         /* ops [Tin R halo h, P R, Tout W]; iparam rows,cols,h;
+                                fparam sdc, rx1, ry1, rz1, amb        (P319).
+                                h > 1 (temporal blocking): one
+                                launch = h iterations of rows [b,e), reading
+                                Tin rows [b-h, e+h); needs cols % 4 == 0 and
+                                16-B aligned buffers, h in {2,3,4,6,8}        */
   MM_OP_ROW_RESIDUAL = 6,    /* ops [Tin R, Tout R, rowsum(f64) W]; iparam rows,cols */
   MM_OP_BLACKSCHOLES = 7,    /* ops [S R, X R, T R, call W, put W]; fparam R, V (P311) */
   MM_OP_SGEMM = 8,           /* ops [A R (K per item), B R (whole), C W (N per item)];
@@ -171,7 +175,9 @@ mm_status mm_app_add_task(mm_app* app, const mm_task_desc* task);
 /* Built-in apps of the paper (Table II) and of BASELINE.json configs. */
 typedef enum {
   MM_APP_STREAM = 1,            /* ip0 n, ip1 passes, ip2 sync; fp0 scalar     */
-  MM_APP_HOTSPOT = 2,           /* ip0 rows, ip1 cols, ip2 iterations           */
+  MM_APP_HOTSPOT = 2,           /* ip0 rows, ip1 cols, ip2 iterations, ip3 granule,
+                                   ip4 min rows, ip5 temporal block h (0/1 = none;
+                                   iterations % h == 0, else MM_EINVAL)        */
   MM_APP_STENCIL_REDUCTION = 3, /* ip0 rows, ip1 cols, ip2 steps, ip3 sync      */
   MM_APP_BLACKSCHOLES = 4,      /* ip0 n; fp0 R, fp1 V                          */
   MM_APP_SGEMM = 5,             /* ip0 M, ip1 N, ip2 K, ip3 variant             */

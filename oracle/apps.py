@@ -29,14 +29,17 @@ def stream(n: int, passes: int = 1, sync: int = SYNC_NONE, granule: int = 32,
     return app
 
 
-def hotspot(rows: int, cols: int, iters: int, granule: int = 1, min_items: int = 1) -> App:
+def hotspot(rows: int, cols: int, iters: int, granule: int = 1, min_items: int = 1, tb: int = 1) -> App:
     """HotSpot (P229-233, P319): one stencil kernel iterated (SK-Loop), row-wise
-    split; slots T_in=0, T_out=1 (ping-pong), P=2; halo one row."""
+    split; slots T_in=0, T_out=1 (ping-pong), P=2; halo one row.  With a
+    temporal block tb > 1 one kernel invocation advances tb
+    iterations, so it reads a halo of tb rows and the loop runs iters/tb times."""
+    assert tb >= 1 and iters % tb == 0
     k = Kernel("hotspot", rows, granule, min_items,
-               [Access(0, READ, cols, 1), Access(2, READ, cols, 0), Access(1, WRITE, cols, 0)])
+               [Access(0, READ, cols, tb), Access(2, READ, cols, 0), Access(1, WRITE, cols, 0)])
     app = App(buffers=[(4, rows * cols)] * 3, kernels=[k], swaps=[(0, 1)])
-    if iters > 1:
-        app.loop = (0, 0, iters)
+    if iters // tb > 1:
+        app.loop = (0, 0, iters // tb)
     return app
 
 

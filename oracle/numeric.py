@@ -107,6 +107,22 @@ def hotspot_rows(tin, pw, tout, r0=0, r1=None, coef=None):
                           r0, rows if r1 is None else r1, C.byref(k))
 
 
+def hotspot_block_rows(tin, pw, tout, r0, r1, h, coef=None):
+    """Temporal block of h iterations for rows [r0, r1) (SURVEY §8(f) f3,
+    Rodinia's pyramid): only rows [r0-h, r1+h) of ``tin`` are read.  Written
+    out as h single steps over shrinking row bands: step s (1..h) recomputes
+    rows [r0-h+s, r1+h-s) (clipped to the grid) from step s-1, so step h holds
+    rows [r0, r1) exactly as h full-grid iterations would (P319 + R16)."""
+    rows, cols = tin.shape
+    cur = np.array(tin, dtype=np.float32, copy=True)
+    for s in range(1, h + 1):
+        lo, hi = max(0, r0 - h + s), min(rows, r1 + h - s)
+        nxt = cur.copy()
+        hotspot_rows(cur, pw, nxt, lo, hi, coef)
+        cur = nxt
+    tout[r0:r1] = cur[r0:r1]
+
+
 def hotspot_run(t0, pw, iters):
     rows, cols = t0.shape
     a = np.ascontiguousarray(t0, dtype=np.float32).copy()

@@ -77,19 +77,25 @@ mm_status hotspot_app(const mm_app_params& p, mm_app* app) {
   const int64_t rows = p.iparam[0], cols = p.iparam[1], iters = std::max<int64_t>(1, p.iparam[2]);
   const int64_t g = p.iparam[3] > 0 ? p.iparam[3] : 1;
   const int64_t mn = p.iparam[4] > 0 ? p.iparam[4] : hot_wave_rows(cols);
+  // temporal blocking: each launch advances tb iterations
+  // with a halo of tb rows; the loop runs iters / tb times
+  const int64_t tb = p.iparam[5] > 1 ? p.iparam[5] : 1;
   if (rows <= 0 || cols <= 0) MM_FAIL(MM_EINVAL, "hotspot: shape");
+  if (tb > 1 && (iters % tb != 0 || cols % 4 != 0 || !(tb <= 4 || tb == 6 || tb == 8)))
+    MM_FAIL(MM_EINVAL, "hotspot: temporal block %lld needs iterations %% tb == 0, cols %% 4 == 0, tb in {2,3,4,6,8}",
+            (long long)tb);
   int32_t tin, tout, pw;
   mm_app_add_buffer(app, 4, rows * cols, &tin);
   mm_app_add_buffer(app, 4, rows * cols, &tout);
   mm_app_add_buffer(app, 4, rows * cols, &pw);
   mm_kernel_desc k = kd("hotspot", MM_OP_HOTSPOT, rows, g, mn);
-  acc(k, tin, MM_READ, cols, 1); acc(k, pw, MM_READ, cols); acc(k, tout, MM_WRITE, cols);
-  k.iparam[0] = rows; k.iparam[1] = cols;
+  acc(k, tin, MM_READ, cols, (int32_t)tb); acc(k, pw, MM_READ, cols); acc(k, tout, MM_WRITE, cols);
+  k.iparam[0] = rows; k.iparam[1] = cols; k.iparam[2] = tb;
   hot_params(k.fparam, p.fparam);
   mm_status st = mm_app_add_kernel(app, &k, nullptr);
   if (st) return st;
   mm_app_set_swap(app, tin, tout);
-  if (iters > 1) mm_app_set_loop(app, 0, 0, iters);
+  if (iters / tb > 1) mm_app_set_loop(app, 0, 0, iters / tb);
   return MM_OK;
 }
 

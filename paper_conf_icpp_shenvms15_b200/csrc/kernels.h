@@ -49,7 +49,7 @@ cudaError_t stream_triad(const float* b, const float* c, float* a, float q, int6
 // HotSpot + residual (kernels_stencil.cu)
 struct HotCoef { float sdc, rx1, ry1, rz1, amb; };
 cudaError_t hotspot_rows(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols,
-                         int64_t r0, int64_t r1, HotCoef c, cudaStream_t s, int sms);
+                         int64_t r0, int64_t r1, HotCoef c, cudaStream_t s, int sms, int steps = 1);
 cudaError_t row_residual(const float* t0, const float* t1, double* rowsum, int64_t cols,
                          int64_t r0, int64_t r1, cudaStream_t s, int sms);
 

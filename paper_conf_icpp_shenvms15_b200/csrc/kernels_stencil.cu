@@ -90,6 +90,246 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
   }
 }
 
+// Temporal blocking (Rodinia's "pyramid"): one launch
+// advances rows [r0, r1) by H iterations, reading T rows [r0-H, r1+H) (the
+// halo the ownership directory pulls, access halo = H rows) and P once.
+// Algorithmic HBM bytes per launch: 12 B per cell for H cell-updates.
+//
+// Each WARP owns an independent tile: 128 columns (one float4 group per lane;
+// the HC = 4*ceil(H/4) columns at each end are halo, recomputed by the
+// neighbouring warp) by a strip of SR output rows, and streams down the strip
+// with an H-level software pipeline: at step r, level s = 1..H computes row
+// r-s from the three newest rows of level s-1.  Level-0 (input) rows of T and
+// the P rows arrive through a per-warp shared-memory ring filled by cp.async
+// kTbAhead rows ahead; levels 1..H-1 keep their 3-row windows in registers
+// (slot = row index mod 3, compile-time because the row loop is unrolled by
+// 3).  Horizontal neighbours come from warp shuffles.  The 4 cells of a lane
+// are updated as two f32x2 pairs (FADD2/FMUL2: same round-to-nearest ops in
+// the oracle's order, half the issue slots).  Rows outside the grid are
+// never stored and halo columns lose one valid column per level and are not
+// stored, so every stored cell went through exactly H applications of the
+// R16 update: bit-identical to H single-step launches.
+constexpr int kTbWarps = 4;                      // warps per CTA
+constexpr int kTbAhead = 6;                      // cp.async prefetch distance (rows)
+
+template <int H>
+struct TbCfg {
+  static constexpr int HC = 4 * ((H + 3) / 4);   // halo columns per side (float4-aligned)
+  static constexpr int OW = 128 - 2 * HC;        // output columns per warp
+  static constexpr int RR = (H + kTbAhead + 1) <= 8 ? 8 : 16;   // ring rows (power of 2 > H + ahead)
+};
+
+struct f2 {
+  unsigned long long v;
+};
+__device__ __forceinline__ f2 pk(float a, float b) {
+  f2 r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r.v) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ void upk(f2 x, float& a, float& b) { asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(x.v)); }
+__device__ __forceinline__ f2 add2(f2 a, f2 b) {
+  f2 r;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r.v) : "l"(a.v), "l"(b.v));
+  return r;
+}
+__device__ __forceinline__ f2 sub2(f2 a, f2 b) {
+  f2 r;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r.v) : "l"(a.v), "l"(b.v));
+  return r;
+}
+
+// products as two scalar __fmul_rn: ptxas contracts mul.rn.f32x2 followed by
+// add.rn.f32x2 into FFMA2 (single rounding), which would break R16's order
+__device__ __forceinline__ f2 mul2s(f2 a, float b) {
+  float x, y;
+  upk(a, x, y);
+  return pk(__fmul_rn(x, b), __fmul_rn(y, b));
+}
+
+// cell() on two cells at once (R16 order, every op rounded to nearest)
+__device__ __forceinline__ f2 cell2(f2 c, f2 n, f2 s, f2 w, f2 e, f2 p, float ry1, float rx1, float rz1, f2 amb,
+                                    float sdc) {
+  const f2 two = add2(c, c);
+  const f2 dv = mul2s(sub2(add2(s, n), two), ry1);
+  const f2 dh = mul2s(sub2(add2(e, w), two), rx1);
+  const f2 dz = mul2s(sub2(amb, c), rz1);
+  const f2 sum = add2(add2(add2(p, dv), dh), dz);
+  return add2(c, mul2s(sum, sdc));
+}
+
+struct HotCoef2 {
+  float ry1, rx1, rz1, sdc;
+  f2 amb;
+};
+
+__device__ __forceinline__ float4 cell4(float4 cu, float4 up, float4 dn, float w, float e, float4 p, const HotCoef2& k) {
+  const f2 a = cell2(pk(cu.x, cu.y), pk(up.x, up.y), pk(dn.x, dn.y), pk(w, cu.x), pk(cu.y, cu.z), pk(p.x, p.y),
+                     k.ry1, k.rx1, k.rz1, k.amb, k.sdc);
+  const f2 b = cell2(pk(cu.z, cu.w), pk(up.z, up.w), pk(dn.z, dn.w), pk(cu.y, cu.z), pk(cu.w, e), pk(p.z, p.w),
+                     k.ry1, k.rx1, k.rz1, k.amb, k.sdc);
+  float4 o;
+  upk(a, o.x, o.y);
+  upk(b, o.z, o.w);
+  return o;
+}
+
+__device__ __forceinline__ void cp16(float4* dst, const float* src) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int H>
+struct TbArgs {
+  const float* tin;
+  const float* pw;
+  float* tout;
+  int rows, cols, x0, Y0, Y1, re;   // 32-bit: rows, cols < 2^31 (checked at launch)
+  bool inx, store_x, wedge, eedge;  // lane in the grid; lane stores; chip-edge lanes
+  int lane;
+};
+
+// issue the copies of level-0 row q (T and P) into the ring, one commit group
+template <int H>
+__device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs<H>& a, int q) {
+  constexpr int RR = TbCfg<H>::RR;
+  if (q < a.re && q >= 0 && q < a.rows && a.inx) {
+    const int slot = (q & (RR - 1)) * 32 + a.lane;
+    const int64_t off = (int64_t)q * a.cols + a.x0;
+    cp16(tr + slot, a.tin + off);
+    cp16(pr + slot, a.pw + off);
+  }
+  cp_commit();
+}
+
+// One step r: level s = 1..H computes row r - s.  EDGE = some row of the
+// step is the grid's first or last row (warp-uniform, so interior steps run
+// without the boundary selects).
+template <int H, int PH, bool EDGE>
+__device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3], const float4* tr, const float4* pr,
+                                          const TbArgs<H>& a, int r, const HotCoef2& k) {
+  constexpr int RR = TbCfg<H>::RR;
+  const int rb = r & (RR - 1);
+#pragma unroll
+  for (int s = 1; s <= H; ++s) {
+    const int y = r - s;
+    float4 cu, up, dn;
+    if (s == 1) {                                 // level 0 rows from the ring
+      cu = tr[((rb - 1) & (RR - 1)) * 32 + a.lane];
+      up = tr[((rb - 2) & (RR - 1)) * 32 + a.lane];
+      dn = tr[rb * 32 + a.lane];
+    } else {
+      cu = W[s - 2][((PH - s) % 3 + 3) % 3];
+      up = W[s - 2][((PH - s - 1) % 3 + 3) % 3];
+      dn = W[s - 2][((PH - s + 1) % 3 + 3) % 3];
+    }
+    if (EDGE) {
+      if (y <= 0) up = cu;                        // chip edge: neighbour = the cell itself
+      if (y + 1 >= a.rows) dn = cu;
+    }
+    const float4 p = pr[((rb - s) & (RR - 1)) * 32 + a.lane];
+    float w = __shfl_up_sync(0xffffffffu, cu.w, 1);
+    float e = __shfl_down_sync(0xffffffffu, cu.x, 1);
+    if (a.wedge) w = cu.x;
+    if (a.eedge) e = cu.w;
+    const float4 o = cell4(cu, up, dn, w, e, p, k);
+    if (s < H) {
+      W[s - 1][((PH - s) % 3 + 3) % 3] = o;
+    } else if (a.store_x && y >= a.Y0 && y < a.Y1) {
+      __stcs(reinterpret_cast<float4*>(a.tout + (int64_t)y * a.cols + a.x0), o);
+    }
+  }
+}
+
+template <int H, int PH>
+__device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3], float4* tr, float4* pr, const TbArgs<H>& a,
+                                        int r, const HotCoef2& k) {
+  tb_fetch<H>(tr, pr, a, r + kTbAhead);
+  cp_wait<kTbAhead>();                            // rows <= r landed (each lane reads only its own copies)
+  if (r - H - 1 >= 0 && r + 1 < a.rows)
+    tb_levels<H, PH, false>(W, tr, pr, a, r, k);
+  else
+    tb_levels<H, PH, true>(W, tr, pr, a, r, k);
+}
+
+template <int H>
+__global__ void __launch_bounds__(32 * kTbWarps) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
+                                                             float* __restrict__ tout, int rows, int cols, int r0, int r1,
+                                                             HotCoef kc, int nwx, int SR) {
+  using C = TbCfg<H>;
+  extern __shared__ float4 tb_smem[];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int gw = blockIdx.x * kTbWarps + wid;
+  const int wx = gw % nwx, wy = gw / nwx;
+  TbArgs<H> a;
+  a.tin = tin; a.pw = pw; a.tout = tout; a.rows = rows; a.cols = cols; a.lane = lane;
+  const int64_t y0 = (int64_t)r0 + (int64_t)wy * SR;
+  if (y0 >= r1) return;                           // whole warp exits together
+  a.Y0 = (int)y0;
+  a.Y1 = a.Y0 + SR < r1 ? a.Y0 + SR : r1;
+  const int X0 = wx * C::OW;                      // first output column
+  a.x0 = X0 - C::HC + 4 * lane;                   // this lane's 4 columns
+  a.inx = a.x0 >= 0 && a.x0 < cols;
+  a.store_x = a.inx && a.x0 >= X0 && a.x0 < X0 + C::OW;
+  a.wedge = a.x0 == 0;
+  a.eedge = a.x0 + 4 == cols;
+  float4* tr = tb_smem + (size_t)wid * 2 * C::RR * 32;
+  float4* pr = tr + C::RR * 32;
+  HotCoef2 k;
+  k.ry1 = kc.ry1; k.rx1 = kc.rx1; k.rz1 = kc.rz1; k.sdc = kc.sdc;
+  k.amb = pk(kc.amb, kc.amb);
+  float4 W[H > 1 ? H - 1 : 1][3];
+#pragma unroll
+  for (int i = 0; i < (H > 1 ? H - 1 : 1); ++i)
+#pragma unroll
+    for (int j = 0; j < 3; ++j) W[i][j] = make_float4(0.f, 0.f, 0.f, 0.f);
+  // level-0 rows [rs, re) = [Y0 - H, Y1 + H); at step r level s computes row
+  // r - s, so steps r in [rs + 1, re) end with level H row Y1 - 1
+  const int rs = a.Y0 - H;
+  a.re = a.Y1 + H;
+  // prologue: rows rs .. rs + kTbAhead in flight (step r fetches r + kTbAhead)
+#pragma unroll
+  for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H>(tr, pr, a, rs + q);
+  const int rb = rs + 1, rend = a.re;
+  for (int r = rb; r < rend; r += 3) {
+    tb_step<H, 0>(W, tr, pr, a, r, k);
+    if (r + 1 < rend) tb_step<H, 1>(W, tr, pr, a, r + 1, k);
+    if (r + 2 < rend) tb_step<H, 2>(W, tr, pr, a, r + 2, k);
+  }
+  cp_wait<0>();
+}
+
+template <int H>
+cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
+                      int64_t r1, HotCoef c, cudaStream_t s, int sms) {
+  using C = TbCfg<H>;
+  if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
+  const int64_t nwx = (cols + C::OW - 1) / C::OW;
+  const size_t smem = (size_t)kTbWarps * 2 * C::RR * 32 * sizeof(float4);
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(hotspot_tb<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  // one wave of ~16 warps per SM; strips at least 8H rows tall (vertical
+  // redundancy (2H+1)/SR)
+  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * 16;
+  const int64_t nr = r1 - r0;
+  int64_t nstrip = (target + nwx - 1) / nwx;
+  int64_t SR = (nr + nstrip - 1) / nstrip;
+  if (SR < 8 * H) SR = 8 * H;
+  nstrip = (nr + SR - 1) / SR;
+  const int64_t warps = nwx * nstrip;
+  if (warps + kTbWarps >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
+  hotspot_tb<H><<<(unsigned)((warps + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, smem, s>>>(
+      tin, pw, tout, (int)rows, (int)cols, (int)r0, (int)r1, c, (int)nwx, (int)SR);
+  return cudaGetLastError();
+}
+
 // Generic shapes: one thread per cell.
 __global__ void hotspot_scalar(const float* __restrict__ tin, const float* __restrict__ pw,
                                float* __restrict__ tout, int64_t rows, int64_t cols, int64_t r0,
@@ -147,8 +387,20 @@ __global__ void __launch_bounds__(kThreads) residual_rows(const float* __restric
 }  // namespace
 
 cudaError_t hotspot_rows(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols,
-                         int64_t r0, int64_t r1, HotCoef c, cudaStream_t s, int sms) {
+                         int64_t r0, int64_t r1, HotCoef c, cudaStream_t s, int sms, int steps) {
   if (r1 <= r0) return cudaSuccess;
+  if (steps > 1) {   // temporal blocking: needs float4 rows (cols % 4 == 0, 16-B aligned)
+    if ((cols % 4) != 0 || (((uintptr_t)tin | (uintptr_t)pw | (uintptr_t)tout) & 15u) != 0)
+      return cudaErrorInvalidValue;
+    switch (steps) {
+      case 2: return launch_tb<2>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+      case 3: return launch_tb<3>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+      case 4: return launch_tb<4>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+      case 6: return launch_tb<6>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+      case 8: return launch_tb<8>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   const bool vec = (cols % 4 == 0) && (((uintptr_t)tin | (uintptr_t)pw | (uintptr_t)tout) & 15u) == 0;
   if (vec) {
     const int64_t ncb = (cols / 4 + kThreads - 1) / kThreads;

@@ -367,7 +367,8 @@ cudaError_t launch_builtin(const Launch& L) {
     case MM_OP_STREAM_TRIAD: return stream_triad(f[0], f[1], f[2], (float)k.fp[0], b, e, L.stream, L.sms);
     case MM_OP_HOTSPOT: {
       HotCoef c{(float)k.fp[0], (float)k.fp[1], (float)k.fp[2], (float)k.fp[3], (float)k.fp[4]};
-      return hotspot_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], b, e, c, L.stream, L.sms);
+      return hotspot_rows(f[0], f[1], f[2], k.ip[0], k.ip[1], b, e, c, L.stream, L.sms,
+                          k.ip[2] > 1 ? (int)k.ip[2] : 1);
     }
     case MM_OP_ROW_RESIDUAL:
       return row_residual(f[0], f[1], reinterpret_cast<double*>(L.opnd[2]), k.ip[1], b, e, L.stream, L.sms);

@@ -17,9 +17,9 @@ def stream_pair(n, passes=1, sync=0, granule=32, min_items=1):
     return app, oa.stream(n, passes, sync, granule, min_items)
 
 
-def hotspot_pair(rows, cols, iters, granule=1, min_items=1):
-    app = mm.mm_app_builtin(mm.MM_APP_HOTSPOT, [rows, cols, iters, granule, min_items])
-    return app, oa.hotspot(rows, cols, iters, granule, min_items)
+def hotspot_pair(rows, cols, iters, granule=1, min_items=1, tb=1):
+    app = mm.mm_app_builtin(mm.MM_APP_HOTSPOT, [rows, cols, iters, granule, min_items, tb])
+    return app, oa.hotspot(rows, cols, iters, granule, min_items, tb)
 
 
 def stencil_pair(rows, cols, steps, sync=1, granule=1):
@@ -230,6 +230,26 @@ def test_plan_hotspot(strategy):
         pc, po = rand_profile(rnd, G, 1)
         check_plan(capp, oapp, pc, po, strategy, kpd=rnd.choice([1, 2, 3]))
         mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("strategy", [oc.SP_SINGLE, oc.DP_PERF, oc.DP_DEP])
+def test_plan_hotspot_temporal_block(strategy):
+    """Temporal blocking: halo tb rows, iters/tb launches."""
+    rnd = random.Random(70 + strategy)
+    for trial in range(5):
+        G = rnd.randint(1, 4)
+        tb = rnd.choice([2, 3, 4])
+        capp, oapp = hotspot_pair(rnd.randint(8, 40), rnd.choice([4, 8]), tb * rnd.randint(1, 3), tb=tb)
+        pc, po = rand_profile(rnd, G, 1)
+        check_plan(capp, oapp, pc, po, strategy, kpd=rnd.choice([1, 2, 3]))
+        mm.mm_app_destroy(capp)
+
+
+@pytest.mark.parametrize("ip", [[64, 8, 7, 1, 1, 2], [64, 6, 8, 1, 1, 2], [64, 8, 10, 1, 1, 5]])
+def test_hotspot_temporal_block_rejected(ip):
+    """iterations % tb != 0, cols % 4 != 0, or an unsupported tb: MM_EINVAL."""
+    with pytest.raises(mm.MMError):
+        mm.mm_app_builtin(mm.MM_APP_HOTSPOT, ip)
 
 
 @pytest.mark.parametrize("strategy", [oc.SP_UNIFIED, oc.SP_VARIED, oc.DP_PERF, oc.DP_DEP])

@@ -87,8 +87,13 @@ def _emulate(rank, world, app_id, iparam, strategy, prof_seed):
             else:
                 src, dst = (0, 1) if o.iter % 2 == 0 else (1, 0)
                 rows = iparam[0]
-                on.hotspot_rows(bufs[src].reshape(rows, cols), bufs[2].reshape(rows, cols),
-                                bufs[dst].reshape(rows, cols), b0, e0)
+                tb = iparam[5] if len(iparam) > 5 and iparam[5] > 1 else 1
+                if tb > 1:   # temporal block: tb iterations per kernel, halo tb rows
+                    on.hotspot_block_rows(bufs[src].reshape(rows, cols), bufs[2].reshape(rows, cols),
+                                          bufs[dst].reshape(rows, cols), b0, e0, tb)
+                else:
+                    on.hotspot_rows(bufs[src].reshape(rows, cols), bufs[2].reshape(rows, cols),
+                                    bufs[dst].reshape(rows, cols), b0, e0)
     # assemble on rank 0 from the final owners
     results = {}
     for s in range(3):
@@ -137,6 +142,8 @@ CASES = [
     (mm.MM_APP_HOTSPOT, [41, 16, 5, 1, 1], mm.MM_SP_SINGLE, 5),
     (mm.MM_APP_HOTSPOT, [41, 16, 4, 1, 1], mm.MM_DP_PERF, 6),
     (mm.MM_APP_HOTSPOT, [41, 16, 3, 1, 1], mm.MM_DP_DEP, 7),
+    (mm.MM_APP_HOTSPOT, [41, 16, 6, 1, 1, 2], mm.MM_SP_SINGLE, 8),   # temporal block 2
+    (mm.MM_APP_HOTSPOT, [41, 16, 9, 1, 1, 3], mm.MM_DP_DEP, 9),      # temporal block 3
 ]
 
 
@@ -159,5 +166,6 @@ def test_two_rank_emulation_matches_oracle():
         else:
             t, p = synthgen.hotspot(ip[0], ip[1])
             ref = on.hotspot_run(t, p, ip[2])
-            slot = 0 if ip[2] % 2 == 0 else 1
+            tb = ip[5] if len(ip) > 5 and ip[5] > 1 else 1
+            slot = 0 if (ip[2] // tb) % 2 == 0 else 1
             assert np.array_equal(res[slot].reshape(ip[0], ip[1]), ref), strategy

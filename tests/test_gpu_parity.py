@@ -103,6 +103,28 @@ def test_hotspot_bit_exact(R, shape, strategy, G):
         assert np.array_equal(got, ref), (SP[strategy], G, shape)
 
 
+@pytest.mark.parametrize("tb", [2, 3, 4, 6, 8])
+@pytest.mark.parametrize("shape", [(257, 256), (100, 36), (64, 1032), (37, 4)])
+@pytest.mark.parametrize("strategy", [1, 4, 5])
+@pytest.mark.parametrize("G", [1, 3])
+def test_hotspot_temporal_block_bit_exact(R, tb, shape, strategy, G):
+    """One launch = tb iterations (warp tiles of 128 columns streaming down
+    row strips with a tb-level register pipeline): bit-identical to 24 plain
+    iterations of the oracle, across partitions and halo exchanges."""
+    mm, runner = R
+    rows, cols = shape
+    iters = 24
+    t0, p = synthgen.hotspot(rows, cols)
+    ref = on.hotspot_run(t0, p, iters)
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1, tb], G=G) as s:
+        s.fill()
+        plan = s.plan(strategy, rand_profile(mm, G, 1, rows + strategy + tb), chunks_per_dev=2)
+        s.run(plan)
+        out_slot = 0 if (iters // tb) % 2 == 0 else 1
+        got = s.collect(plan, out_slot).reshape(rows, cols)
+        assert np.array_equal(got, ref), (SP[strategy], G, shape, tb)
+
+
 @pytest.mark.parametrize("strategy", [2, 3, 4, 5])
 def test_stencil_reduction(R, strategy):
     mm, runner = R
@@ -207,6 +229,28 @@ def test_hotspot_full_size_sampled_rows(R):
     for y in sample:
         lo, hi = max(0, y - iters - 1), min(rows, y + iters + 2)
         # window rows at the cut are wrong after k steps only within k rows of the cut
+        ref = on.hotspot_run(t_full[lo:hi], p_full[lo:hi], iters)
+        assert np.array_equal(got[y], ref[y - lo]), y
+
+
+@pytest.mark.parametrize("tb", [4, 8])
+def test_hotspot_temporal_block_full_size_sampled_rows(R, tb):
+    """BASELINE configs[2] grid (8192^2), 2 temporal blocks, in the launch
+    configuration bench.py times: sampled rows (strip and warp-tile seams
+    included) vs the oracle on a row window."""
+    mm, runner = R
+    rows = cols = 8192
+    iters = 2 * tb
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 0, 0, tb], G=1) as s:
+        s.fill()
+        plan = s.plan(1)
+        s.run(plan)
+        out = s.bufs[(0, 0)].view(rows, cols)
+        sample = [0, 1, 2, 127, 128, 255, 256, 4095, 4096, rows - 2, rows - 1]
+        got = {y: out[y].cpu().numpy() for y in sample}
+    t_full, p_full = synthgen.hotspot(rows, cols)
+    for y in sample:
+        lo, hi = max(0, y - iters - 1), min(rows, y + iters + 2)
         ref = on.hotspot_run(t_full[lo:hi], p_full[lo:hi], iters)
         assert np.array_equal(got[y], ref[y - lo]), y
 

@@ -123,6 +123,24 @@ def test_hotspot_row_range_partition_invariance():
     assert np.array_equal(full, part)
 
 
+@pytest.mark.parametrize("h", [1, 2, 3, 5])
+def test_hotspot_block_rows_is_h_full_steps_and_reads_only_the_halo(h):
+    """Temporal block: rows [r0, r1) after one block of h
+    iterations equal h full-grid iterations (P319), and rows of T_in outside
+    [r0-h, r1+h) are never read (poisoned with NaN)."""
+    rows, cols = 29, 13
+    t, p = synthgen.hotspot(rows, cols)
+    full = on.hotspot_run(t, p, h)
+    for r0, r1 in [(0, rows), (0, 7), (9, 17), (20, rows), (14, 15)]:
+        tp = t.copy()
+        tp[: max(0, r0 - h)] = np.nan
+        tp[min(rows, r1 + h):] = np.nan
+        out = np.full_like(t, -1.0)
+        on.hotspot_block_rows(tp, p, out, r0, r1, h)
+        assert np.array_equal(out[r0:r1], full[r0:r1]), (r0, r1)
+        assert np.all(out[:r0] == -1.0) and np.all(out[r1:] == -1.0)
+
+
 def test_hotspot_stable_over_many_iterations():
     # R15 coefficients keep the explicit scheme stable (sum of coefficients
     # < 1): after 1000 iterations the grid stays within the initial range
