@@ -55,7 +55,7 @@ APPS = {
 FLOP_APPS = ("sgemm", "matmul1k", "cholesky", "nbody")
 # HotSpot temporal block: iterations per launch in the bench
 # step (1000 % HOTSPOT_TB == 0); the result is bit-identical for every value
-HOTSPOT_TB = 4
+HOTSPOT_TB = 8
 # FP32 lane-ops per HotSpot cell update (R16: 9 add/sub + 5 mul)
 HOT_FLOPS = 14
 # kernel whose roofline is reported, and its algorithmic bytes per item
