@@ -433,13 +433,16 @@ def main():
         del host
     except Exception as ex:  # report, never hide
         e2e = {"value": None, "unit": unit, "error": str(ex)[:200]}
+    # comparators outside Table I: SP-Cyclic for MK-DAG (P201; BASELINE
+    # configs[4]); §V's DP-Static conversion (P565) for the range apps
+    extras = [mm.MM_SP_CYCLIC] if args.app == "cholesky" else [mm.MM_DP_STATIC]
     if args.app == "cholesky":
-        ranked = list(ranked) + [mm.MM_SP_CYCLIC]   # static comparator (P201; BASELINE configs[4])
+        ranked = list(ranked) + [mm.MM_SP_CYCLIC]
 
     # --- every Table I strategy for this class, w/o and w/ sync (ranking) ----
     strategies = {}
     if not args.no_strategies:
-        for s_id in ranked:
+        for s_id in list(ranked) + [x for x in extras if x not in ranked]:
             try:
                 p = sess.plan(s_id, prof)
                 step(p)

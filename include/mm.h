@@ -59,9 +59,18 @@ typedef enum { MM_SK_ONE = 1, MM_SK_LOOP = 2, MM_MK_SEQ = 3, MM_MK_LOOP = 4,
 
 /* Partitioning strategies, §III-C (P117-119).  MM_SP_CYCLIC is the static
  * 2-D block-cyclic owner-computes mapping used as the "static" comparator for
- * MK-DAG apps (P201; BASELINE configs[4]); it is not part of Table I. */
+ * MK-DAG apps (P201; BASELINE configs[4]); it is not part of Table I.
+ * MM_DP_STATIC is §V's conversion of dynamic partitioning into static (P565):
+ * (1) the static ratio from Glinda's model with the task size = the whole
+ * problem (SP-Single's split for one kernel, SP-Unified's for several on one
+ * index space, else SP-Varied's per kernel); (2) that ratio converted into
+ * task-instance counts per device over the DP chunks (largest remainder,
+ * ties to the lower device id); (3) each device gets its count of
+ * consecutive chunks, in device id order.  Not defined for MK-DAG apps
+ * (MM_EINVAL). */
 typedef enum { MM_SP_SINGLE = 1, MM_SP_UNIFIED = 2, MM_SP_VARIED = 3,
-               MM_DP_PERF = 4, MM_DP_DEP = 5, MM_SP_CYCLIC = 6 } mm_strategy;
+               MM_DP_PERF = 4, MM_DP_DEP = 5, MM_SP_CYCLIC = 6,
+               MM_DP_STATIC = 7 } mm_strategy;
 
 /* Inter-kernel synchronization (P51 taskwait; P119 SP-Varied conditions).
  * BARRIER: all devices finish the kernel before any starts the next.
@@ -379,6 +388,20 @@ typedef struct {
  * devices are done).  buffers as in mm_profile_run. */
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan, void* const* buffers, const mm_run_opts* opts,
                  mm_run_stats* stats);
+
+/* Task-size auto-tuning (§V, P565: "the task size variation leads to
+ * performance variation. Thus, auto-tuning is recommended to find the best
+ * performing one").  For each of the n candidate task counts per device
+ * (chunks_per_dev >= 1), builds the plan `base` with that count (base must
+ * be DP-Perf, DP-Dep or DP-Static, else MM_EINVAL), runs it reps times after
+ * one warm-up run (reps < 1 -> 3) and takes the median device time
+ * (mm_run_stats.device_ms; multi-process: max over ranks, so every rank
+ * picks the same value).  *best = the fastest candidate (ties -> the smaller
+ * count); times_ms[n] (optional, caller-owned) = each candidate's median.
+ * The buffers' contents are overwritten by the runs. */
+mm_status mm_tune_chunks(mm_ctx* ctx, const mm_app* app, const mm_profile* prof, const mm_plan_opts* base,
+                         const int32_t* candidates, int32_t n, void* const* buffers, int32_t reps,
+                         int32_t* best, double* times_ms);
 
 /* Decisions of the last adaptive run of this plan (creation order). */
 mm_status mm_run_decisions(const mm_plan* plan, mm_decision* out, int64_t cap, int64_t* count);

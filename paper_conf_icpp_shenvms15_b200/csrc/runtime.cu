@@ -1344,6 +1344,58 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   return MM_OK;
 }
 
+mm_status mm_tune_chunks(mm_ctx* ctx, const mm_app* app, const mm_profile* prof, const mm_plan_opts* base,
+                         const int32_t* candidates, int32_t n, void* const* buffers, int32_t reps, int32_t* best,
+                         double* times_ms) {
+  if (!ctx || !app || !prof || !base || !candidates || n < 1 || !buffers || !best)
+    MM_FAIL(MM_EINVAL, "tune_chunks: null argument or no candidate");
+  if (base->strategy != MM_DP_PERF && base->strategy != MM_DP_DEP && base->strategy != MM_DP_STATIC)
+    MM_FAIL(MM_EINVAL, "tune_chunks: strategy %d has no task size (DP strategies only)", base->strategy);
+  if (reps < 1) reps = 3;
+  std::vector<double> t(n, 0.0);
+  for (int32_t c = 0; c < n; ++c) {
+    if (candidates[c] < 1) MM_FAIL(MM_EINVAL, "tune_chunks: candidate %d < 1", candidates[c]);
+    mm_plan_opts o = *base;
+    o.chunks_per_dev = candidates[c];
+    mm_plan* p = nullptr;
+    mm_status st = mm_plan_build(app, prof, &o, &p);
+    if (st) return st;
+    std::vector<double> v;
+    for (int32_t r = 0; r <= reps && !st; ++r) {   // run 0 = warm-up
+      mm_run_stats rs{};
+      st = mm_run(ctx, p, buffers, nullptr, &rs);
+      if (r > 0) v.push_back(rs.device_ms);
+    }
+    mm_plan_destroy(p);
+    if (st) return st;
+    std::sort(v.begin(), v.end());
+    t[c] = v[v.size() / 2];
+  }
+  if (ctx->world > 1) {   // every rank must pick the same candidate: max over ranks
+    const int32_t me = first_owned(ctx);
+    CU_OK(cudaSetDevice(ctx->dev[me].phys));
+    double* dbuf = nullptr;
+    CU_OK(cudaMalloc(&dbuf, sizeof(double) * n));
+    cudaStream_t s = ctx->dev[me].stream;
+    cudaError_t e = cudaMemcpyAsync(dbuf, t.data(), sizeof(double) * n, cudaMemcpyHostToDevice, s);
+    ncclResult_t nr = e == cudaSuccess ? nccl().AllReduce(dbuf, dbuf, n, ncclFloat64, ncclMax, ctx->comm, s)
+                                       : ncclSuccess;
+    if (e == cudaSuccess && nr == ncclSuccess)
+      e = cudaMemcpyAsync(t.data(), dbuf, sizeof(double) * n, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && nr == ncclSuccess) e = cudaStreamSynchronize(s);
+    cudaFree(dbuf);
+    if (nr != ncclSuccess) MM_FAIL(MM_ENCCL, "tune_chunks: allreduce failed (%d)", (int)nr);
+    CU_OK(e);
+  }
+  int32_t b = 0;
+  for (int32_t c = 1; c < n; ++c)
+    if (t[c] < t[b] || (t[c] == t[b] && candidates[c] < candidates[b])) b = c;
+  *best = candidates[b];
+  if (times_ms)
+    for (int32_t c = 0; c < n; ++c) times_ms[c] = t[c];
+  return MM_OK;
+}
+
 mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan_h, void* const* buffers, int32_t slot, void* dst,
                      int32_t dst_device) {
   if (!ctx || !plan_h || !buffers || !dst) MM_FAIL(MM_EINVAL, "collect: null argument");

@@ -20,7 +20,7 @@ MM_MAX_DEV, MM_MAX_K, MM_MAX_ACCESS, MM_MAX_BUF, MM_MAX_PARAM = 8, 16, 8, 32, 8
 (MM_OK, MM_EINVAL, MM_ENOMEM, MM_ECUDA, MM_ENCCL, MM_ESTATE, MM_ENOTSUP,
  MM_ERANGE) = 0, -1, -2, -3, -4, -5, -6, -7
 MM_SK_ONE, MM_SK_LOOP, MM_MK_SEQ, MM_MK_LOOP, MM_MK_DAG = 1, 2, 3, 4, 5
-MM_SP_SINGLE, MM_SP_UNIFIED, MM_SP_VARIED, MM_DP_PERF, MM_DP_DEP, MM_SP_CYCLIC = 1, 2, 3, 4, 5, 6
+MM_SP_SINGLE, MM_SP_UNIFIED, MM_SP_VARIED, MM_DP_PERF, MM_DP_DEP, MM_SP_CYCLIC, MM_DP_STATIC = 1, 2, 3, 4, 5, 6, 7
 MM_SYNC_NONE, MM_SYNC_BARRIER, MM_SYNC_FLUSH = 0, 1, 2
 MM_READ, MM_WRITE, MM_RW = 1, 2, 3
 (MM_OP_CUSTOM, MM_OP_STREAM_COPY, MM_OP_STREAM_SCALE, MM_OP_STREAM_ADD, MM_OP_STREAM_TRIAD,
@@ -31,7 +31,8 @@ MM_OPK_KERNEL, MM_OPK_XFER, MM_OPK_BARRIER, MM_OPK_FLUSH = 1, 2, 3, 4
  MM_APP_CHOLESKY, MM_APP_NBODY) = 1, 2, 3, 4, 5, 6, 7
 
 STRATEGY_NAMES = {MM_SP_SINGLE: "SP-Single", MM_SP_UNIFIED: "SP-Unified", MM_SP_VARIED: "SP-Varied",
-                  MM_DP_PERF: "DP-Perf", MM_DP_DEP: "DP-Dep", MM_SP_CYCLIC: "SP-Cyclic"}
+                  MM_DP_PERF: "DP-Perf", MM_DP_DEP: "DP-Dep", MM_SP_CYCLIC: "SP-Cyclic",
+                  MM_DP_STATIC: "DP-Static"}
 CLASS_NAMES = {MM_SK_ONE: "SK-One", MM_SK_LOOP: "SK-Loop", MM_MK_SEQ: "MK-Seq",
                MM_MK_LOOP: "MK-Loop", MM_MK_DAG: "MK-DAG"}
 
@@ -187,6 +188,8 @@ _SIGS = {
     "mm_run": [_P, _P, C.POINTER(_P), C.POINTER(mm_run_opts), C.POINTER(mm_run_stats)],
     "mm_collect": [_P, _P, C.POINTER(_P), C.c_int32, C.c_void_p, C.c_int32],
     "mm_run_decisions": [_P, C.POINTER(mm_decision), C.c_int64, C.POINTER(C.c_int64)],
+    "mm_tune_chunks": [_P, _P, C.POINTER(mm_profile), C.POINTER(mm_plan_opts), C.POINTER(C.c_int32), C.c_int32,
+                       C.POINTER(_P), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_double)],
     "mm_abi_sizes": [C.POINTER(C.c_int64), C.c_int32, C.POINTER(C.c_int32)],
 }
 for _name, _args in _SIGS.items():
@@ -523,6 +526,17 @@ def mm_run(ctx: int, plan: int, buffers: Sequence[int], use_graph: bool = False,
     st = mm_run_stats()
     _call("mm_run", ctx, plan, _ptr_array(buffers), C.byref(o), C.byref(st))
     return st
+
+
+def mm_tune_chunks(ctx: int, app: int, prof: mm_profile, opts: mm_plan_opts, candidates: Sequence[int],
+                   buffers: Sequence[int], reps: int = 3):
+    """-> (best chunks_per_dev, [median device ms per candidate])."""
+    cand = (C.c_int32 * len(candidates))(*candidates)
+    times = (C.c_double * len(candidates))()
+    best = C.c_int32()
+    _call("mm_tune_chunks", ctx, app, C.byref(prof), C.byref(opts), cand, len(candidates), _ptr_array(buffers),
+          reps, C.byref(best), times)
+    return best.value, list(times)
 
 
 def mm_run_decisions(plan: int) -> List[mm_decision]:

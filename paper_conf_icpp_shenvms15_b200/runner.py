@@ -147,6 +147,12 @@ class Session:
     def run(self, plan: int, **kw) -> mm.mm_run_stats:
         return mm.mm_run(self.ctx, plan, self.ptrs(), **kw)
 
+    def tune_chunks(self, strategy: int, prof: mm.mm_profile, candidates=(1, 2, 4, 8, 16, 32), reps: int = 3,
+                    **opts):
+        """Task-size auto-tuning (P565) through mm_tune_chunks -> (best, ms per candidate)."""
+        return mm.mm_tune_chunks(self.ctx, self.app, prof, mm.plan_opts(strategy, **opts), list(candidates),
+                                 self.ptrs(), reps)
+
     def stream(self, d: int = 0) -> torch.cuda.Stream:
         return torch.cuda.ExternalStream(mm.mm_ctx_stream(self.ctx, d), device=f"cuda:{self.cuda_devices[d]}")
 

@@ -84,6 +84,9 @@ def oracle_plan(oapp, po, strategy, kpd=8, staged=False, one_shot=True):
     elif strategy == oc.DP_DEP:
         tasks, dev = oc.dp_dep(oapp, G, kpd)
         fin = [0] * len(tasks)
+    elif strategy == oc.DP_STATIC:
+        tasks, dev = oc.dp_static(oapp, po, kpd)
+        fin = [0] * len(tasks)
     else:
         tasks, dev = oc.sp_cyclic(oapp, G)
         fin = [0] * len(tasks)
@@ -242,6 +245,50 @@ def test_plan_hotspot_temporal_block(strategy):
         capp, oapp = hotspot_pair(rnd.randint(8, 40), rnd.choice([4, 8]), tb * rnd.randint(1, 3), tb=tb)
         pc, po = rand_profile(rnd, G, 1)
         check_plan(capp, oapp, pc, po, strategy, kpd=rnd.choice([1, 2, 3]))
+        mm.mm_app_destroy(capp)
+
+
+def test_plan_dp_static_all_range_apps():
+    """§V conversion (P565): chunk counts from the static ratio, consecutive
+    chunks per device; bit-exact plans (chunks, devices, op program) for
+    SK-One, SK-Loop, MK-Seq/MK-Loop (with and without sync) and MK-Loop
+    stencil+reduction under random heterogeneous profiles."""
+    rnd = random.Random(565)
+    makers = [lambda: bs_pair(rnd.randint(50, 900)), lambda: sgemm_pair(rnd.randint(20, 90), 6, 5),
+              lambda: hotspot_pair(rnd.randint(8, 40), 4, rnd.randint(1, 3)),
+              lambda: stream_pair(rnd.choice([64, 1000, 4099]), rnd.choice([1, 2]), rnd.choice([0, 1, 2]),
+                                  rnd.choice([1, 32]), 1),
+              lambda: stencil_pair(rnd.randint(8, 30), 5, rnd.randint(1, 3), rnd.choice([0, 1]))]
+    for trial in range(12):
+        for mk in makers:
+            capp, oapp = mk()
+            G = rnd.randint(1, 5)
+            K = mm.mm_app_info(capp)[0]
+            pc, po = rand_profile(rnd, G, K)
+            check_plan(capp, oapp, pc, po, oc.DP_STATIC, kpd=rnd.choice([1, 2, 3, 8]))
+            mm.mm_app_destroy(capp)
+
+
+def test_dp_static_counts_follow_the_static_ratio():
+    """Worked case: MatrixMul-like SK-One with a 9:1 cost ratio between two
+    devices (P329: SP-Single puts ~90% on the GPU) and 10 chunks: the slow
+    device gets 1 instance, the fast one 9 (P565 step 2); with 20 chunks, 2
+    and 18; the fast device's chunks come first (P565 step 3)."""
+    app = oa.single("mm", 1000, granule=1)
+    for kpd, want in ((5, (9, 1)), (10, (18, 2))):
+        prof = oc.Profile(G=2, fs_item=[[1000], [9000]], chunk_est_ns=[[1], [1]], link_Bps=[1, 1])
+        tasks, dev = oc.dp_static(app, prof, kpd)
+        assert (dev.count(0), dev.count(1)) == want
+        assert dev == sorted(dev)
+
+
+def test_dp_static_rejects_dag():
+    capp = mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [256, 64])
+    try:
+        with pytest.raises(mm.MMError):
+            mm.mm_plan_build(capp, mm.make_profile(2, [[1000] * 4] * 2, [[1000] * 4] * 2, [10 ** 9] * 2),
+                             mm.plan_opts(mm.MM_DP_STATIC))
+    finally:
         mm.mm_app_destroy(capp)
 
 

@@ -125,6 +125,62 @@ def test_hotspot_temporal_block_bit_exact(R, tb, shape, strategy, G):
         assert np.array_equal(got, ref), (SP[strategy], G, shape, tb)
 
 
+@pytest.mark.parametrize("case", ["stream", "hotspot", "hotspot_tb4", "blackscholes"])
+def test_dp_static_bit_exact(R, case):
+    """§V conversion (P565): DP chunks assigned by the static ratio run
+    through the same engine; results identical to the oracle."""
+    mm, runner = R
+    G = 3
+    if case == "stream":
+        n = 100003
+        with runner.session(mm.MM_APP_STREAM, [n, 2, 0, 32, 1], G=G) as s:
+            s.fill()
+            plan = s.plan(mm.MM_DP_STATIC, rand_profile(mm, G, 4, 7), chunks_per_dev=3)
+            s.run(plan)
+            got = [s.collect(plan, k) for k in range(3)]
+        ref = on.stream_run(*synthgen.stream_random(n), 2)
+        for g_, r_ in zip(got, ref):
+            assert np.array_equal(g_, r_)
+    elif case.startswith("hotspot"):
+        rows, cols, tb = 203, 132, (4 if case.endswith("tb4") else 1)
+        iters = 8
+        t0, p = synthgen.hotspot(rows, cols)
+        ref = on.hotspot_run(t0, p, iters)
+        with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1, tb], G=G) as s:
+            s.fill()
+            plan = s.plan(mm.MM_DP_STATIC, rand_profile(mm, G, 1, 11), chunks_per_dev=4)
+            s.run(plan)
+            got = s.collect(plan, 0 if (iters // tb) % 2 == 0 else 1).reshape(rows, cols)
+        assert np.array_equal(got, ref)
+    else:
+        n = 50021
+        S, X, T = synthgen.blackscholes(n)
+        with runner.session(mm.MM_APP_BLACKSCHOLES, [n, 32, 1], G=G) as s:
+            s.fill()
+            plan = s.plan(mm.MM_DP_STATIC, rand_profile(mm, G, 1, 5), chunks_per_dev=2)
+            s.run(plan)
+            call, put = s.collect(plan, 3), s.collect(plan, 4)
+        rc, rp = on.blackscholes(S, X, T)
+        assert np.max(np.abs(call - rc) / np.maximum(np.abs(rc), 1.0)) < 1e-5
+        assert np.max(np.abs(put - rp) / np.maximum(np.abs(rp), 1.0)) < 1e-5
+
+
+@pytest.mark.parametrize("strategy", [4, 5, 7])
+def test_tune_chunks(R, strategy):
+    """Task-size auto-tuning (P565): the returned count is a candidate with the
+    smallest median time; a non-DP strategy is rejected."""
+    mm, runner = R
+    with runner.session(mm.MM_APP_STREAM, [1 << 20, 1, 0, 32, 1], G=2) as s:
+        s.fill()
+        prof = s.profile(reps=2)
+        cand = [1, 2, 8, 32]
+        best, ms = s.tune_chunks(strategy, prof, cand, reps=2)
+        assert best in cand and all(t > 0 for t in ms)
+        assert ms[cand.index(best)] == min(ms)
+        with pytest.raises(mm.MMError):
+            s.tune_chunks(mm.MM_SP_UNIFIED, prof, cand)
+
+
 @pytest.mark.parametrize("strategy", [2, 3, 4, 5])
 def test_stencil_reduction(R, strategy):
     mm, runner = R

@@ -83,7 +83,9 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 host.append(h)
         times, shares = {}, {}
         adaptive_ms, ad_share = None, None
-        strategies = list(order) + ([mm.MM_SP_CYCLIC] if cls == mm.MM_MK_DAG else [])
+        # comparators outside Table I: SP-Cyclic (MK-DAG, P201); DP-Static,
+        # §V's conversion of dynamic into static partitioning (P565)
+        strategies = list(order) + ([mm.MM_SP_CYCLIC] if cls == mm.MM_MK_DAG else [mm.MM_DP_STATIC])
         for st in strategies:
             p = s.plan(st, prof, staged=staged)
             kw = {"host": [h.data_ptr() for h in host]} if staged else {}
