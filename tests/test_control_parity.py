@@ -375,3 +375,39 @@ def test_errors_are_status_codes():
     with pytest.raises(mm.MMError):
         mm.mm_split(capp, mm.make_profile(2, [[1] * 4] * 2), mm.MM_SP_SINGLE)  # 4 kernels
     mm.mm_app_destroy(capp)
+
+
+def test_het_k_instance_assignment_matches_p329():
+    """HET-k: one fast device + 3 slow ones (6x per-item
+    cost), SK-One app, one task instance per device (kpd = 1).  P329:
+    DP-Dep "does not take into account their different hardware
+    capabilities ... only one task instance is assigned to the GPU";
+    DP-Perf "assigns all the task instances to the GPU"; SP-Single splits by
+    the capability ratio (6 : 1 : 1 : 1 -> 2/3 on the fast device); DP-Static
+    converts that ratio into instance counts (P565)."""
+    n, G = 4096, 4
+    capp, oapp = bs_pair(n)
+    ps = [[1000]] + [[6000]] * 3
+    est = [[10 ** 5]] + [[6 * 10 ** 5]] * 3
+    link = [10 ** 12] * G
+    pc = mm.make_profile(G, ps, est, link)
+    po = oc.Profile(G=G, fs_item=ps, chunk_est_ns=est, link_Bps=link)
+    try:
+        for strategy, kpd in ((oc.DP_DEP, 1), (oc.DP_PERF, 1), (oc.SP_SINGLE, 1), (oc.DP_STATIC, 3)):
+            check_plan(capp, oapp, pc, po, strategy, kpd=kpd)
+        _, dev = oc.dp_dep(oapp, G, 1)
+        assert dev.count(0) == 1                       # one instance on the fast device
+        _, dev, _ = oc.dp_perf(oapp, po, 1)
+        assert dev.count(0) == len(dev)                # all instances on the fast device
+        r = oc.sp_split(oapp, po, oc.SP_SINGLE)[0]
+        share = (r[0][1] - r[0][0]) / n
+        assert abs(share - 2 / 3) < 0.01
+        # SP-Single items [2752, 480, 480, 384] (granule 32); 12 instances:
+        # quotas 12*items/n = [8.06, 1.41, 1.41, 1.13] -> floors [8, 1, 1, 1],
+        # the one left over to the largest remainder (tie d1/d2 -> d1)
+        assert [b - a for a, b in r] == [2752, 480, 480, 384]
+        _, dev = oc.dp_static(oapp, po, 3)
+        assert [dev.count(d) for d in range(G)] == [8, 2, 1, 1]
+        assert dev == sorted(dev)
+    finally:
+        mm.mm_app_destroy(capp)

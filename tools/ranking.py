@@ -44,6 +44,13 @@ APPS = [
 ]
 
 
+# SM budgets per logical device (0 = the rest of the GPU).  HET-k (SURVEY
+# §8(f) f2): one fast device + m slow ones, the paper's GPU + CPU-worker mix
+# (P329: DP-Dep "uses all the CPU cores and the GPU" as equal workers).
+PLATFORMS = {"HET-2": [0, 16], "HOMO-2": [0, 0], "HET-4": [0, 16, 16, 16], "HOMO-4": [0, 0, 0, 0],
+             "HET-8": [0, 8, 8, 8, 8, 8, 8, 8]}
+
+
 def expected_order(cls, sync):
     return mm.mm_rank(cls, sync)
 
@@ -64,7 +71,8 @@ def verdict(order, times):
 
 
 def run_config(name, app_id, ip, budgets, staged, reps):
-    s = runner.session(app_id, ip, G=2, sm_budgets=budgets)
+    G = len(budgets)
+    s = runner.session(app_id, ip, G=G, sm_budgets=budgets)
     try:
         cls = s.classify()
         ns = mm.mm_needs_sync(s.app)
@@ -81,7 +89,7 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 h = torch.empty(max(n, 1), dtype=runner._DT[eb], pin_memory=True)
                 h.copy_(s.bufs[(slot, 0)].cpu())
                 host.append(h)
-        times, shares = {}, {}
+        times, shares, instances = {}, {}, {}
         adaptive_ms, ad_share = None, None
         # comparators outside Table I: SP-Cyclic (MK-DAG, P201); DP-Static,
         # §V's conversion of dynamic into static partitioning (P565)
@@ -101,21 +109,25 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 ta = [s.run(p, adaptive=True).device_ms for _ in range(reps)]
                 adaptive_ms = statistics.median(ta)
                 decs = mm.mm_run_decisions(p)
-                ad_share = [sum(1 for dc in decs if dc.chosen == d) / max(1, len(decs)) for d in range(2)]
+                ad_share = [sum(1 for dc in decs if dc.chosen == d) / max(1, len(decs)) for d in range(G)]
             info = mm.mm_plan_info(p)
-            tot = [sum(info.items[d][k] for k in range(s.K)) for d in range(2)]
+            tot = [sum(info.items[d][k] for k in range(s.K)) for d in range(G)]
+            if st in (mm.MM_DP_PERF, mm.MM_DP_DEP, mm.MM_DP_STATIC):
+                ch = mm.mm_plan_chunks(p)
+                instances[mm.mm_strategy_name(st)] = [sum(1 for c in ch if c.device == d) for d in range(G)]
             shares[mm.mm_strategy_name(st)] = [round(x / max(1, sum(tot)), 4) for x in tot]
         ok, pairs = verdict(order, times)
         return {"app": name, "class": mm.mm_class_name(cls), "needs_sync": ns, "mode": "staged" if staged else "resident",
-                "sms": [mm.mm_ctx_sm_count(s.ctx, 0), mm.mm_ctx_sm_count(s.ctx, 1)],
+                "sms": [mm.mm_ctx_sm_count(s.ctx, d) for d in range(G)],
                 "expected_order": [mm.mm_strategy_name(x) for x in order],
                 "ms": {mm.mm_strategy_name(k): round(v, 4) for k, v in times.items()},
                 "measured_order": [mm.mm_strategy_name(k) for k, _ in sorted(times.items(), key=lambda kv: kv[1])],
-                "share_per_device": shares, "ranking_holds": ok, "pairs": pairs,
+                "share_per_device": shares, "task_instances_per_device": instances,
+                "ranking_holds": ok, "pairs": pairs,
                 "dp_perf_adaptive_ms": None if adaptive_ms is None else round(adaptive_ms, 4),
                 "dp_perf_adaptive_task_share": ad_share,
-                "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(2)],
-                "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(2)]}
+                "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(G)],
+                "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(G)]}
     finally:
         s.close()
 
@@ -125,11 +137,14 @@ def main():
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r1_ranking.json"))
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--platforms", default="HET-2,HOMO-2",
+                    help="comma list of " + ",".join(PLATFORMS))
     args = ap.parse_args()
     torch.cuda.set_device(0)
-    res = {"platforms": {"HET-2": [0, 16], "HOMO-2": None}, "tolerance": TOL, "configs": []}
+    plats = [(n, PLATFORMS[n]) for n in args.platforms.split(",")]
+    res = {"platforms": {n: b for n, b in plats}, "tolerance": TOL, "configs": []}
     t0 = time.time()
-    for pname, budgets in (("HET-2", [0, 16]), ("HOMO-2", [0, 0])):
+    for pname, budgets in plats:
         for name, app_id, ip in APPS:
             modes = [False]
             if app_id == mm.MM_APP_STREAM and not args.quick:
