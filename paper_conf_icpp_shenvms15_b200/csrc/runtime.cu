@@ -14,6 +14,7 @@
 #include <deque>
 #include <memory>
 #include <new>
+#include <map>
 #include <vector>
 
 #include "kernels.h"
@@ -1106,13 +1107,28 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
     CUdevResource all;
     DRV_OK(D.DeviceGetDevResource(cudev, &all, CU_DEV_RESOURCE_TYPE_SM));
     CUdevResource rest = all;
+    // devices with equal budgets are split off in ONE call (nbGroups = their
+    // count): the driver rejects splitting a remainder again on B200
+    std::map<int32_t, std::vector<int32_t>> by_budget;
+    for (int32_t q = 0; q < G; ++q) {
+      DevRt& rq = ctx->dev[q];
+      if (rq.mine && rq.phys == r.phys && rq.budget > 0) by_budget[rq.budget].push_back(q);
+    }
+    std::map<int32_t, CUdevResource> group_of;
+    for (auto& kv : by_budget) {
+      std::vector<CUdevResource> grps(kv.second.size());
+      CUdevResource remaining;
+      unsigned n = (unsigned)kv.second.size();
+      DRV_OK(D.DevSmResourceSplitByCount(grps.data(), &n, &rest, &remaining, 0, (unsigned)kv.first));
+      if (n < kv.second.size())
+        MM_FAIL(MM_ECUDA, "SM split: %u of %zu groups of %d SMs", n, kv.second.size(), kv.first);
+      for (size_t i = 0; i < kv.second.size(); ++i) group_of[kv.second[i]] = grps[i];
+      rest = remaining;
+    }
     for (int32_t q = 0; q < G; ++q) {
       DevRt& rq = ctx->dev[q];
       if (!rq.mine || rq.phys != r.phys || rq.budget <= 0) continue;
-      CUdevResource grp, remaining;
-      unsigned n = 1;
-      DRV_OK(D.DevSmResourceSplitByCount(&grp, &n, &rest, &remaining, 0, (unsigned)rq.budget));
-      if (n < 1) MM_FAIL(MM_ECUDA, "SM split for device %d gave no group", q);
+      CUdevResource grp = group_of[q];
       CUdevResourceDesc desc;
       DRV_OK(D.DevResourceGenerateDesc(&desc, &grp, 1));
       DRV_OK(D.GreenCtxCreate(&rq.gctx, desc, cudev, CU_GREEN_CTX_DEFAULT_STREAM));
@@ -1127,7 +1143,6 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       DRV_OK(D.GreenCtxStreamCreate(&cs, rq.gctx, CU_STREAM_NON_BLOCKING, -1));
       rq.lane1 = (cudaStream_t)cs;
       rq.sms = (int32_t)grp.sm.smCount;
-      rest = remaining;
     }
     for (int32_t q = 0; q < G; ++q) {
       DevRt& rq = ctx->dev[q];

@@ -117,13 +117,15 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 instances[mm.mm_strategy_name(st)] = [sum(1 for c in ch if c.device == d) for d in range(G)]
             shares[mm.mm_strategy_name(st)] = [round(x / max(1, sum(tot)), 4) for x in tot]
         ok, pairs = verdict(order, times)
+        table = {k: v for k, v in times.items() if k in order}
+        top_ok = times[order[0]] <= min(table.values()) * (1 + TOL)
         return {"app": name, "class": mm.mm_class_name(cls), "needs_sync": ns, "mode": "staged" if staged else "resident",
                 "sms": [mm.mm_ctx_sm_count(s.ctx, d) for d in range(G)],
                 "expected_order": [mm.mm_strategy_name(x) for x in order],
                 "ms": {mm.mm_strategy_name(k): round(v, 4) for k, v in times.items()},
                 "measured_order": [mm.mm_strategy_name(k) for k, _ in sorted(times.items(), key=lambda kv: kv[1])],
                 "share_per_device": shares, "task_instances_per_device": instances,
-                "ranking_holds": ok, "pairs": pairs,
+                "ranking_holds": ok, "top_choice_holds": top_ok, "pairs": pairs,
                 "dp_perf_adaptive_ms": None if adaptive_ms is None else round(adaptive_ms, 4),
                 "dp_perf_adaptive_task_share": ad_share,
                 "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(G)],
@@ -156,13 +158,15 @@ def main():
                     r = {"app": name, "mode": "staged" if staged else "resident", "error": str(e)[:300]}
                 r["platform"] = pname
                 res["configs"].append(r)
-                print(json.dumps({k: r.get(k) for k in ("platform", "app", "mode", "ms", "ranking_holds",
+                print(json.dumps({k: r.get(k) for k in ("platform", "app", "mode", "ms", "ranking_holds", "top_choice_holds",
                                                          "dp_perf_adaptive_ms", "share_per_device", "error")}),
                       flush=True)
     res["wall_s"] = round(time.time() - t0, 1)
     held = [c.get("ranking_holds") for c in res["configs"] if "ranking_holds" in c]
+    top = [c.get("top_choice_holds") for c in res["configs"] if "top_choice_holds" in c]
     res["summary"] = {"configs": len(res["configs"]), "ranking_holds": sum(bool(h) for h in held),
-                      "ranking_violated": sum(not h for h in held)}
+                      "ranking_violated": sum(not h for h in held),
+                      "top_choice_holds": sum(bool(h) for h in top), "top_choice_violated": sum(not h for h in top)}
     with open(args.out, "w") as f:
         json.dump(res, f, indent=1)
     print(json.dumps(res["summary"]))
