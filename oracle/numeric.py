@@ -195,14 +195,34 @@ def cholesky(A):
 NBODY_DT, NBODY_EPS2 = 1e-3, 1e-2
 
 
-def nbody_run(pos, vel, iters, dt=NBODY_DT, eps2=NBODY_EPS2):
-    """pos, vel: (n, 4) float32.  Returns (pos, vel) after `iters` steps."""
+def _nbody_lib():
     L = lib()
     if not hasattr(L, "_nbody_ready"):
         f32p = np.ctypeslib.ndpointer(np.float32, flags="C_CONTIGUOUS")
         L.or_nbody_step.argtypes = [f32p, f32p, f32p, f32p, C.c_int64, C.c_int64, C.c_int64,
                                     C.c_double, C.c_double]
         L._nbody_ready = True
+    return L
+
+
+def nbody_step_bodies(pos, vel, bodies, dt=NBODY_DT, eps2=NBODY_EPS2):
+    """One step for the listed bodies only (each sums over ALL n bodies):
+    returns (pos', vel') rows of shape (len(bodies), 4)."""
+    L = _nbody_lib()
+    n = pos.shape[0]
+    p = np.ascontiguousarray(pos, dtype=np.float32)
+    v = np.ascontiguousarray(vel, dtype=np.float32)
+    p2, v2 = np.zeros_like(p), np.zeros_like(v)
+    for i in bodies:
+        L.or_nbody_step(p.reshape(-1), v.reshape(-1), p2.reshape(-1), v2.reshape(-1), n, int(i), int(i) + 1,
+                        dt, eps2)
+    idx = np.asarray(bodies)
+    return p2[idx].copy(), v2[idx].copy()
+
+
+def nbody_run(pos, vel, iters, dt=NBODY_DT, eps2=NBODY_EPS2):
+    """pos, vel: (n, 4) float32.  Returns (pos, vel) after `iters` steps."""
+    L = _nbody_lib()
     n = pos.shape[0]
     p = np.ascontiguousarray(pos, dtype=np.float32).copy()
     v = np.ascontiguousarray(vel, dtype=np.float32).copy()
