@@ -215,6 +215,8 @@ def main():
     ap.add_argument("--app", default="stream", choices=sorted(APPS))
     ap.add_argument("--tb", type=int, default=None,
                     help="HotSpot temporal block h (iterations per launch; default 4 for --app hotspot)")
+    ap.add_argument("--chol-tile", type=int, default=None, help="Cholesky tile b (default 1024)")
+    ap.add_argument("--chol-n", type=int, default=None, help="Cholesky order n (default 32768)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
@@ -247,6 +249,8 @@ def main():
     if args.app == "hotspot":
         tb = args.tb if args.tb is not None else HOTSPOT_TB
         iparam = iparam + [0, 0, tb]
+    if args.app == "cholesky":
+        iparam = [args.chol_n or iparam[0], args.chol_tile or iparam[1]]
     algo_bytes = APPS[args.app][2](iparam)
     sess = runner.session(app_id, iparam, G=G, cuda_devices=[local] * G, rank=rank, world=world,
                           nccl_id=nccl_id)

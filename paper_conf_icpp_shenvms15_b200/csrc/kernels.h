@@ -64,9 +64,9 @@ cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int6
 size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows);
 
 // Cholesky tiles (kernels_chol.cu); A tile-major, T x T tiles of b x b.
-constexpr int kCholBatch = 128;   // tasks per batched launch
-cudaError_t chol_task(int32_t op, float* A, int64_t T, int64_t b, int64_t i, int64_t j, int64_t k,
-                      cudaStream_t s, int sms);
+constexpr int kCholBatch = 512;   // tasks per batched launch (a whole MK-DAG step at T = 32)
+// Device scratch of every Cholesky op: 3xTF32 panel split + POTRF flags.
+size_t chol_scratch_bytes(int64_t T, int64_t b);
 // n independent tasks of one kernel (ijk = n triples) in one launch.
 cudaError_t chol_batch(int32_t op, float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n,
                        cudaStream_t s, int sms, Scratch* scr);
@@ -74,6 +74,14 @@ cudaError_t chol_batch(int32_t op, float* A, int64_t T, int64_t b, const int32_t
 size_t chol_tc_scratch(int64_t T, int64_t b);
 cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n, cudaStream_t s,
                            Scratch* scr);
+
+// TRSM on the split panel slots (kernels_gemm_tc.cu): L_kk split into its
+// slot; slots marked split; block update columns [n0, b) -= X[:, kx0:kx0+K] L^T.
+cudaError_t chol_trsm_prepare(float* A, int64_t T, int64_t b, int32_t k, cudaStream_t s, Scratch* scr,
+                              float** hi, float** lo, int32_t* slot0);
+void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, int32_t n);
+cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n,
+                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr);
 
 // Nbody step for bodies [r0, r1) (kernels_nbody.cu); float4 bodies.
 cudaError_t nbody_rows_launch(const float* pin, const float* vin, float* pout, float* vout, int64_t n, int64_t r0,

@@ -20,6 +20,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <vector>
 
 #include "kernels.h"
 
@@ -37,13 +38,19 @@ constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
 constexpr int SMEM_BYTES = kStages * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 constexpr int kThreadsGemm = 192;
 
-// Batched Cholesky trailing update (mode 1): task z updates tile (ti, tj) of a
-// tile-major matrix, C_tile -= P_i P_j^T, with the split panel tiles at rows
-// slot*b of the hi/lo panel buffers.
+// Batched Cholesky tile work on the split panel buffers (slot s = rows s*b of
+// the hi/lo buffers, K-major):
+//  mode 1 (SYRK/GEMM): task z updates tile (ti, tj): C -= P_i P_j^T, with P_i
+//          in slot slot0+ti, P_j in slot slot0+tj, K = b;
+//  mode 2 (TRSM block update): C = columns [n0, n0+ncols) of tile (ti, tj)
+//          -= X_i[:, kx0:kx0+K] L[n0:n0+ncols, kx0:kx0+K]^T, X_i in slot
+//          slot0+ti, L = tile (tj, tj) in slot slot0+tj.
 struct GemmJob {
-  int32_t mode;            // 0: rows of a plain SGEMM, 1: Cholesky tile batch
+  int32_t mode;            // 0: rows of a plain SGEMM, 1: tile update, 2: TRSM block update
   int32_t n;
   int64_t T, b;
+  int32_t slot0;           // first slot of this step's parity
+  int32_t kx0, n0, ncols;  // mode 2
   int32_t ti[kCholBatch], tj[kCholBatch];
 };
 
@@ -104,12 +111,18 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int m_blk = blockIdx.y, n_blk = blockIdx.x;
   // operand row coordinates in the tensor maps, and the output tile
-  int32_t ya = m_blk * BM, yb = n_blk * BN;
-  if (job.mode == 1) {
+  int32_t ya = m_blk * BM, yb = n_blk * BN, kx0 = 0, ncols = BN;
+  if (job.mode >= 1) {
     const int z = blockIdx.z;
-    ya += (int32_t)(job.ti[z] * job.b);
-    yb += (int32_t)(job.tj[z] * job.b);
+    ya += (int32_t)((job.slot0 + job.ti[z]) * job.b);
+    yb += (int32_t)((job.slot0 + job.tj[z]) * job.b);
     C += ((int64_t)job.ti[z] * job.T + job.tj[z]) * job.b * job.b;
+    if (job.mode == 2) {
+      C += job.n0;
+      yb += job.n0;
+      kx0 = job.kx0;
+      ncols = min(BN, job.ncols - n_blk * BN);
+    }
   }
 
   if (warp == 0 && lane == 0) {
@@ -140,10 +153,11 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
         if (kb >= kStages) mbar_wait(&empty[s], (uint32_t)(((kb / kStages) - 1) & 1));
         uint8_t* st = base + s * STAGE_BYTES;
         mbar_expect_tx(&full[s], STAGE_BYTES);
-        tma_load_2d(st, &tAhi, kb * BK, ya, &full[s]);
-        tma_load_2d(st + A_BYTES, &tAlo, kb * BK, ya, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES, &tBhi, kb * BK, yb, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kb * BK, yb, &full[s]);
+        const int32_t kx = kx0 + kb * BK;
+        tma_load_2d(st, &tAhi, kx, ya, &full[s]);
+        tma_load_2d(st + A_BYTES, &tAlo, kx, ya, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES, &tBhi, kx, yb, &full[s]);
+        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, yb, &full[s]);
       }
     }
     __syncwarp();
@@ -177,9 +191,9 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     const int g = warp & 3;
     const int64_t r = (int64_t)m_blk * BM + g * 32 + lane;  // row within [0, mrows)
     const bool row_ok = r < mrows;
-    float* crow = job.mode == 1 ? C + r * job.b : C + (row0 + r) * N;
+    float* crow = job.mode >= 1 ? C + r * job.b : C + (row0 + r) * N;
 #pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
+    for (int c = 0; c < ncols; c += 16) {
       uint32_t v[16];
       const uint32_t ta = tmem + ((uint32_t)(g * 32) << 16) + (uint32_t)c;
       asm volatile(
@@ -189,7 +203,7 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
           : "r"(ta));
       asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
       const int64_t n0 = (int64_t)n_blk * BN + c;
-      if (job.mode == 1) {   // C_tile -= acc (tile row r, ldc = b)
+      if (job.mode >= 1) {   // C_tile -= acc (tile row r, ldc = b)
         float4* p = reinterpret_cast<float4*>(crow + n0);
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
@@ -263,15 +277,15 @@ __global__ void split_transpose(const float* __restrict__ B, float* __restrict__
   }
 }
 
-// Split panel tiles: tile (list[t].i, k) of the tile-major matrix -> slot i of
-// the hi/lo panel buffers (b x b each, row-major = K-major rows).
+// Split panel tiles: tile (list[t].i, k) of the tile-major matrix -> slot
+// slot0 + i of the hi/lo panel buffers (b x b each, row-major = K-major rows).
 __global__ void split_tiles(const float* __restrict__ A, float* __restrict__ hi, float* __restrict__ lo,
                             int64_t T, int64_t b, const __grid_constant__ GemmJob list, int32_t k) {
   const int t = blockIdx.y;
   const int64_t i = list.ti[t];
   const float* src = A + (i * T + k) * b * b;
-  float* h = hi + i * b * b;
-  float* l = lo + i * b * b;
+  float* h = hi + (list.slot0 + i) * b * b;
+  float* l = lo + (list.slot0 + i) * b * b;
   const int64_t n = b * b / 4;
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
     const float4 x = reinterpret_cast<const float4*>(src)[e];
@@ -287,63 +301,148 @@ __global__ void split_tiles(const float* __restrict__ A, float* __restrict__ hi,
 
 }  // namespace
 
+// Split panel buffers: two step parities x T slots x (hi, lo) x b*b floats.
+// Step k uses slots [(k&1)*T, (k&1)*T + T): slot i holds tile (i,k)'s split
+// (written by the TRSM leaves, or by split_tiles when the tile came from
+// another device), slot k holds L_kk's; the TRSM of step k+1 (lane 1) thus
+// never overwrites what step k's updates (lane 0) still read.
 size_t chol_tc_scratch(int64_t T, int64_t b) {
-  return (b % BN == 0) ? (size_t)(2 * T * b * b) * sizeof(float) : 0;
+  return (b % 128 == 0) ? (size_t)(4 * T * b * b) * sizeof(float) : 0;
 }
+
+namespace {
+
+uint64_t split_tag(const Scratch* scr, int32_t k) { return (scr->epoch << 20) | (uint64_t)(k + 1); }
+
+cudaError_t set_gemm_smem() {
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  return cudaSuccess;
+}
+
+// Split the tiles (i, k) of `need` (slot not yet tagged for step k) into this
+// step's slots.
+cudaError_t split_needed(float* A, int64_t T, int64_t b, int32_t k, const int32_t* need, int32_t n_need,
+                         cudaStream_t s, Scratch* scr) {
+  float* hi = static_cast<float*>(scr->ptr);
+  float* lo = hi + 2 * T * b * b;
+  if (scr->panel.size() != (size_t)(2 * T)) scr->panel.assign(2 * T, 0);
+  const int32_t par = k & 1;
+  const uint64_t tag = split_tag(scr, k);
+  GemmJob sl;
+  sl.mode = 1;
+  sl.n = 0;
+  sl.T = T;
+  sl.b = b;
+  sl.slot0 = par * (int32_t)T;
+  for (int32_t q = 0; q < n_need; ++q) {
+    const int32_t i = need[q];
+    if (scr->panel[par * T + i] != tag && sl.n < kCholBatch) {
+      scr->panel[par * T + i] = tag;
+      sl.ti[sl.n++] = i;
+    }
+  }
+  if (sl.n) split_tiles<<<dim3((unsigned)std::min<int64_t>(b * b / 4 / 256, 64), (unsigned)sl.n), 256, 0, s>>>(
+      A, hi, lo, T, b, sl, k);
+  return cudaSuccess;
+}
+
+cudaError_t panel_maps(Scratch* scr, int64_t T, int64_t b, CUtensorMap* ta_hi, CUtensorMap* ta_lo,
+                       CUtensorMap* tb_hi, CUtensorMap* tb_lo) {
+  float* hi = static_cast<float*>(scr->ptr);
+  float* lo = hi + 2 * T * b * b;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(ta_hi, hi, b, 2 * T * b, b * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(ta_lo, lo, b, 2 * T * b, b * 4, BK, BM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(tb_hi, hi, b, 2 * T * b, b * 4, BK, BN)) != cudaSuccess) return e;
+  return encode_tmap_2d_f32(tb_lo, lo, b, 2 * T * b, b * 4, BK, BN);
+}
+
+}  // namespace
 
 // Batched C(i,j) -= A(i,k) A(j,k)^T with 3xTF32 tcgen05 (b % 256 == 0).
 cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, int32_t n, cudaStream_t s,
                            Scratch* scr) {
   if (n <= 0) return cudaSuccess;
   if (b % BN != 0 || !scr || !scr->ptr || scr->bytes < chol_tc_scratch(T, b)) return cudaErrorNotSupported;
-  float* hi = static_cast<float*>(scr->ptr);
-  float* lo = hi + T * b * b;
-  if (scr->panel.size() != (size_t)T) scr->panel.assign(T, 0);
   const int32_t k = ijk[2];
-  const uint64_t tag = (scr->epoch << 20) | (uint64_t)(k + 1);
   // 1. split the panel tiles this batch needs that are not split for step k yet
-  GemmJob sl;
-  sl.mode = 1;
-  sl.n = 0;
-  sl.T = T;
-  sl.b = b;
-  auto need = [&](int32_t i) {
-    if (scr->panel[i] != tag && sl.n < kCholBatch) {
-      scr->panel[i] = tag;
-      sl.ti[sl.n++] = i;
-    }
-  };
+  std::vector<int32_t> need;
   for (int32_t q = 0; q < n; ++q) {
     if (ijk[3 * q + 2] != k) return cudaErrorInvalidValue;  // one step per batch
-    need(ijk[3 * q]);
-    need(ijk[3 * q + 1]);
+    need.push_back(ijk[3 * q]);
+    need.push_back(ijk[3 * q + 1]);
   }
-  if (sl.n) split_tiles<<<dim3((unsigned)std::min<int64_t>(b * b / 4 / 256, 64), (unsigned)sl.n), 256, 0, s>>>(
-      A, hi, lo, T, b, sl, k);
+  cudaError_t e = split_needed(A, T, b, k, need.data(), (int32_t)need.size(), s, scr);
+  if (e != cudaSuccess) return e;
   // 2. one batched GEMM launch over all tasks
   CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
-  cudaError_t e;
-  if ((e = encode_tmap_2d_f32(&ta_hi, hi, b, T * b, b * 4, BK, BM)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&ta_lo, lo, b, T * b, b * 4, BK, BM)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&tb_hi, hi, b, T * b, b * 4, BK, BN)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&tb_lo, lo, b, T * b, b * 4, BK, BN)) != cudaSuccess) return e;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
-    attr = true;
-  }
+  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo)) != cudaSuccess) return e;
+  if ((e = set_gemm_smem()) != cudaSuccess) return e;
   for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
     GemmJob job;
     job.mode = 1;
     job.n = std::min<int32_t>(kCholBatch, n - q0);
     job.T = T;
     job.b = b;
+    job.slot0 = (k & 1) * (int32_t)T;
+    job.kx0 = job.n0 = 0;
+    job.ncols = (int32_t)b;
     for (int32_t q = 0; q < job.n; ++q) {
       job.ti[q] = ijk[3 * (q0 + q)];
       job.tj[q] = ijk[3 * (q0 + q) + 1];
     }
     dim3 grid((unsigned)(b / BN), (unsigned)(b / BM), (unsigned)job.n);
     gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job);
+  }
+  return cudaGetLastError();
+}
+
+// TRSM support: hi/lo slot pointers of step k, L_kk split into slot k.
+cudaError_t chol_trsm_prepare(float* A, int64_t T, int64_t b, int32_t k, cudaStream_t s, Scratch* scr,
+                              float** hi, float** lo, int32_t* slot0) {
+  if (!scr || !scr->ptr || scr->bytes < chol_tc_scratch(T, b)) return cudaErrorNotSupported;
+  *hi = static_cast<float*>(scr->ptr);
+  *lo = *hi + 2 * T * b * b;
+  *slot0 = (k & 1) * (int32_t)T;
+  return split_needed(A, T, b, k, &k, 1, s, scr);
+}
+
+// Mark panel slots of step k as split (the TRSM leaves wrote them).
+void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, int32_t n) {
+  if (scr->panel.size() != (size_t)(2 * T)) scr->panel.assign(2 * T, 0);
+  for (int32_t q = 0; q < n; ++q) scr->panel[(k & 1) * T + tiles[q]] = split_tag(scr, k);
+}
+
+// TRSM block update over a batch: columns [n0, b) of tiles (ti[q], k) -=
+// X_i[:, kx0:kx0+K] L_kk[n0:b, kx0:kx0+K]^T (3xTF32, split operands in slots).
+cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n,
+                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr) {
+  if (n <= 0 || n0 >= b) return cudaSuccess;
+  CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
+  cudaError_t e;
+  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo)) != cudaSuccess) return e;
+  if ((e = set_gemm_smem()) != cudaSuccess) return e;
+  for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
+    GemmJob job;
+    job.mode = 2;
+    job.n = std::min<int32_t>(kCholBatch, n - q0);
+    job.T = T;
+    job.b = b;
+    job.slot0 = (k & 1) * (int32_t)T;
+    job.kx0 = kx0;
+    job.n0 = n0;
+    job.ncols = (int32_t)(b - n0);
+    for (int32_t q = 0; q < job.n; ++q) {
+      job.ti[q] = ti[q0 + q];
+      job.tj[q] = k;
+    }
+    dim3 grid((unsigned)((b - n0 + BN - 1) / BN), (unsigned)(b / BM), (unsigned)job.n);
+    gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job);
   }
   return cudaGetLastError();
 }
@@ -389,16 +488,14 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   if ((e = encode_tmap_2d_f32(&ta_lo, alo, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
-    attr = true;
-  }
+  if ((e = set_gemm_smem()) != cudaSuccess) return e;
   dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((mrows + BM - 1) / BM));
   GemmJob job;
   job.mode = 0;
   job.n = 0;
   job.T = job.b = 0;
+  job.slot0 = job.kx0 = job.n0 = 0;
+  job.ncols = BN;
   gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows,
                                                      (int)(Kp / BK), job);
   return cudaGetLastError();

@@ -10,6 +10,8 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <memory>
@@ -229,11 +231,12 @@ bool is_batchable_op(int32_t op) {
 // A member joins only if no other op of that device lies between, all of its
 // cross-stream waits point before the head, and it neither reads nor writes
 // what an earlier member writes (nor writes what an earlier member reads).
-// Batch key: tasks of one batch must share it.  Cholesky lookahead: GEMM
-// updates are batched per output column j and SYRK(k+1, k) runs alone, so
-// step k+1's POTRF / TRSM (lane 1) wait only for the updates they read.
+// Batch key: tasks of one batch must share it.  Cholesky lookahead: the GEMM
+// updates of column k+1 and SYRK(k+1, k) run as their own launches, so step
+// k+1's POTRF / TRSM (lane 1) wait only for the updates they read; the rest
+// of step k's GEMMs is one launch (no per-column waves of partial occupancy).
 int64_t batch_key(const Kernel& k, const Task& t) {
-  if (k.op == MM_OP_CHOL_GEMM) return t.ip[2] * 1000003 + t.ip[1];
+  if (k.op == MM_OP_CHOL_GEMM) return t.ip[2] * 2 + (t.ip[1] == t.ip[2] + 1 ? 1 : 0);
   if (k.op == MM_OP_CHOL_SYRK) return t.ip[2] * 2 + (t.ip[0] == t.ip[2] + 1 ? 1 : 0);
   return t.ip[2];
 }
@@ -347,7 +350,8 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
 size_t builtin_scratch_bytes(const Kernel& k, const Task& t) {
   if (k.op == MM_OP_SGEMM && (k.ip[3] == 0 || k.ip[3] == 2))
     return sgemm_tf32x3_scratch(k.ip[1], k.ip[2], t.e - t.b);
-  if (k.op == MM_OP_CHOL_SYRK || k.op == MM_OP_CHOL_GEMM) return chol_tc_scratch(k.ip[0], k.ip[1]);
+  if (k.op == MM_OP_CHOL_POTRF || k.op == MM_OP_CHOL_TRSM || k.op == MM_OP_CHOL_SYRK || k.op == MM_OP_CHOL_GEMM)
+    return chol_scratch_bytes(k.ip[0], k.ip[1]);
   return 0;
 }
 
@@ -1346,9 +1350,23 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   float ms = 0.f;
   CU_OK(cudaEventElapsedTime(&ms, rt->t_start, rt->t_stop));
   S->device_ms = ms;
+  // MM_TRACE=<file>: per kernel launch (batch heads) of a timed run, append
+  // "kernel,ip0,ip1,ip2,device,tasks,start_ms,end_ms" relative to the run start
+  static const char* trace_path = getenv("MM_TRACE");
+  FILE* trace = (timing && trace_path) ? fopen(trace_path, "a") : nullptr;
   for (size_t i = 0; i < plan.ops.size(); ++i) {
     const mm_op_rec& op = plan.ops[i];
     if (op.kind != MM_OPK_KERNEL || !ctx->dev[op.device].mine) continue;
+    if (trace && rt->kev[2 * i] && rt->batch_head[i] < 0) {
+      float a = 0.f, z = 0.f;
+      if (cudaEventElapsedTime(&a, rt->t_start, rt->kev[2 * i]) == cudaSuccess &&
+          cudaEventElapsedTime(&z, rt->t_start, rt->kev[2 * i + 1]) == cudaSuccess) {
+        const Task& t = plan.tasks[op.task];
+        fprintf(trace, "%s,%lld,%lld,%lld,%d,%zu,%.4f,%.4f\n", plan.app.kernels[op.kernel].name.c_str(),
+                (long long)t.ip[0], (long long)t.ip[1], (long long)t.ip[2], op.device, rt->members[i].size() + 1,
+                a, z);
+      }
+    }
     S->kernel_launches[op.device][op.kernel]++;
     if (timing && rt->kev[2 * i] && rt->batch_head[i] < 0) {   // batch members: timed with their head
       float k = 0.f;
@@ -1356,6 +1374,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       S->kernel_ms[op.device][op.kernel] += k;
     }
   }
+  if (trace) fclose(trace);
   return MM_OK;
 }
 
