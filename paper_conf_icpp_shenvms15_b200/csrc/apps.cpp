@@ -163,7 +163,6 @@ mm_status sgemm_app(const mm_app_params& p, mm_app* app) {
 mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
   const int64_t n = p.iparam[0], b = p.iparam[1] > 0 ? p.iparam[1] : 1024;
   if (n <= 0 || n % b) MM_FAIL(MM_EINVAL, "cholesky: n must be a multiple of the tile");
-  if (b % 128 || b > 2048) MM_FAIL(MM_EINVAL, "cholesky: tile must be a multiple of 128, at most 2048");
   const int64_t T = n / b, bb = b * b;
   int32_t A;
   mm_app_add_buffer(app, 4, n * n, &A);   // tile-major: tile (i,j) at (i*T+j)*b*b
