@@ -11,12 +11,16 @@
 //  1. split: A rows [r0,r1) -> A_hi, A_lo (row-major, K padded to 32);
 //     B (K x N) -> B_hi^T, B_lo^T (N x K, "K-major") through a 32x32 smem
 //     transpose.  HBM-bound elementwise passes into library scratch.
-//  2. gemm: 128 x 256 output tile per CTA; warp 0 = TMA producer (four 2-D
-//     tensor maps, SWIZZLE_128B boxes of 32 fp32 along K), warp 1 = TMEM
-//     allocator + single-thread tcgen05.mma issuer (kind::tf32, M=128 N=256
-//     K=8, 3 MMAs per K step), warps 2-5 = epilogue (tcgen05.ld 32x32b ->
-//     registers -> global).  mbarrier ring of kStages stages between TMA and
-//     MMA; tcgen05.commit frees a stage and signals the epilogue.
+//  2. gemm: 128 x 256 output tiles, each CTA walks a run of tiles
+//     (persistent): warp 0 = TMA producer (four 2-D tensor maps, SWIZZLE_64B
+//     boxes of 16 fp32 along K) into a kStages-deep mbarrier ring, warp 1 =
+//     TMEM allocator + single-thread tcgen05.mma issuer (kind::tf32, M=128
+//     N=256 K=8, 3 MMAs per K step) into one of two 256-column TMEM
+//     accumulators, warps 2-5 = epilogue (tcgen05.ld 32x32b -> registers ->
+//     global) of the other accumulator, so tile t's epilogue overlaps tile
+//     t+1's main loop.  tcgen05.commit frees ring stages and hands finished
+//     accumulators to the epilogue; the epilogue hands them back through an
+//     mbarrier.
 #include <cuda.h>
 
 #include <algorithm>
@@ -31,26 +35,29 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
 
 namespace {
 
-constexpr int BM = 128, BN = 256, BK = 32, kStages = 2;
-constexpr int A_BYTES = BM * BK * 4;                 // 16 KB
-constexpr int B_BYTES = BN * BK * 4;                 // 32 KB
+constexpr int BM = 128, BN = 256, BK = 16, kStages = 4, KPAD = 32;
+constexpr int A_BYTES = BM * BK * 4;                 // 8 KB
+constexpr int B_BYTES = BN * BK * 4;                 // 16 KB
 constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
 constexpr int SMEM_BYTES = kStages * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 constexpr int kThreadsGemm = 192;
+constexpr int kAccCols = 2 * BN;                     // two TMEM accumulators
 
-// Batched Cholesky tile work on the split panel buffers (slot s = rows s*b of
-// the hi/lo buffers, K-major):
+// Tile work of one launch:
+//  mode 0 (SGEMM rows): C[row0 + r][n] = (A B)[r][n], r < mrows, n < N;
 //  mode 1 (SYRK/GEMM): task z updates tile (ti, tj): C -= P_i P_j^T, with P_i
-//          in slot slot0+ti, P_j in slot slot0+tj, K = b;
+//          in panel slot slot0+ti, P_j in slot slot0+tj, K = b;
 //  mode 2 (TRSM block update): C = columns [n0, n0+ncols) of tile (ti, tj)
 //          -= X_i[:, kx0:kx0+K] L[n0:n0+ncols, kx0:kx0+K]^T, X_i in slot
 //          slot0+ti, L = tile (tj, tj) in slot slot0+tj.
+// (slot s = rows s*b of the hi/lo panel buffers, K-major.)
 struct GemmJob {
   int32_t mode;            // 0: rows of a plain SGEMM, 1: tile update, 2: TRSM block update
-  int32_t n;
+  int32_t n;               // tasks (modes 1, 2)
   int64_t T, b;
   int32_t slot0;           // first slot of this step's parity
   int32_t kx0, n0, ncols;  // mode 2
+  int32_t mblk, nblk;      // output tiles per task
   int32_t ti[kCholBatch], tj[kCholBatch];
 };
 
@@ -61,6 +68,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t c) {
 }
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(saddr(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(saddr(b)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
   asm volatile(
@@ -76,14 +86,15 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, i
       "l"((uint64_t)map), "r"(x), "r"(y), "r"(saddr(bar))
       : "memory");
 }
-// UMMA shared-memory descriptor: K-major, SWIZZLE_128B, 8-row groups 1024 B apart.
+// UMMA shared-memory descriptor: K-major, SWIZZLE_64B (rows of 64 B, 8-row
+// core-matrix groups 512 B apart).
 __device__ __forceinline__ uint64_t sdesc(const void* p) {
   const uint64_t a = saddr(p);
   uint64_t d = (a >> 4) & 0x3FFFull;         // start address
-  d |= 1ull << 16;                           // leading byte offset (unused for SW128 K-major)
-  d |= (uint64_t)(1024 >> 4) << 32;          // stride byte offset
+  d |= 1ull << 16;                           // leading byte offset (unused for swizzled K-major)
+  d |= (uint64_t)(512 >> 4) << 32;           // stride byte offset
   d |= 1ull << 46;                           // descriptor version (sm_100)
-  d |= 2ull << 61;                           // SWIZZLE_128B
+  d |= 4ull << 61;                           // SWIZZLE_64B
   return d;
 }
 __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
@@ -97,40 +108,60 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
                : "memory");
 }
 
+// Operand coordinates and output of tile `tile` (task-major, n fastest).
+struct TileGeo {
+  int32_t ya, yb, kx0, m_blk, n_blk, ncols;
+  float* C;
+};
+__device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile) {
+  TileGeo g;
+  const int per = job.mblk * job.nblk;
+  const int z = tile / per, rem = tile % per;
+  g.m_blk = rem / job.nblk;
+  g.n_blk = rem % job.nblk;
+  g.ya = g.m_blk * BM;
+  g.yb = g.n_blk * BN;
+  g.kx0 = 0;
+  g.ncols = BN;
+  g.C = C;
+  if (job.mode >= 1) {
+    g.ya += (int32_t)((job.slot0 + job.ti[z]) * job.b);
+    g.yb += (int32_t)((job.slot0 + job.tj[z]) * job.b);
+    g.C += ((int64_t)job.ti[z] * job.T + job.tj[z]) * job.b * job.b;
+    if (job.mode == 2) {
+      g.C += job.n0;
+      g.yb += job.n0;
+      g.kx0 = job.kx0;
+      g.ncols = min(BN, job.ncols - g.n_blk * BN);
+    }
+  }
+  return g;
+}
+
+// Tiles [tile0, tile1) of the job, stepping by `stride` from blockIdx.x.
 __global__ void __launch_bounds__(kThreadsGemm, 1)
     gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
                 const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
-                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb,
+                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb, int ntiles,
                 const __grid_constant__ GemmJob job) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full = reinterpret_cast<uint64_t*>(base + kStages * STAGE_BYTES);
   uint64_t* empty = full + kStages;
-  uint64_t* tfull = empty + kStages;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+  uint64_t* tfull = empty + kStages;       // [2] accumulator ready for the epilogue
+  uint64_t* tempty = tfull + 2;            // [2] accumulator drained by the epilogue
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m_blk = blockIdx.y, n_blk = blockIdx.x;
-  // operand row coordinates in the tensor maps, and the output tile
-  int32_t ya = m_blk * BM, yb = n_blk * BN, kx0 = 0, ncols = BN;
-  if (job.mode >= 1) {
-    const int z = blockIdx.z;
-    ya += (int32_t)((job.slot0 + job.ti[z]) * job.b);
-    yb += (int32_t)((job.slot0 + job.tj[z]) * job.b);
-    C += ((int64_t)job.ti[z] * job.T + job.tj[z]) * job.b * job.b;
-    if (job.mode == 2) {
-      C += job.n0;
-      yb += job.n0;
-      kx0 = job.kx0;
-      ncols = min(BN, job.ncols - n_blk * BN);
-    }
-  }
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < kStages; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
-    mbar_init(tfull, 1);
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], 4);            // one arrival per epilogue warp
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tAhi) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tAlo) : "memory");
@@ -138,7 +169,8 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBlo) : "memory");
   }
   if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)), "n"(BN));
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)),
+                 "n"(kAccCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -148,16 +180,20 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
 
   if (warp == 0) {
     if (lane == 0) {  // ===== TMA producer
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % kStages;
-        if (kb >= kStages) mbar_wait(&empty[s], (uint32_t)(((kb / kStages) - 1) & 1));
-        uint8_t* st = base + s * STAGE_BYTES;
-        mbar_expect_tx(&full[s], STAGE_BYTES);
-        const int32_t kx = kx0 + kb * BK;
-        tma_load_2d(st, &tAhi, kx, ya, &full[s]);
-        tma_load_2d(st + A_BYTES, &tAlo, kx, ya, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES, &tBhi, kx, yb, &full[s]);
-        tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, yb, &full[s]);
+      int it = 0;
+      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const TileGeo g = tile_geo(job, C, tile);
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % kStages;
+          if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1));
+          uint8_t* st = base + s * STAGE_BYTES;
+          mbar_expect_tx(&full[s], STAGE_BYTES);
+          const int32_t kx = g.kx0 + kb * BK;
+          tma_load_2d(st, &tAhi, kx, g.ya, &full[s]);
+          tma_load_2d(st + A_BYTES, &tAlo, kx, g.ya, &full[s]);
+          tma_load_2d(st + 2 * A_BYTES, &tBhi, kx, g.yb, &full[s]);
+          tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, g.yb, &full[s]);
+        }
       }
     }
     __syncwarp();
@@ -166,74 +202,89 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
       const uint32_t idesc = (1u << 4)                 // D: fp32
                              | (2u << 7) | (2u << 10)  // A, B: tf32
                              | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % kStages;
-        mbar_wait(&full[s], (uint32_t)((kb / kStages) & 1));
+      int it = 0, lt = 0;
+      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++lt) {
+        const int ab = lt & 1;
+        if (lt >= 2) mbar_wait(&tempty[ab], (uint32_t)(((lt >> 1) - 1) & 1));
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        uint8_t* st = base + s * STAGE_BYTES;
-        const uint64_t ahi = sdesc(st), alo = sdesc(st + A_BYTES);
-        const uint64_t bhi = sdesc(st + 2 * A_BYTES), blo = sdesc(st + 2 * A_BYTES + B_BYTES);
+        const uint32_t acc_t = tmem + (uint32_t)(ab * BN);
+        for (int kb = 0; kb < nkb; ++kb, ++it) {
+          const int s = it % kStages;
+          mbar_wait(&full[s], (uint32_t)((it / kStages) & 1));
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          uint8_t* st = base + s * STAGE_BYTES;
+          const uint64_t ahi = sdesc(st), alo = sdesc(st + A_BYTES);
+          const uint64_t bhi = sdesc(st + 2 * A_BYTES), blo = sdesc(st + 2 * A_BYTES + B_BYTES);
 #pragma unroll
-        for (int kk = 0; kk < BK / 8; ++kk) {
-          const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 fp32 = 32 B along K inside the swizzle atom
-          mma_tf32(tmem, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
-          mma_tf32(tmem, ahi + adv, blo + adv, idesc, 1u);
-          mma_tf32(tmem, ahi + adv, bhi + adv, idesc, 1u);
+          for (int kk = 0; kk < BK / 8; ++kk) {
+            const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 fp32 = 32 B along K inside the swizzle atom
+            mma_tf32(acc_t, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
+            mma_tf32(acc_t, ahi + adv, blo + adv, idesc, 1u);
+            mma_tf32(acc_t, ahi + adv, bhi + adv, idesc, 1u);
+          }
+          mma_commit(&empty[s]);
         }
-        mma_commit(&empty[s]);
+        mma_commit(&tfull[ab]);
       }
-      mma_commit(tfull);
     }
     __syncwarp();
   } else {  // ===== epilogue: warps 2..5 -> TMEM lane groups (warp % 4)
-    mbar_wait(tfull, 0);
-    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    const int g = warp & 3;
-    const int64_t r = (int64_t)m_blk * BM + g * 32 + lane;  // row within [0, mrows)
-    const bool row_ok = r < mrows;
-    float* crow = job.mode >= 1 ? C + r * job.b : C + (row0 + r) * N;
+    const int grp = warp & 3;
+    int lt = 0;
+    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++lt) {
+      const int ab = lt & 1;
+      const TileGeo g = tile_geo(job, C, tile);
+      mbar_wait(&tfull[ab], (uint32_t)((lt >> 1) & 1));
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const int64_t r = (int64_t)g.m_blk * BM + grp * 32 + lane;  // output row
+      const bool row_ok = job.mode >= 1 || r < mrows;
+      float* crow = job.mode >= 1 ? g.C + r * job.b : g.C + (row0 + r) * N;
 #pragma unroll 1
-    for (int c = 0; c < ncols; c += 16) {
-      uint32_t v[16];
-      const uint32_t ta = tmem + ((uint32_t)(g * 32) << 16) + (uint32_t)c;
-      asm volatile(
-          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-          : "r"(ta));
-      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-      const int64_t n0 = (int64_t)n_blk * BN + c;
-      if (job.mode >= 1) {   // C_tile -= acc (tile row r, ldc = b)
-        float4* p = reinterpret_cast<float4*>(crow + n0);
+      for (int c = 0; c < g.ncols; c += 16) {
+        uint32_t v[16];
+        const uint32_t ta = tmem + (uint32_t)(ab * BN) + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+              "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+            : "r"(ta));
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        const int64_t n0 = (int64_t)g.n_blk * BN + c;
+        if (job.mode >= 1) {   // C_tile -= acc (tile row r, ldc = b)
+          float4* p = reinterpret_cast<float4*>(crow + n0);
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          float4 o = p[q];
-          o.x -= __uint_as_float(v[4 * q]);
-          o.y -= __uint_as_float(v[4 * q + 1]);
-          o.z -= __uint_as_float(v[4 * q + 2]);
-          o.w -= __uint_as_float(v[4 * q + 3]);
-          p[q] = o;
-        }
-      } else if (row_ok) {
-        if (n0 + 16 <= N && (N & 3) == 0) {
+          for (int q = 0; q < 4; ++q) {
+            float4 o = p[q];
+            o.x -= __uint_as_float(v[4 * q]);
+            o.y -= __uint_as_float(v[4 * q + 1]);
+            o.z -= __uint_as_float(v[4 * q + 2]);
+            o.w -= __uint_as_float(v[4 * q + 3]);
+            p[q] = o;
+          }
+        } else if (row_ok) {
+          if (n0 + 16 <= N && (N & 3) == 0) {
 #pragma unroll
-          for (int q = 0; q < 4; ++q)
-            *reinterpret_cast<float4*>(crow + n0 + 4 * q) =
-                make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
-                            __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
-        } else {
+            for (int q = 0; q < 4; ++q)
+              *reinterpret_cast<float4*>(crow + n0 + 4 * q) =
+                  make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
+                              __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
+          } else {
 #pragma unroll
-          for (int q = 0; q < 16; ++q)
-            if (n0 + q < N) crow[n0 + q] = __uint_as_float(v[q]);
+            for (int q = 0; q < 16; ++q)
+              if (n0 + q < N) crow[n0 + q] = __uint_as_float(v[q]);
+          }
         }
       }
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[ab]);
     }
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   if (warp == 1) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(BN));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kAccCols));
   }
 }
 
@@ -324,6 +375,22 @@ cudaError_t set_gemm_smem() {
   return cudaSuccess;
 }
 
+// Launch the persistent GEMM over ntiles tiles: at most `cap` CTAs when set
+// (mode 0: one run of tiles per SM), else runs of up to 4 tiles per CTA so
+// CTAs retire regularly and other streams' kernels get SMs (MK-DAG lookahead).
+cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, const CUtensorMap& tb_hi,
+                        const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
+                        const GemmJob& job, int cap, cudaStream_t s) {
+  const int ntiles = job.mblk * job.nblk * (job.mode >= 1 ? job.n : 1);
+  if (ntiles <= 0) return cudaSuccess;
+  int grid;
+  if (cap > 0) grid = std::min(ntiles, cap);
+  else grid = std::max(std::min(ntiles, 148), (ntiles + 3) / 4);
+  gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0, mrows, nkb, ntiles,
+                                                     job);
+  return cudaSuccess;
+}
+
 // Split the tiles (i, k) of `need` (slot not yet tagged for step k) into this
 // step's slots.
 cudaError_t split_needed(float* A, int64_t T, int64_t b, int32_t k, const int32_t* need, int32_t n_need,
@@ -396,8 +463,9 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
       job.ti[q] = ijk[3 * (q0 + q)];
       job.tj[q] = ijk[3 * (q0 + q) + 1];
     }
-    dim3 grid((unsigned)(b / BN), (unsigned)(b / BM), (unsigned)job.n);
-    gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job);
+    job.mblk = (int32_t)(b / BM);
+    job.nblk = (int32_t)(b / BN);
+    launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job, 0, s);
   }
   return cudaGetLastError();
 }
@@ -441,25 +509,25 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
       job.ti[q] = ti[q0 + q];
       job.tj[q] = k;
     }
-    dim3 grid((unsigned)((b - n0 + BN - 1) / BN), (unsigned)(b / BM), (unsigned)job.n);
-    gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job);
+    job.mblk = (int32_t)(b / BM);
+    job.nblk = (int32_t)((b - n0 + BN - 1) / BN);
+    launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job, 0, s);
   }
   return cudaGetLastError();
 }
 
 size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
-  const int64_t Kp = (K + BK - 1) / BK * BK;
+  const int64_t Kp = (K + KPAD - 1) / KPAD * KPAD;
   return (size_t)(2 * mrows * Kp + 2 * N * Kp) * sizeof(float);
 }
 
 cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
                               int64_t r0, int64_t r1, cudaStream_t s, int sms, Scratch* scr, bool b_readonly) {
   (void)M;
-  (void)sms;
   const int64_t mrows = r1 - r0;
   if (mrows <= 0 || N <= 0) return cudaSuccess;
   if (!scr || !scr->ptr || scr->bytes < sgemm_tf32x3_scratch(N, K, mrows)) return cudaErrorNotSupported;
-  const int64_t Kp = (K + BK - 1) / BK * BK;
+  const int64_t Kp = (K + KPAD - 1) / KPAD * KPAD;
   // scratch layout: [B_hi^T | B_lo^T] (N x Kp each) then [A_hi | A_lo] (mrows x Kp each)
   float* bhi = static_cast<float*>(scr->ptr);
   float* blo = bhi + N * Kp;
@@ -489,15 +557,15 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
-  dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((mrows + BM - 1) / BM));
   GemmJob job;
   job.mode = 0;
-  job.n = 0;
+  job.n = 1;
   job.T = job.b = 0;
   job.slot0 = job.kx0 = job.n0 = 0;
   job.ncols = BN;
-  gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows,
-                                                     (int)(Kp / BK), job);
+  job.mblk = (int32_t)((mrows + BM - 1) / BM);
+  job.nblk = (int32_t)((N + BN - 1) / BN);
+  launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, sms > 0 ? sms : 148, s);
   return cudaGetLastError();
 }
 

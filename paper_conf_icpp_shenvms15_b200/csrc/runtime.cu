@@ -332,7 +332,8 @@ inline cudaStream_t sid_stream(const mm_ctx* ctx, int32_t sid) {
 
 namespace mm {
 
-// 2-D fp32 tensor map with a SWIZZLE_128B box (box_inner * 4 must be <= 128 B).
+// 2-D fp32 tensor map; the swizzle span equals the box row (box_inner * 4 =
+// 128, 64 or 32 bytes -> SWIZZLE_128B / 64B / 32B).
 cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
                                uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer) {
   Drv& D = drv();
@@ -342,7 +343,10 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
   const cuuint32_t box[2] = {box_inner, box_outer};
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = D.TensorMapEncodeTiled(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides,
-                                      box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                                      box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                      box_inner * 4 == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                      : box_inner * 4 == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                            : CU_TENSOR_MAP_SWIZZLE_32B,
                                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
