@@ -35,13 +35,14 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
 
 namespace {
 
+// BN = 256 (the default tile), or 64 for plain SGEMMs too small to give
+// every SM a 128 x 256 tile (BASELINE configs[0], 1024^2: 32 -> 128 tiles).
 constexpr int BM = 128, BN = 256, BK = 16, kStages = 4, KPAD = 32;
 constexpr int A_BYTES = BM * BK * 4;                 // 8 KB
-constexpr int B_BYTES = BN * BK * 4;                 // 16 KB
-constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
-constexpr int SMEM_BYTES = kStages * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+template <int BN_> constexpr int b_bytes() { return BN_ * BK * 4; }
+template <int BN_> constexpr int stage_bytes() { return 2 * A_BYTES + 2 * b_bytes<BN_>(); }
+template <int BN_> constexpr int smem_bytes() { return kStages * stage_bytes<BN_>() + 1024 /*align*/ + 256 /*barriers*/; }
 constexpr int kThreadsGemm = 192;
-constexpr int kAccCols = 2 * BN;                     // two TMEM accumulators
 
 // Tile work of one launch:
 //  mode 0 (SGEMM rows): C[row0 + r][n] = (A B)[r][n], r < mrows, n < N;
@@ -113,6 +114,7 @@ struct TileGeo {
   int32_t ya, yb, kx0, m_blk, n_blk, ncols;
   float* C;
 };
+template <int BN>
 __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile) {
   TileGeo g;
   const int per = job.mblk * job.nblk;
@@ -138,12 +140,14 @@ __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int ti
   return g;
 }
 
-// Tiles [tile0, tile1) of the job, stepping by `stride` from blockIdx.x.
+// Tiles blockIdx.x, blockIdx.x + gridDim.x, ... of the job.
+template <int BN>
 __global__ void __launch_bounds__(kThreadsGemm, 1)
     gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
                 const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
                 float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb, int ntiles,
                 const __grid_constant__ GemmJob job) {
+  constexpr int B_BYTES = b_bytes<BN>(), STAGE_BYTES = stage_bytes<BN>(), kAccCols = 2 * BN;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full = reinterpret_cast<uint64_t*>(base + kStages * STAGE_BYTES);
@@ -182,7 +186,7 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     if (lane == 0) {  // ===== TMA producer
       int it = 0;
       for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const TileGeo g = tile_geo(job, C, tile);
+        const TileGeo g = tile_geo<BN>(job, C, tile);
         for (int kb = 0; kb < nkb; ++kb, ++it) {
           const int s = it % kStages;
           if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1));
@@ -233,7 +237,7 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     int lt = 0;
     for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++lt) {
       const int ab = lt & 1;
-      const TileGeo g = tile_geo(job, C, tile);
+      const TileGeo g = tile_geo<BN>(job, C, tile);
       mbar_wait(&tfull[ab], (uint32_t)((lt >> 1) & 1));
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const int64_t r = (int64_t)g.m_blk * BM + grp * 32 + lane;  // output row
@@ -368,7 +372,9 @@ uint64_t split_tag(const Scratch* scr, int32_t k) { return (scr->epoch << 20) | 
 cudaError_t set_gemm_smem() {
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(gemm_tf32x3, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    cudaError_t e = cudaFuncSetAttribute(gemm_tf32x3<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes<256>());
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(gemm_tf32x3<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes<64>());
     if (e != cudaSuccess) return e;
     attr = true;
   }
@@ -378,6 +384,7 @@ cudaError_t set_gemm_smem() {
 // Launch the persistent GEMM over ntiles tiles: at most `cap` CTAs when set
 // (mode 0: one run of tiles per SM), else runs of up to 4 tiles per CTA so
 // CTAs retire regularly and other streams' kernels get SMs (MK-DAG lookahead).
+template <int BN_>
 cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, const CUtensorMap& tb_hi,
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
                         const GemmJob& job, int cap, cudaStream_t s) {
@@ -386,8 +393,8 @@ cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, cons
   int grid;
   if (cap > 0) grid = std::min(ntiles, cap);
   else grid = std::max(std::min(ntiles, 148), (ntiles + 3) / 4);
-  gemm_tf32x3<<<grid, kThreadsGemm, SMEM_BYTES, s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0, mrows, nkb, ntiles,
-                                                     job);
+  gemm_tf32x3<BN_><<<grid, kThreadsGemm, smem_bytes<BN_>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0, mrows,
+                                                                 nkb, ntiles, job);
   return cudaSuccess;
 }
 
@@ -465,7 +472,7 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
     }
     job.mblk = (int32_t)(b / BM);
     job.nblk = (int32_t)(b / BN);
-    launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job, 0, s);
+    launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job, 0, s);
   }
   return cudaGetLastError();
 }
@@ -511,7 +518,7 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
     }
     job.mblk = (int32_t)(b / BM);
     job.nblk = (int32_t)((b - n0 + BN - 1) / BN);
-    launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job, 0, s);
+    launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job, 0, s);
   }
   return cudaGetLastError();
 }
@@ -554,8 +561,11 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   cudaError_t e;
   if ((e = encode_tmap_2d_f32(&ta_hi, ahi, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&ta_lo, alo, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, BN)) != cudaSuccess) return e;
+  const int cap = sms > 0 ? sms : 148;
+  const bool narrow = ((mrows + BM - 1) / BM) * ((N + BN - 1) / BN) < cap;   // fewer 128x256 tiles than SMs
+  const uint32_t bn = narrow ? 64 : BN;
+  if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, bn)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, bn)) != cudaSuccess) return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
   GemmJob job;
   job.mode = 0;
@@ -564,8 +574,9 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   job.slot0 = job.kx0 = job.n0 = 0;
   job.ncols = BN;
   job.mblk = (int32_t)((mrows + BM - 1) / BM);
-  job.nblk = (int32_t)((N + BN - 1) / BN);
-  launch_gemm(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, sms > 0 ? sms : 148, s);
+  job.nblk = (int32_t)((N + bn - 1) / bn);
+  if (narrow) return launch_gemm<64>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s);
+  return launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s);
   return cudaGetLastError();
 }
 
