@@ -24,6 +24,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <vector>
 
 #include "kernels.h"
@@ -39,9 +40,6 @@ namespace {
 // every SM a 128 x 256 tile (BASELINE configs[0], 1024^2: 32 -> 128 tiles).
 constexpr int BM = 128, BN = 256, BK = 16, kStages = 4, KPAD = 32;
 constexpr int A_BYTES = BM * BK * 4;                 // 8 KB
-template <int BN_> constexpr int b_bytes() { return BN_ * BK * 4; }
-template <int BN_> constexpr int stage_bytes() { return 2 * A_BYTES + 2 * b_bytes<BN_>(); }
-template <int BN_> constexpr int smem_bytes() { return kStages * stage_bytes<BN_>() + 1024 /*align*/ + 256 /*barriers*/; }
 constexpr int kThreadsGemm = 192;
 
 // Tile work of one launch:
@@ -114,12 +112,15 @@ struct TileGeo {
   int32_t ya, yb, kx0, m_blk, n_blk, ncols;
   float* C;
 };
-template <int BN>
-__device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile) {
+// PAIR (2-CTA cluster) mode: `tile` enumerates tile pairs (m-blocks 2p, 2p+1
+// with one n-block), the CTA of cluster rank `rank` takes m-block 2p + rank.
+template <int BN, bool MC>
+__device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile, int rank) {
   TileGeo g;
-  const int per = job.mblk * job.nblk;
+  const int mb = MC ? job.mblk / 2 : job.mblk;
+  const int per = mb * job.nblk;
   const int z = tile / per, rem = tile % per;
-  g.m_blk = rem / job.nblk;
+  g.m_blk = MC ? 2 * (rem / job.nblk) + rank : rem / job.nblk;
   g.n_blk = rem % job.nblk;
   g.ya = g.m_blk * BM;
   g.yb = g.n_blk * BN;
@@ -140,31 +141,79 @@ __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int ti
   return g;
 }
 
-// Tiles blockIdx.x, blockIdx.x + gridDim.x, ... of the job.
-template <int BN>
-__global__ void __launch_bounds__(kThreadsGemm, 1)
-    gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
-                const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
-                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb, int ntiles,
-                const __grid_constant__ GemmJob job) {
-  constexpr int B_BYTES = b_bytes<BN>(), STAGE_BYTES = stage_bytes<BN>(), kAccCols = 2 * BN;
+__device__ __forceinline__ uint32_t peer_addr(const void* p, uint32_t rank) {   // shared::cluster address in CTA `rank`
+  uint32_t a;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(saddr(p)), "r"(rank));
+  return a;
+}
+// Pair-mode TMA: data into this CTA's smem, completion bytes on the leader's barrier.
+__device__ __forceinline__ void tma_load_2d_pair(void* dst, const CUtensorMap* map, int32_t x, int32_t y,
+                                                 uint32_t bar_cluster) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3}], [%4];" ::"r"(saddr(dst)),
+      "l"((uint64_t)map), "r"(x), "r"(y), "r"(bar_cluster)
+      : "memory");
+}
+__device__ __forceinline__ void mma_tf32_pair(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_commit_pair(uint64_t* bar) {   // arrive on `bar` in both CTAs
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          saddr(bar)),
+      "h"((uint16_t)0x3)
+      : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <int BN, bool PAIR> constexpr int gemm_stages() { return PAIR ? 6 : kStages; }
+template <int BN, bool PAIR> constexpr int gemm_stage_bytes() {
+  return 2 * A_BYTES + 2 * (PAIR ? BN / 2 : BN) * BK * 4;
+}
+template <int BN, bool PAIR> constexpr int gemm_smem() {
+  return gemm_stages<BN, PAIR>() * gemm_stage_bytes<BN, PAIR>() + 1024 /*align*/ + 256 /*barriers*/;
+}
+
+// Work units blockIdx.x, blockIdx.x + gridDim.x, ... of the job.  PAIR:
+// units are tile pairs (m-blocks 2p, 2p+1, one n-block) run by a cluster of 2
+// CTAs as ONE M=256 x N=256 tcgen05 MMA (cta_group::2): each CTA stages its
+// own 128 rows of A and one half (128 rows) of the B tile, the leader CTA
+// issues the MMAs, each CTA's TMEM receives its 128 output rows.  Per SM the
+// operand traffic is 2/3 of the single-CTA tile (A + half of B).
+template <int BN, bool PAIR>
+__device__ __forceinline__ void gemm_body(const CUtensorMap& tAhi, const CUtensorMap& tAlo, const CUtensorMap& tBhi,
+                                          const CUtensorMap& tBlo, float* __restrict__ C, int64_t N, int64_t row0,
+                                          int64_t mrows, int nkb, int ntiles, const GemmJob& job) {
+  constexpr int S = gemm_stages<BN, PAIR>(), STAGE_BYTES = gemm_stage_bytes<BN, PAIR>();
+  constexpr int B_BYTES = (PAIR ? BN / 2 : BN) * BK * 4, kAccCols = 2 * BN;
+  uint32_t rank = 0;
+  if (PAIR) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const bool leader = rank == 0;
+  const int unit0 = PAIR ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ustride = PAIR ? (int)(gridDim.x >> 1) : (int)gridDim.x;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full = reinterpret_cast<uint64_t*>(base + kStages * STAGE_BYTES);
-  uint64_t* empty = full + kStages;
-  uint64_t* tfull = empty + kStages;       // [2] accumulator ready for the epilogue
-  uint64_t* tempty = tfull + 2;            // [2] accumulator drained by the epilogue
+  uint64_t* full = reinterpret_cast<uint64_t*>(base + S * STAGE_BYTES);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;             // [2] accumulator ready for the epilogue
+  uint64_t* tempty = tfull + 2;            // [2] accumulator drained by the epilogue (leader's, in PAIR)
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
   if (warp == 0 && lane == 0) {
-    for (int s = 0; s < kStages; ++s) {
+    for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], 4);            // one arrival per epilogue warp
+      mbar_init(&tempty[a], PAIR ? 8 : 4);   // one arrival per epilogue warp (of both CTAs)
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tAhi) : "memory");
@@ -173,48 +222,65 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBlo) : "memory");
   }
   if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)),
-                 "n"(kAccCols));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    if (PAIR) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)),
+                   "n"(kAccCols));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)),
+                   "n"(kAccCols));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
+  if (PAIR) cluster_sync_all();   // both CTAs' barriers initialised before any cross-CTA traffic
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tslot;
 
   if (warp == 0) {
-    if (lane == 0) {  // ===== TMA producer
+    if (lane == 0) {  // ===== TMA producer (both CTAs in PAIR mode)
       int it = 0;
-      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const TileGeo g = tile_geo<BN>(job, C, tile);
+      for (int tile = unit0; tile < ntiles; tile += ustride) {
+        const TileGeo g = tile_geo<BN, PAIR>(job, C, tile, (int)rank);
         for (int kb = 0; kb < nkb; ++kb, ++it) {
-          const int s = it % kStages;
-          if (it >= kStages) mbar_wait(&empty[s], (uint32_t)(((it / kStages) - 1) & 1));
+          const int s = it % S;
+          if (it >= S) mbar_wait(&empty[s], (uint32_t)(((it / S) - 1) & 1));
           uint8_t* st = base + s * STAGE_BYTES;
-          mbar_expect_tx(&full[s], STAGE_BYTES);
           const int32_t kx = g.kx0 + kb * BK;
-          tma_load_2d(st, &tAhi, kx, g.ya, &full[s]);
-          tma_load_2d(st + A_BYTES, &tAlo, kx, g.ya, &full[s]);
-          tma_load_2d(st + 2 * A_BYTES, &tBhi, kx, g.yb, &full[s]);
-          tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, g.yb, &full[s]);
+          if (PAIR) {
+            if (leader) mbar_expect_tx(&full[s], 2 * STAGE_BYTES);
+            const uint32_t fb = peer_addr(&full[s], 0);
+            const int32_t yb = g.yb + (int32_t)rank * (BN / 2);
+            tma_load_2d_pair(st, &tAhi, kx, g.ya, fb);
+            tma_load_2d_pair(st + A_BYTES, &tAlo, kx, g.ya, fb);
+            tma_load_2d_pair(st + 2 * A_BYTES, &tBhi, kx, yb, fb);
+            tma_load_2d_pair(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, yb, fb);
+          } else {
+            mbar_expect_tx(&full[s], STAGE_BYTES);
+            tma_load_2d(st, &tAhi, kx, g.ya, &full[s]);
+            tma_load_2d(st + A_BYTES, &tAlo, kx, g.ya, &full[s]);
+            tma_load_2d(st + 2 * A_BYTES, &tBhi, kx, g.yb, &full[s]);
+            tma_load_2d(st + 2 * A_BYTES + B_BYTES, &tBlo, kx, g.yb, &full[s]);
+          }
         }
       }
     }
     __syncwarp();
   } else if (warp == 1) {
-    if (lane == 0) {  // ===== MMA issuer
+    if (lane == 0 && leader) {  // ===== MMA issuer (the leader CTA in PAIR mode)
       const uint32_t idesc = (1u << 4)                 // D: fp32
                              | (2u << 7) | (2u << 10)  // A, B: tf32
-                             | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+                             | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)((PAIR ? 2 * BM : BM) >> 4) << 24);
       int it = 0, lt = 0;
-      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++lt) {
+      for (int tile = unit0; tile < ntiles; tile += ustride, ++lt) {
         const int ab = lt & 1;
         if (lt >= 2) mbar_wait(&tempty[ab], (uint32_t)(((lt >> 1) - 1) & 1));
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t acc_t = tmem + (uint32_t)(ab * BN);
         for (int kb = 0; kb < nkb; ++kb, ++it) {
-          const int s = it % kStages;
-          mbar_wait(&full[s], (uint32_t)((it / kStages) & 1));
+          const int s = it % S;
+          mbar_wait(&full[s], (uint32_t)((it / S) & 1));
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           uint8_t* st = base + s * STAGE_BYTES;
           const uint64_t ahi = sdesc(st), alo = sdesc(st + A_BYTES);
@@ -222,29 +288,69 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
 #pragma unroll
           for (int kk = 0; kk < BK / 8; ++kk) {
             const uint64_t adv = (uint64_t)(kk * 32) >> 4;  // 8 fp32 = 32 B along K inside the swizzle atom
-            mma_tf32(acc_t, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
-            mma_tf32(acc_t, ahi + adv, blo + adv, idesc, 1u);
-            mma_tf32(acc_t, ahi + adv, bhi + adv, idesc, 1u);
+            if (PAIR) {
+              mma_tf32_pair(acc_t, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
+              mma_tf32_pair(acc_t, ahi + adv, blo + adv, idesc, 1u);
+              mma_tf32_pair(acc_t, ahi + adv, bhi + adv, idesc, 1u);
+            } else {
+              mma_tf32(acc_t, alo + adv, bhi + adv, idesc, (kb | kk) != 0);
+              mma_tf32(acc_t, ahi + adv, blo + adv, idesc, 1u);
+              mma_tf32(acc_t, ahi + adv, bhi + adv, idesc, 1u);
+            }
           }
-          mma_commit(&empty[s]);
+          if (PAIR) mma_commit_pair(&empty[s]);
+          else mma_commit(&empty[s]);
         }
-        mma_commit(&tfull[ab]);
+        if (PAIR) mma_commit_pair(&tfull[ab]);
+        else mma_commit(&tfull[ab]);
       }
     }
     __syncwarp();
   } else {  // ===== epilogue: warps 2..5 -> TMEM lane groups (warp % 4)
     const int grp = warp & 3;
     int lt = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x, ++lt) {
+    for (int tile = unit0; tile < ntiles; tile += ustride, ++lt) {
       const int ab = lt & 1;
-      const TileGeo g = tile_geo<BN>(job, C, tile);
+      const TileGeo g = tile_geo<BN, PAIR>(job, C, tile, (int)rank);
       mbar_wait(&tfull[ab], (uint32_t)((lt >> 1) & 1));
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const int64_t r = (int64_t)g.m_blk * BM + grp * 32 + lane;  // output row
       const bool row_ok = job.mode >= 1 || r < mrows;
       float* crow = job.mode >= 1 ? g.C + r * job.b : g.C + (row0 + r) * N;
+      if (job.mode >= 1) {
+        // C_tile -= acc (tile row r, ldc = b), 64 columns per round: the 16
+        // float4 loads of C are issued before the TMEM loads so their latency
+        // overlaps (ncols is a multiple of 128 in modes 1 and 2)
 #pragma unroll 1
-      for (int c = 0; c < g.ncols; c += 16) {
+        for (int c = 0; c < g.ncols; c += 64) {
+          float4* p = reinterpret_cast<float4*>(crow + (int64_t)g.n_blk * BN + c);
+          float4 o[16];
+#pragma unroll
+          for (int q = 0; q < 16; ++q) o[q] = p[q];
+          uint32_t v[64];
+          const uint32_t ta = tmem + (uint32_t)(ab * BN) + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
+#pragma unroll
+          for (int h = 0; h < 4; ++h)
+            asm volatile(
+                "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+                : "=r"(v[16 * h + 0]), "=r"(v[16 * h + 1]), "=r"(v[16 * h + 2]), "=r"(v[16 * h + 3]),
+                  "=r"(v[16 * h + 4]), "=r"(v[16 * h + 5]), "=r"(v[16 * h + 6]), "=r"(v[16 * h + 7]),
+                  "=r"(v[16 * h + 8]), "=r"(v[16 * h + 9]), "=r"(v[16 * h + 10]), "=r"(v[16 * h + 11]),
+                  "=r"(v[16 * h + 12]), "=r"(v[16 * h + 13]), "=r"(v[16 * h + 14]), "=r"(v[16 * h + 15])
+                : "r"(ta + (uint32_t)(16 * h)));
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+          for (int q = 0; q < 16; ++q) {
+            o[q].x -= __uint_as_float(v[4 * q]);
+            o[q].y -= __uint_as_float(v[4 * q + 1]);
+            o[q].z -= __uint_as_float(v[4 * q + 2]);
+            o[q].w -= __uint_as_float(v[4 * q + 3]);
+            p[q] = o[q];
+          }
+        }
+      }
+#pragma unroll 1
+      for (int c = 0; job.mode == 0 && c < g.ncols; c += 16) {
         uint32_t v[16];
         const uint32_t ta = tmem + (uint32_t)(ab * BN) + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
         asm volatile(
@@ -254,18 +360,7 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
             : "r"(ta));
         asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
         const int64_t n0 = (int64_t)g.n_blk * BN + c;
-        if (job.mode >= 1) {   // C_tile -= acc (tile row r, ldc = b)
-          float4* p = reinterpret_cast<float4*>(crow + n0);
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            float4 o = p[q];
-            o.x -= __uint_as_float(v[4 * q]);
-            o.y -= __uint_as_float(v[4 * q + 1]);
-            o.z -= __uint_as_float(v[4 * q + 2]);
-            o.w -= __uint_as_float(v[4 * q + 3]);
-            p[q] = o;
-          }
-        } else if (row_ok) {
+        if (row_ok) {
           if (n0 + 16 <= N && (N & 3) == 0) {
 #pragma unroll
             for (int q = 0; q < 4; ++q)
@@ -281,15 +376,43 @@ __global__ void __launch_bounds__(kThreadsGemm, 1)
       }
       asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
       __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[ab]);
+      if (lane == 0) {
+        if (PAIR)
+          asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(peer_addr(&tempty[ab], 0))
+                       : "memory");
+        else
+          mbar_arrive(&tempty[ab]);
+      }
     }
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
+  if (PAIR) cluster_sync_all();   // no TMA, MMA or remote arrive may target an exited CTA
   if (warp == 1) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kAccCols));
+    if (PAIR)
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kAccCols));
+    else
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kAccCols));
   }
+}
+
+template <int BN>
+__global__ void __launch_bounds__(kThreadsGemm, 1)
+    gemm_tf32x3(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
+                const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
+                float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb, int ntiles,
+                const __grid_constant__ GemmJob job) {
+  gemm_body<BN, false>(tAhi, tAlo, tBhi, tBlo, C, N, row0, mrows, nkb, ntiles, job);
+}
+
+template <int BN>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreadsGemm, 1)
+    gemm_tf32x3_pair(const __grid_constant__ CUtensorMap tAhi, const __grid_constant__ CUtensorMap tAlo,
+                   const __grid_constant__ CUtensorMap tBhi, const __grid_constant__ CUtensorMap tBlo,
+                   float* __restrict__ C, int64_t N, int64_t row0, int64_t mrows, int nkb, int npairs,
+                   const __grid_constant__ GemmJob job) {
+  gemm_body<BN, true>(tAhi, tAlo, tBhi, tBlo, C, N, row0, mrows, nkb, npairs, job);
 }
 
 __device__ __forceinline__ float tf32_rn(float x) {
@@ -372,29 +495,48 @@ uint64_t split_tag(const Scratch* scr, int32_t k) { return (scr->epoch << 20) | 
 cudaError_t set_gemm_smem() {
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(gemm_tf32x3<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes<256>());
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(gemm_tf32x3<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes<64>());
-    if (e != cudaSuccess) return e;
+    const void* fns[4] = {(const void*)gemm_tf32x3<256>, (const void*)gemm_tf32x3<64>,
+                          (const void*)gemm_tf32x3_pair<256>, (const void*)gemm_tf32x3_pair<64>};
+    const int sm[4] = {gemm_smem<256, false>(), gemm_smem<64, false>(), gemm_smem<256, true>(),
+                       gemm_smem<64, true>()};
+    for (int i = 0; i < 4; ++i) {
+      cudaError_t e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, sm[i]);
+      if (e != cudaSuccess) return e;
+    }
     attr = true;
   }
   return cudaSuccess;
 }
 
-// Launch the persistent GEMM over ntiles tiles: at most `cap` CTAs when set
-// (mode 0: one run of tiles per SM), else runs of up to 4 tiles per CTA so
-// CTAs retire regularly and other streams' kernels get SMs (MK-DAG lookahead).
+// 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0
+// turns it off).
+bool use_mc(const GemmJob& job) {
+  static const int env = getenv("MM_GEMM_PAIR") ? atoi(getenv("MM_GEMM_PAIR")) : 1;
+  return env != 0 && job.mblk >= 2 && job.mblk % 2 == 0;
+}
+
+// Launch the persistent GEMM: at most `cap` CTAs when set (mode 0: one run
+// of work units per SM), else runs of up to 4 units per CTA so CTAs retire
+// regularly and other streams' kernels get SMs (MK-DAG lookahead).  The B
+// tensor maps must have BN/2-row boxes when use_mc(job).
 template <int BN_>
 cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, const CUtensorMap& tb_hi,
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
                         const GemmJob& job, int cap, cudaStream_t s) {
+  const bool mc = use_mc(job);
   const int ntiles = job.mblk * job.nblk * (job.mode >= 1 ? job.n : 1);
   if (ntiles <= 0) return cudaSuccess;
+  const int units = mc ? ntiles / 2 : ntiles;
+  const int slots = mc ? 74 : 148;            // CTA (pairs) resident at once
   int grid;
-  if (cap > 0) grid = std::min(ntiles, cap);
-  else grid = std::max(std::min(ntiles, 148), (ntiles + 3) / 4);
-  gemm_tf32x3<BN_><<<grid, kThreadsGemm, smem_bytes<BN_>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0, mrows,
-                                                                 nkb, ntiles, job);
+  if (cap > 0) grid = std::min(units, mc ? cap / 2 : cap);
+  else grid = std::max(std::min(units, slots), (units + 3) / 4);
+  if (mc)
+    gemm_tf32x3_pair<BN_><<<2 * grid, kThreadsGemm, gemm_smem<BN_, true>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N,
+                                                                               row0, mrows, nkb, units, job);
+  else
+    gemm_tf32x3<BN_><<<grid, kThreadsGemm, gemm_smem<BN_, false>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0,
+                                                                         mrows, nkb, units, job);
   return cudaSuccess;
 }
 
@@ -426,14 +568,14 @@ cudaError_t split_needed(float* A, int64_t T, int64_t b, int32_t k, const int32_
 }
 
 cudaError_t panel_maps(Scratch* scr, int64_t T, int64_t b, CUtensorMap* ta_hi, CUtensorMap* ta_lo,
-                       CUtensorMap* tb_hi, CUtensorMap* tb_lo) {
+                       CUtensorMap* tb_hi, CUtensorMap* tb_lo, uint32_t b_box) {
   float* hi = static_cast<float*>(scr->ptr);
   float* lo = hi + 2 * T * b * b;
   cudaError_t e;
   if ((e = encode_tmap_2d_f32(ta_hi, hi, b, 2 * T * b, b * 4, BK, BM)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(ta_lo, lo, b, 2 * T * b, b * 4, BK, BM)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(tb_hi, hi, b, 2 * T * b, b * 4, BK, BN)) != cudaSuccess) return e;
-  return encode_tmap_2d_f32(tb_lo, lo, b, 2 * T * b, b * 4, BK, BN);
+  if ((e = encode_tmap_2d_f32(tb_hi, hi, b, 2 * T * b, b * 4, BK, b_box)) != cudaSuccess) return e;
+  return encode_tmap_2d_f32(tb_lo, lo, b, 2 * T * b, b * 4, BK, b_box);
 }
 
 }  // namespace
@@ -455,7 +597,10 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
   if (e != cudaSuccess) return e;
   // 2. one batched GEMM launch over all tasks
   CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
-  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo)) != cudaSuccess) return e;
+  GemmJob probe;
+  probe.mblk = (int32_t)(b / BM);
+  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo, use_mc(probe) ? BN / 2 : BN)) != cudaSuccess)
+    return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
   for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
     GemmJob job;
@@ -500,7 +645,10 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
   if (n <= 0 || n0 >= b) return cudaSuccess;
   CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
   cudaError_t e;
-  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo)) != cudaSuccess) return e;
+  GemmJob probe;
+  probe.mblk = (int32_t)(b / BM);
+  if ((e = panel_maps(scr, T, b, &ta_hi, &ta_lo, &tb_hi, &tb_lo, use_mc(probe) ? BN / 2 : BN)) != cudaSuccess)
+    return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
   for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
     GemmJob job;
@@ -564,8 +712,11 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   const int cap = sms > 0 ? sms : 148;
   const bool narrow = ((mrows + BM - 1) / BM) * ((N + BN - 1) / BN) < cap;   // fewer 128x256 tiles than SMs
   const uint32_t bn = narrow ? 64 : BN;
-  if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, bn)) != cudaSuccess) return e;
-  if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, bn)) != cudaSuccess) return e;
+  GemmJob probe;
+  probe.mblk = (int32_t)((mrows + BM - 1) / BM);
+  const uint32_t b_box = use_mc(probe) ? bn / 2 : bn;
+  if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, b_box)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, b_box)) != cudaSuccess) return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
   GemmJob job;
   job.mode = 0;
