@@ -173,6 +173,28 @@ def cpu_baseline(app: str, seconds: float = 10.0):
         dt = time.perf_counter() - t0
         return {"value": 20 * n * k / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
                 "sample": f"{k} passes over 2^22 options"}
+    if app == "cholesky":
+        n = 768
+        A = synthgen.spd_random(n).astype(np.float64)
+        t0 = time.perf_counter()
+        k = 0
+        while time.perf_counter() - t0 < seconds:
+            on.cholesky(A)
+            k += 1
+        dt = time.perf_counter() - t0
+        return {"value": n ** 3 / 3 * k / dt / 1e12, "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
+                "sample": f"{k} unblocked FP64 Cholesky factorizations of a 768^2 SPD matrix (n^3/3 flop each)"}
+    if app == "nbody":
+        n = 1 << 20
+        pos, vel = synthgen.nbody(n)
+        t0 = time.perf_counter()
+        k = 0
+        while time.perf_counter() - t0 < seconds:
+            on.nbody_step_bodies(pos, vel, list(range(k % n, k % n + 256)))
+            k += 256
+        dt = time.perf_counter() - t0
+        return {"value": 20 * n * k / dt / 1e12, "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
+                "sample": f"{k} bodies of the 2^20-body step, each summed over all 2^20 bodies (20 flop/interaction)"}
     n = 512
     A, B = synthgen.matmul_uniform(n, n, n)
     t0 = time.perf_counter()
@@ -189,7 +211,7 @@ def run_reference(args):
     world, rank, local = dist_env()
     if rank != 0:
         return
-    unit = "TFLOP/s" if args.app == "sgemm" else "GB/s"
+    unit = "TFLOP/s" if args.app in FLOP_APPS else "GB/s"
     # each step = a bounded sample of the workload on the oracle (host cores)
     vals = []
     for i in range(args.warmup + args.steps):

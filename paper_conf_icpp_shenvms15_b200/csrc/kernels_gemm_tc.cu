@@ -510,9 +510,10 @@ cudaError_t set_gemm_smem() {
 
 // 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0
 // turns it off).
-bool use_mc(const GemmJob& job) {
+// The 128x64 narrow tiles of small SGEMMs stay single-SM (measured faster).
+bool use_mc(const GemmJob& job, int bn = BN) {
   static const int env = getenv("MM_GEMM_PAIR") ? atoi(getenv("MM_GEMM_PAIR")) : 1;
-  return env != 0 && job.mblk >= 2 && job.mblk % 2 == 0;
+  return env != 0 && bn == BN && job.mblk >= 2 && job.mblk % 2 == 0;
 }
 
 // Launch the persistent GEMM: at most `cap` CTAs when set (mode 0: one run
@@ -523,7 +524,7 @@ template <int BN_>
 cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, const CUtensorMap& tb_hi,
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
                         const GemmJob& job, int cap, cudaStream_t s) {
-  const bool mc = use_mc(job);
+  const bool mc = use_mc(job, BN_);
   const int ntiles = job.mblk * job.nblk * (job.mode >= 1 ? job.n : 1);
   if (ntiles <= 0) return cudaSuccess;
   const int units = mc ? ntiles / 2 : ntiles;
@@ -714,7 +715,7 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   const uint32_t bn = narrow ? 64 : BN;
   GemmJob probe;
   probe.mblk = (int32_t)((mrows + BM - 1) / BM);
-  const uint32_t b_box = use_mc(probe) ? bn / 2 : bn;
+  const uint32_t b_box = use_mc(probe, (int)bn) ? bn / 2 : bn;
   if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, b_box)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, b_box)) != cudaSuccess) return e;
   if ((e = set_gemm_smem()) != cudaSuccess) return e;
