@@ -359,6 +359,70 @@ def test_cholesky_random_spd(R, nb):
     assert np.max(np.abs(L - ref)) / np.max(np.abs(ref)) <= 1e-4
 
 
+_CHOL_SCRIPT = r"""
+import sys, numpy as np
+sys.path.insert(0, {root!r})
+import synthgen
+from paper_conf_icpp_shenvms15_b200 import mm, runner
+n, b = {n}, {b}
+A = synthgen.spd_random(n)
+T = n // b
+At = A.reshape(T, b, T, b).transpose(0, 2, 1, 3).reshape(-1)
+rnd = np.random.default_rng(3)
+G = 1
+prof = mm.make_profile(G, rnd.integers(500, 3000, size=(G, 4)).tolist(),
+                       rnd.integers(10 ** 4, 10 ** 6, size=(G, 4)).tolist(), [10 ** 10])
+with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=G) as s:
+    s.load(0, At)
+    plan = s.plan(4, prof)
+    s.run(plan)
+    np.save({out!r}, s.collect(plan, 0))
+"""
+
+
+@pytest.mark.parametrize("nb", [(1024, 256), (1024, 128)])
+def test_cholesky_random_spd_schedule_invariant(R, nb):
+    """on random SPD data (inexact arithmetic) the factor is the
+    same bit for bit under every schedule and device count — each tile's
+    updates run in the WAW-chain order, and no kernel's arithmetic depends on
+    how the runtime batches the tasks of a step."""
+    mm, runner = R
+    n, b = nb
+    A = synthgen.spd_random(n)
+    ref = None
+    for strategy, G in ((4, 1), (4, 2), (5, 3), (6, 2), (4, 3)):
+        with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=G) as s:
+            s.load(0, _to_tiles(A, b))
+            plan = s.plan(strategy, rand_profile(mm, G, 4, 11 * G + strategy))
+            s.run(plan)
+            got = s.collect(plan, 0)
+        if ref is None:
+            ref = got
+        assert np.array_equal(got, ref), (strategy, G)
+
+
+def test_cholesky_trsm_leaf_variants_identical(gpu, tmp_path):
+    """The wide (one 256-row CTA per SM, large batches) and narrow (64-row
+    CTAs, small batches) TRSM leaves do the same arithmetic: forcing the wide
+    leaf for every batch (MM_LEAF_WIDE_MIN=1, a fresh process) gives the
+    default run's factor bit for bit."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    outs = []
+    for env_min in (None, "1"):
+        out = str(tmp_path / f"chol_{env_min}.npy")
+        env = dict(os.environ)
+        env.pop("MM_LEAF_WIDE_MIN", None)
+        if env_min:
+            env["MM_LEAF_WIDE_MIN"] = env_min
+        code = _CHOL_SCRIPT.format(root=root, n=2048, b=512, out=out)
+        subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=root, timeout=600)
+        outs.append(np.load(out))
+    assert np.array_equal(outs[0], outs[1])
+
+
 def test_cholesky_device_spd_generator(R):
     mm, runner = R
     n, b = 384, 128
