@@ -310,14 +310,17 @@ cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t ro
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
   const size_t smem = (size_t)kTbWarps * 2 * C::RR * 32 * sizeof(float4);
   static bool attr = false;
+  static int per_sm = 0;   // resident CTAs per SM (registers bound it)
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(hotspot_tb<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hotspot_tb<H>, 32 * kTbWarps, smem);
+    if (e != cudaSuccess || per_sm < 1) per_sm = 1;
     attr = true;
   }
-  // one wave of ~16 warps per SM; strips at least 8H rows tall (vertical
-  // redundancy (2H+1)/SR)
-  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * 16;
+  // exactly one wave of resident warps (a partial second wave left SMs
+  // idle); strips at least 8H rows tall (vertical redundancy (2H+1)/SR)
+  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm * kTbWarps;
   const int64_t nr = r1 - r0;
   int64_t nstrip = (target + nwx - 1) / nwx;
   int64_t SR = (nr + nstrip - 1) / nstrip;
