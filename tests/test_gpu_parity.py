@@ -322,7 +322,7 @@ def _from_tiles(t, n, b):
     return t.reshape(T, T, b, b).transpose(0, 2, 1, 3).reshape(n, n)
 
 
-@pytest.mark.parametrize("nb", [(512, 128), (1024, 256)])
+@pytest.mark.parametrize("nb", [(512, 128), (1024, 256), (2048, 128)])
 @pytest.mark.parametrize("strategy", [4, 5, 6])
 @pytest.mark.parametrize("G", [1, 2, 3])
 def test_cholesky_exact_factor(R, strategy, G, nb):
@@ -345,7 +345,7 @@ def test_cholesky_exact_factor(R, strategy, G, nb):
         assert np.all(np.triu(blk, 1) == 0)
 
 
-@pytest.mark.parametrize("nb", [(512, 128), (1024, 256)])
+@pytest.mark.parametrize("nb", [(512, 128), (1024, 256), (2048, 256)])
 def test_cholesky_random_spd(R, nb):
     mm, runner = R
     n, b = nb
@@ -380,7 +380,7 @@ with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=G) as s:
 """
 
 
-@pytest.mark.parametrize("nb", [(1024, 256), (1024, 128)])
+@pytest.mark.parametrize("nb", [(1024, 256), (1024, 128), (2048, 128)])
 def test_cholesky_random_spd_schedule_invariant(R, nb):
     """on random SPD data (inexact arithmetic) the factor is the
     same bit for bit under every schedule and device count — each tile's
