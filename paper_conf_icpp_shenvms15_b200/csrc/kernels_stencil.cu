@@ -110,13 +110,20 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
 // stored, so every stored cell went through exactly H applications of the
 // R16 update: bit-identical to H single-step launches.
 constexpr int kTbWarps = 4;                      // warps per CTA
-constexpr int kTbAhead = 6;                      // cp.async prefetch distance (rows)
+constexpr int kTbAhead = 5;                      // cp.async prefetch distance (rows)
+#ifndef TB_MIN_BLOCKS
+#define TB_MIN_BLOCKS 3
+#endif
+constexpr int kTbMinBlocks = TB_MIN_BLOCKS;       // resident CTAs per SM (4 = 128 registers: spills, measured slower)
 
 template <int H>
 struct TbCfg {
   static constexpr int HC = 4 * ((H + 3) / 4);   // halo columns per side (float4-aligned)
   static constexpr int OW = 128 - 2 * HC;        // output columns per warp
-  static constexpr int RR = (H + kTbAhead + 1) <= 8 ? 8 : 16;   // ring rows (power of 2 > H + ahead)
+  // ring rows (powers of 2): T rows r-2 .. r+ahead (level 1 only), P rows
+  // r-H .. r+ahead (every level)
+  static constexpr int RT = (kTbAhead + 3) <= 8 ? 8 : 16;
+  static constexpr int RP = (H + kTbAhead + 1) <= 8 ? 8 : 16;
 };
 
 struct f2 {
@@ -203,12 +210,11 @@ struct TbArgs {
 // issue the copies of level-0 row q (T and P) into the ring, one commit group
 template <int H>
 __device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs<H>& a, int q) {
-  constexpr int RR = TbCfg<H>::RR;
+  constexpr int RT = TbCfg<H>::RT, RP = TbCfg<H>::RP;
   if (q < a.re && q >= 0 && q < a.rows && a.inx) {
-    const int slot = (q & (RR - 1)) * 32 + a.lane;
     const int64_t off = (int64_t)q * a.cols + a.x0;
-    cp16(tr + slot, a.tin + off);
-    cp16(pr + slot, a.pw + off);
+    cp16(tr + (q & (RT - 1)) * 32 + a.lane, a.tin + off);
+    cp16(pr + (q & (RP - 1)) * 32 + a.lane, a.pw + off);
   }
   cp_commit();
 }
@@ -219,16 +225,15 @@ __device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs<H>
 template <int H, int PH, bool EDGE>
 __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3], const float4* tr, const float4* pr,
                                           const TbArgs<H>& a, int r, const HotCoef2& k) {
-  constexpr int RR = TbCfg<H>::RR;
-  const int rb = r & (RR - 1);
+  constexpr int RT = TbCfg<H>::RT, RP = TbCfg<H>::RP;
 #pragma unroll
   for (int s = 1; s <= H; ++s) {
     const int y = r - s;
     float4 cu, up, dn;
     if (s == 1) {                                 // level 0 rows from the ring
-      cu = tr[((rb - 1) & (RR - 1)) * 32 + a.lane];
-      up = tr[((rb - 2) & (RR - 1)) * 32 + a.lane];
-      dn = tr[rb * 32 + a.lane];
+      cu = tr[((r - 1) & (RT - 1)) * 32 + a.lane];
+      up = tr[((r - 2) & (RT - 1)) * 32 + a.lane];
+      dn = tr[(r & (RT - 1)) * 32 + a.lane];
     } else {
       cu = W[s - 2][((PH - s) % 3 + 3) % 3];
       up = W[s - 2][((PH - s - 1) % 3 + 3) % 3];
@@ -238,7 +243,7 @@ __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3], con
       if (y <= 0) up = cu;                        // chip edge: neighbour = the cell itself
       if (y + 1 >= a.rows) dn = cu;
     }
-    const float4 p = pr[((rb - s) & (RR - 1)) * 32 + a.lane];
+    const float4 p = pr[((r - s) & (RP - 1)) * 32 + a.lane];
     float w = __shfl_up_sync(0xffffffffu, cu.w, 1);
     float e = __shfl_down_sync(0xffffffffu, cu.x, 1);
     if (a.wedge) w = cu.x;
@@ -264,7 +269,7 @@ __device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3], float
 }
 
 template <int H>
-__global__ void __launch_bounds__(32 * kTbWarps) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
+__global__ void __launch_bounds__(32 * kTbWarps, kTbMinBlocks) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
                                                              float* __restrict__ tout, int rows, int cols, int r0, int r1,
                                                              HotCoef kc, int nwx, int SR) {
   using C = TbCfg<H>;
@@ -284,8 +289,8 @@ __global__ void __launch_bounds__(32 * kTbWarps) hotspot_tb(const float* __restr
   a.store_x = a.inx && a.x0 >= X0 && a.x0 < X0 + C::OW;
   a.wedge = a.x0 == 0;
   a.eedge = a.x0 + 4 == cols;
-  float4* tr = tb_smem + (size_t)wid * 2 * C::RR * 32;
-  float4* pr = tr + C::RR * 32;
+  float4* tr = tb_smem + (size_t)wid * (C::RT + C::RP) * 32;
+  float4* pr = tr + C::RT * 32;
   HotCoef2 k;
   k.ry1 = kc.ry1; k.rx1 = kc.rx1; k.rz1 = kc.rz1; k.sdc = kc.sdc;
   k.amb = pk(kc.amb, kc.amb);
@@ -316,7 +321,7 @@ cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t ro
   using C = TbCfg<H>;
   if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
-  const size_t smem = (size_t)kTbWarps * 2 * C::RR * 32 * sizeof(float4);
+  const size_t smem = (size_t)kTbWarps * (C::RT + C::RP) * 32 * sizeof(float4);
   static bool attr = false;
   static int per_sm = 0;   // resident CTAs per SM (registers bound it)
   if (!attr) {
