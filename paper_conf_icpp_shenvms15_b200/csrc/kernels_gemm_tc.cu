@@ -49,13 +49,16 @@ constexpr int kThreadsGemm = 192;
 //  mode 2 (TRSM block update): C = columns [n0, n0+ncols) of tile (ti, tj)
 //          -= X_i[:, kx0:kx0+K] L[n0:n0+ncols, kx0:kx0+K]^T, X_i in slot
 //          slot0+ti, L = tile (tj, tj) in slot slot0+tj.
+//  mode 3 (SGEMM rows, split K): task z = K split z: partial z (stride b
+//          floats, row-major mrows x N) = A[:, z*kx0 : (z+1)*kx0] B[...]^T;
+//          split_k_reduce adds the n partials in split order.
 // (slot s = rows s*b of the hi/lo panel buffers, K-major.)
 struct GemmJob {
-  int32_t mode;            // 0: rows of a plain SGEMM, 1: tile update, 2: TRSM block update
-  int32_t n;               // tasks (modes 1, 2)
+  int32_t mode;            // 0: rows of a plain SGEMM, 1: tile update, 2: TRSM block update, 3: split-K rows
+  int32_t n;               // tasks (modes 1, 2), K splits (mode 3)
   int64_t T, b;
   int32_t slot0;           // first slot of this step's parity
-  int32_t kx0, n0, ncols;  // mode 2
+  int32_t kx0, n0, ncols;  // mode 2 (mode 3: kx0 = K columns per split)
   int32_t mblk, nblk;      // output tiles per task
   int32_t ti[kCholBatch], tj[kCholBatch];
 };
@@ -127,7 +130,10 @@ __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int ti
   g.kx0 = 0;
   g.ncols = BN;
   g.C = C;
-  if (job.mode >= 1) {
+  if (job.mode == 3) {
+    g.kx0 = z * job.kx0;
+    g.C += (int64_t)z * job.b;
+  } else if (job.mode >= 1) {
     g.ya += (int32_t)((job.slot0 + job.ti[z]) * job.b);
     g.yb += (int32_t)((job.slot0 + job.tj[z]) * job.b);
     g.C += ((int64_t)job.ti[z] * job.T + job.tj[z]) * job.b * job.b;
@@ -315,9 +321,10 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tAhi, const CUtenso
       mbar_wait(&tfull[ab], (uint32_t)((lt >> 1) & 1));
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const int64_t r = (int64_t)g.m_blk * BM + grp * 32 + lane;  // output row
-      const bool row_ok = job.mode >= 1 || r < mrows;
-      float* crow = job.mode >= 1 ? g.C + r * job.b : g.C + (row0 + r) * N;
-      if (job.mode >= 1) {
+      const bool rmw = job.mode == 1 || job.mode == 2;
+      const bool row_ok = rmw || r < mrows;
+      float* crow = rmw ? g.C + r * job.b : g.C + (job.mode == 3 ? r : row0 + r) * N;
+      if (rmw) {
         // C_tile -= acc (tile row r, ldc = b), 64 columns per round: the 16
         // float4 loads of C are issued before the TMEM loads so their latency
         // overlaps (ncols is a multiple of 128 in modes 1 and 2)
@@ -350,7 +357,7 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tAhi, const CUtenso
         }
       }
 #pragma unroll 1
-      for (int c = 0; job.mode == 0 && c < g.ncols; c += 16) {
+      for (int c = 0; !rmw && c < g.ncols; c += 16) {
         uint32_t v[16];
         const uint32_t ta = tmem + (uint32_t)(ab * BN) + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
         asm volatile(
@@ -511,10 +518,11 @@ cudaError_t set_gemm_smem() {
 // 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0
 // turns it off).
 // The 128x64 narrow tiles of small SGEMMs stay single-SM (measured faster).
-bool use_mc(const GemmJob& job, int bn = BN) {
+bool use_mc_env() {
   static const int env = getenv("MM_GEMM_PAIR") ? atoi(getenv("MM_GEMM_PAIR")) : 1;
-  return env != 0 && bn == BN && job.mblk >= 2 && job.mblk % 2 == 0;
+  return env != 0;
 }
+bool use_mc(const GemmJob& job, int bn = BN) { return use_mc_env() && bn == BN && job.mblk >= 2 && job.mblk % 2 == 0; }
 
 // Launch the persistent GEMM: at most `cap` CTAs when set (mode 0: one run
 // of work units per SM), else runs of up to 4 units per CTA so CTAs retire
@@ -672,9 +680,48 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
   return cudaGetLastError();
 }
 
+namespace {
+// C[row0 + r][n] = ((p_0 + p_1) + ...) + p_{S-1}  (fixed split order)
+__global__ void split_k_reduce(const float* __restrict__ part, float* __restrict__ C, int64_t N, int64_t row0,
+                               int64_t mrows, int S) {
+  const int64_t stride = mrows * N;
+  if ((N & 3) == 0) {
+    const int64_t n4 = stride / 4;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+      float4 a = reinterpret_cast<const float4*>(part)[i];
+      for (int z = 1; z < S; ++z) {
+        const float4 b = reinterpret_cast<const float4*>(part + z * stride)[i];
+        a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+      }
+      reinterpret_cast<float4*>(C + row0 * N)[i] = a;
+    }
+  } else {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < stride; i += (int64_t)gridDim.x * blockDim.x) {
+      float a = part[i];
+      for (int z = 1; z < S; ++z) a += part[z * stride + i];
+      C[row0 * N + i] = a;
+    }
+  }
+}
+}  // namespace
+
+// K splits for a row range too small to give every SM pair a 256 x 256 tile
+// pair: S in {4, 3, 2} dividing the K blocks with >= 8 blocks per split and
+// pairs * S <= the 74 pair slots; 1 = no split.  Depends only on the shape,
+// so every run of the same row range does the same arithmetic.
+int splitk_factor(int64_t mrows, int64_t N, int64_t Kp) {
+  const int64_t mblk = (mrows + BM - 1) / BM, nblk = (N + BN - 1) / BN, nkb = Kp / BK;
+  if (mblk < 2 || mblk % 2) return 1;
+  const int64_t pairs = mblk / 2 * nblk;
+  for (int S = 4; S >= 2; --S)
+    if (pairs * S <= 74 && nkb % S == 0 && nkb / S >= 8) return S;
+  return 1;
+}
+
 size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
   const int64_t Kp = (K + KPAD - 1) / KPAD * KPAD;
-  return (size_t)(2 * mrows * Kp + 2 * N * Kp) * sizeof(float);
+  const int S = splitk_factor(mrows, N, Kp);
+  return (size_t)(2 * mrows * Kp + 2 * N * Kp + (S > 1 ? S * mrows * N : 0)) * sizeof(float);
 }
 
 cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
@@ -711,6 +758,33 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   if ((e = encode_tmap_2d_f32(&ta_hi, ahi, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
   if ((e = encode_tmap_2d_f32(&ta_lo, alo, Kp, mrows, Kp * 4, BK, BM)) != cudaSuccess) return e;
   const int cap = sms > 0 ? sms : 148;
+  const int S = cap >= 148 && use_mc_env() ? splitk_factor(mrows, N, Kp) : 1;
+  if (S > 1) {   // 2-SM 256 x 256 tile pairs over K splits, then the ordered reduction
+    GemmJob probe;
+    probe.mblk = (int32_t)((mrows + BM - 1) / BM);
+    if ((e = encode_tmap_2d_f32(&tb_hi, bhi, Kp, N, Kp * 4, BK, BN / 2)) != cudaSuccess) return e;
+    if ((e = encode_tmap_2d_f32(&tb_lo, blo, Kp, N, Kp * 4, BK, BN / 2)) != cudaSuccess) return e;
+    if ((e = set_gemm_smem()) != cudaSuccess) return e;
+    float* part = alo + mrows * Kp;
+    GemmJob job;
+    job.mode = 3;
+    job.n = S;
+    job.T = 0;
+    job.b = mrows * N;
+    job.slot0 = job.n0 = 0;
+    job.kx0 = (int32_t)(Kp / S);
+    job.ncols = BN;
+    job.mblk = probe.mblk;
+    job.nblk = (int32_t)((N + BN - 1) / BN);
+    if ((e = launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, part, N, 0, mrows, (int)(Kp / S / BK), job, cap, s)) !=
+        cudaSuccess)
+      return e;
+    const int64_t work = (N & 3) == 0 ? mrows * N / 4 : mrows * N;
+    int64_t blocks = (work + 255) / 256;
+    if (blocks > 148 * 8) blocks = 148 * 8;
+    split_k_reduce<<<(unsigned)blocks, 256, 0, s>>>(part, C, N, r0, mrows, S);
+    return cudaGetLastError();
+  }
   const bool narrow = ((mrows + BM - 1) / BM) * ((N + BN - 1) / BN) < cap;   // fewer 128x256 tiles than SMs
   const uint32_t bn = narrow ? 64 : BN;
   GemmJob probe;
