@@ -2,10 +2,26 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <atomic>
 #include <cstdint>
 #include <vector>
 
 namespace mm {
+
+// Kernel attributes (cudaFuncSetAttribute) are per CUDA device: run `set`
+// once for each device this process launches on (a context may span several
+// GPUs), thread-safe; `done` is a per-call-site bitmask of device ordinals.
+template <class F>
+cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const uint64_t bit = 1ull << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  e = set();
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+  return e;
+}
 
 struct Kernel;
 struct Task;

@@ -500,8 +500,8 @@ namespace {
 uint64_t split_tag(const Scratch* scr, int32_t k) { return (scr->epoch << 20) | (uint64_t)(k + 1); }
 
 cudaError_t set_gemm_smem() {
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<uint64_t> done{0};
+  return once_per_device(done, [] {
     const void* fns[4] = {(const void*)gemm_tf32x3<256>, (const void*)gemm_tf32x3<64>,
                           (const void*)gemm_tf32x3_pair<256>, (const void*)gemm_tf32x3_pair<64>};
     const int sm[4] = {gemm_smem<256, false>(), gemm_smem<64, false>(), gemm_smem<256, true>(),
@@ -510,9 +510,8 @@ cudaError_t set_gemm_smem() {
       cudaError_t e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, sm[i]);
       if (e != cudaSuccess) return e;
     }
-    attr = true;
-  }
-  return cudaSuccess;
+    return cudaSuccess;
+  });
 }
 
 // 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0

@@ -322,18 +322,21 @@ cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t ro
   if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
   const size_t smem = (size_t)kTbWarps * (C::RT + C::RP) * 32 * sizeof(float4);
-  static bool attr = false;
-  static int per_sm = 0;   // resident CTAs per SM (registers bound it)
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(hotspot_tb<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hotspot_tb<H>, 32 * kTbWarps, smem);
-    if (e != cudaSuccess || per_sm < 1) per_sm = 1;
-    attr = true;
-  }
+  static std::atomic<uint64_t> attr{0};
+  static std::atomic<int> per_sm{0};   // resident CTAs per SM (registers bound it; same on every B200)
+  cudaError_t e = once_per_device(attr, [&] {
+    cudaError_t r = cudaFuncSetAttribute(hotspot_tb<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (r != cudaSuccess) return r;
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, hotspot_tb<H>, 32 * kTbWarps, smem) != cudaSuccess || n < 1)
+      n = 1;
+    per_sm.store(n);
+    return cudaSuccess;
+  });
+  if (e != cudaSuccess) return e;
   // exactly one wave of resident warps (a partial second wave left SMs
   // idle); strips at least 8H rows tall (vertical redundancy (2H+1)/SR)
-  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm * kTbWarps;
+  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm.load() * kTbWarps;
   const int64_t nr = r1 - r0;
   int64_t nstrip = (target + nwx - 1) / nwx;
   int64_t SR = (nr + nstrip - 1) / nstrip;
