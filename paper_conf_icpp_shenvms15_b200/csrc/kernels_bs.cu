@@ -4,12 +4,14 @@
 // European call and put per option (NVIDIA SDK formulation [ext]):
 //   d1 = (ln(S/X) + (R + V^2/2) T) / (V sqrt T), d2 = d1 - V sqrt T
 //   call = S N(d1) - X e^{-RT} N(d2), put = X e^{-RT} (1 - N(d2)) - S (1 - N(d1))
-// N = Abramowitz-Stegun 26.2.17.  FP32; the accurate libdevice logf and sqrtf
-// (ln(S/X) near 0 needs the absolute accuracy) with the SFU exp (ex2.approx)
-// and approximate division elsewhere — the accurate versions made the kernel
+// N = Abramowitz-Stegun 26.2.17.  FP32; the accurate libdevice logf (ln(S/X)
+// near 0 needs the absolute accuracy) with the SFU exp2 / rcp / rsqrt
+// (approx.ftz) elsewhere — the accurate versions made the kernel
 // ALU-bound (61% of HBM peak measured); the error stays far inside the 1e-5
 // tolerance (R19).  20 algorithmic bytes per option, HBM-bound; float4 I/O,
 // 4 options per thread.
+#include <cstdlib>
+
 #include "kernels.h"
 
 namespace mm {
@@ -18,23 +20,46 @@ namespace {
 
 constexpr int kThreads = 256;
 
+// SFU approximations in their flush-to-zero forms: the non-ftz intrinsics
+// (__expf, __fdividef, rsqrtf) wrap every MUFU op in a denormal range check
+// (FSETP + FMUL + FSEL), which made the kernel issue-bound (ncu: 106
+// instructions per option, issue slots 86 % busy).  Arguments here are normal
+// (S, X, T > 0; |d| moderate) and a denormal result is a price below 1e-38,
+// far inside the 1e-5 tolerance (R19).
+__device__ __forceinline__ float ex2_ftz(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ float rcp_ftz(float x) {
+  float y;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ float rsqrt_ftz(float x) {
+  float y;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ float exp_ftz(float x) { return ex2_ftz(x * 1.4426950408889634f); }
+
 __device__ __forceinline__ float cnd(float d) {
   const float A1 = 0.31938153f, A2 = -0.356563782f, A3 = 1.781477937f, A4 = -1.821255978f,
               A5 = 1.330274429f, RSQRT2PI = 0.39894228040143267793994605993438f;
-  const float k = __fdividef(1.0f, 1.0f + 0.2316419f * fabsf(d));
-  float c = RSQRT2PI * __expf(-0.5f * d * d) * (k * (A1 + k * (A2 + k * (A3 + k * (A4 + k * A5)))));
+  const float k = rcp_ftz(1.0f + 0.2316419f * fabsf(d));
+  float c = RSQRT2PI * exp_ftz(-0.5f * d * d) * (k * (A1 + k * (A2 + k * (A3 + k * (A4 + k * A5)))));
   if (d > 0) c = 1.0f - c;
   return c;
 }
 
 __device__ __forceinline__ void option(float s, float x, float t, float R, float V, float& call,
                                        float& put) {
-  const float rsT = rsqrtf(t);                     // MUFU.RSQ: 1/sqrt(T)
+  const float rsT = rsqrt_ftz(t);                  // MUFU.RSQ: 1/sqrt(T)
   const float vst = V * (t * rsT);                 // V sqrt(T)
-  const float d1 = (logf(__fdividef(s, x)) + (R + 0.5f * V * V) * t) * (rsT * (1.0f / V));
+  const float d1 = (logf(s * rcp_ftz(x)) + (R + 0.5f * V * V) * t) * (rsT * (1.0f / V));
   const float d2 = d1 - vst;
   const float n1 = cnd(d1), n2 = cnd(d2);
-  const float expRT = __expf(-R * t);
+  const float expRT = exp_ftz(-R * t);
   call = s * n1 - x * expRT * n2;
   put = x * expRT * (1.0f - n2) - s * (1.0f - n1);
 }
@@ -93,8 +118,12 @@ cudaError_t blackscholes(const float* S, const float* X, const float* T, float* 
     const int64_t n4 = n / 4;
     if (n4) {
       int64_t blocks = (n4 + kThreads - 1) / kThreads;
-      const int64_t cap = (int64_t)(sms > 0 ? sms : 148) * 8;  // persistent: 8 CTAs per SM
-      if (blocks > cap) blocks = cap;
+      // persistent grid of 4 CTAs (32 warps) per SM: measured 95.9 % of the copy
+      // peak at 80.5M options vs 74-93 % for 2, 3, 5, 6, 8, 12, 16 CTAs or a
+      // non-persistent grid (MM_BS_CTAS overrides; 0 = one CTA per 512 groups)
+      static const int per_sm = getenv("MM_BS_CTAS") ? atoi(getenv("MM_BS_CTAS")) : 4;
+      const int64_t cap = (int64_t)(sms > 0 ? sms : 148) * per_sm;
+      if (per_sm > 0 && blocks > cap) blocks = cap;
       bs_vec<<<(unsigned)blocks, kThreads, 0, s>>>(
           reinterpret_cast<const float4*>(S), reinterpret_cast<const float4*>(X),
           reinterpret_cast<const float4*>(T), reinterpret_cast<float4*>(call),
