@@ -222,11 +222,13 @@ def test_blackscholes(R, G, strategy):
     assert np.max(np.abs(par) / np.maximum(S, X)) < 4e-6
 
 
-@pytest.mark.parametrize("shape", [(300, 200, 96), (257, 520, 77), (1024, 1024, 1024)])
+@pytest.mark.parametrize("shape", [(300, 200, 96), (257, 520, 77), (1024, 1024, 1024), (512, 301, 1000)])
 @pytest.mark.parametrize("variant", [1, 2])
 @pytest.mark.parametrize("G", [1, 2])
 def test_sgemm(R, variant, G, shape):
-    """variant 1 = FFMA, 2 = tcgen05 3xTF32 (TMA + TMEM); ragged M, N, K."""
+    """variant 1 = FFMA, 2 = tcgen05 3xTF32 (TMA + TMEM); ragged M, N, K.
+    1024^3 and 512 x 301 x 1000 take the split-K path (4 K splits of 2-SM
+    tile pairs + ordered reduction; the latter with a ragged N and K)."""
     mm, runner = R
     M, N, K = shape
     Ai, Bi = synthgen.matmul_integer(M, K, N)
