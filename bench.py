@@ -485,6 +485,7 @@ def main():
 
     # --- every Table I strategy for this class, w/o and w/ sync (ranking) ----
     strategies = {}
+    strategies_graph = {}
     if not args.no_strategies:
         for s_id in list(ranked) + [x for x in extras if x not in ranked]:
             try:
@@ -496,6 +497,10 @@ def main():
                     st = sess.run(p)
                     ts.append(st.device_ms)
                 ms = statistics.median(ts)
+                if world == 1:   # the same op program captured once and replayed as a CUDA graph
+                    sess.run(p, use_graph=True)
+                    tg = [sess.run(p, use_graph=True).device_ms for _ in range(3)]
+                    strategies_graph[mm.mm_strategy_name(s_id)] = round(statistics.median(tg), 4)
                 if world > 1:
                     t = torch.tensor([ms], dtype=torch.float64)
                     dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -519,7 +524,7 @@ def main():
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
                        **({"temporal_block": tb} if args.app == "hotspot" else {})},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
-            "clocks": clk.summary(), "strategies_ms": strategies,
+            "clocks": clk.summary(), "strategies_ms": strategies, "strategies_graph_ms": strategies_graph,
             "kernel_ms_per_step": {kname_map[k]: round(sum(kms[d][k] for d in my) / args.steps, 4)
                                    for k in range(K)},
             "ranking": [mm.mm_strategy_name(s) for s in ranked],
