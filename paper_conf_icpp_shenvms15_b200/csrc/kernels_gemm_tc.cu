@@ -428,37 +428,58 @@ __device__ __forceinline__ float tf32_rn(float x) {
   return __uint_as_float(r);
 }
 
-// A rows [r0, r0+mrows) x K -> hi/lo, row stride Kp (zero padding K..Kp).
-__global__ void split_rows(const float* __restrict__ A, float* __restrict__ hi, float* __restrict__ lo,
-                           int64_t K, int64_t Kp, int64_t r0, int64_t mrows) {
-  const int64_t n = mrows * Kp;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t r = i / Kp, k = i % Kp;
-    const float x = k < K ? A[(r0 + r) * K + k] : 0.f;
-    const float h = tf32_rn(x);
-    hi[i] = h;
-    lo[i] = tf32_rn(x - h);
-  }
+__device__ __forceinline__ void split2(float x, float& h, float& l) {
+  h = tf32_rn(x);
+  l = tf32_rn(x - h);
 }
 
-// B (K x N) -> hi^T/lo^T (N x Kp), 32x32 tiles through shared memory.
-__global__ void split_transpose(const float* __restrict__ B, float* __restrict__ hi, float* __restrict__ lo,
-                                int64_t K, int64_t N, int64_t Kp) {
+// One launch for both SGEMM operands: blocks [0, nblk_a) split A rows
+// [r0, r0+mrows) into hi/lo (row stride Kp, zero padding K..Kp; float4 when
+// K == Kp), blocks [nblk_a, ...) split one 32(k) x 32(n) tile of B (K x N) each
+// into hi^T/lo^T (N x Kp) through shared memory.  256 threads.
+__global__ void __launch_bounds__(256) split_ab(const float* __restrict__ A, float* __restrict__ ahi,
+                                                float* __restrict__ alo, const float* __restrict__ B,
+                                                float* __restrict__ bhi, float* __restrict__ blo, int64_t K,
+                                                int64_t N, int64_t Kp, int64_t r0, int64_t mrows, int nblk_a,
+                                                int ntn) {
   __shared__ float t[32][33];
-  const int64_t k0 = (int64_t)blockIdx.y * 32, n0 = (int64_t)blockIdx.x * 32;
-  for (int j = threadIdx.y; j < 32; j += blockDim.y) {
-    const int64_t k = k0 + j, n = n0 + threadIdx.x;
-    t[j][threadIdx.x] = (k < K && n < N) ? B[k * N + n] : 0.f;
+  if ((int)blockIdx.x < nblk_a) {
+    const int64_t stride = (int64_t)nblk_a * 256;
+    if (K == Kp && (K & 3) == 0) {
+      const float4* src = reinterpret_cast<const float4*>(A + r0 * K);
+      const int64_t n4 = mrows * K / 4;
+      for (int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x; i < n4; i += stride) {
+        const float4 x = src[i];
+        float4 h, l;
+        split2(x.x, h.x, l.x);
+        split2(x.y, h.y, l.y);
+        split2(x.z, h.z, l.z);
+        split2(x.w, h.w, l.w);
+        reinterpret_cast<float4*>(ahi)[i] = h;
+        reinterpret_cast<float4*>(alo)[i] = l;
+      }
+    } else {
+      const int64_t n = mrows * Kp;
+      for (int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x; i < n; i += stride) {
+        const int64_t r = i / Kp, k = i % Kp;
+        split2(k < K ? A[(r0 + r) * K + k] : 0.f, ahi[i], alo[i]);
+      }
+    }
+    return;
+  }
+  const int tb = (int)blockIdx.x - nblk_a;
+  const int64_t k0 = (int64_t)(tb / ntn) * 32, n0 = (int64_t)(tb % ntn) * 32;
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+#pragma unroll
+  for (int j = ty; j < 32; j += 8) {
+    const int64_t k = k0 + j, n = n0 + tx;
+    t[j][tx] = (k < K && n < N) ? B[k * N + n] : 0.f;
   }
   __syncthreads();
-  for (int j = threadIdx.y; j < 32; j += blockDim.y) {
-    const int64_t n = n0 + j, k = k0 + threadIdx.x;
-    if (n < N && k < Kp) {
-      const float x = t[threadIdx.x][j];
-      const float h = tf32_rn(x);
-      hi[n * Kp + k] = h;
-      lo[n * Kp + k] = tf32_rn(x - h);
-    }
+#pragma unroll
+  for (int j = ty; j < 32; j += 8) {
+    const int64_t n = n0 + j, k = k0 + tx;
+    if (n < N && k < Kp) split2(t[tx][j], bhi[n * Kp + k], blo[n * Kp + k]);
   }
 }
 
@@ -679,24 +700,31 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
   return cudaGetLastError();
 }
 
+
 namespace {
-// C[row0 + r][n] = ((p_0 + p_1) + ...) + p_{S-1}  (fixed split order)
-__global__ void split_k_reduce(const float* __restrict__ part, float* __restrict__ C, int64_t N, int64_t row0,
-                               int64_t mrows, int S) {
+// C[row0 + r][n] = ((p_0 + p_1) + ...) + p_{S-1}  (fixed split order; the S
+// loads of an element are issued before the adds)
+template <int S>
+__global__ void __launch_bounds__(256) split_k_reduce(const float* __restrict__ part, float* __restrict__ C, int64_t N,
+                                                      int64_t row0, int64_t mrows) {
   const int64_t stride = mrows * N;
   if ((N & 3) == 0) {
     const int64_t n4 = stride / 4;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
-      float4 a = reinterpret_cast<const float4*>(part)[i];
+      float4 v[S];
+#pragma unroll
+      for (int z = 0; z < S; ++z) v[z] = __ldcs(reinterpret_cast<const float4*>(part + z * stride) + i);
+      float4 a = v[0];
+#pragma unroll
       for (int z = 1; z < S; ++z) {
-        const float4 b = reinterpret_cast<const float4*>(part + z * stride)[i];
-        a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+        a.x += v[z].x; a.y += v[z].y; a.z += v[z].z; a.w += v[z].w;
       }
       reinterpret_cast<float4*>(C + row0 * N)[i] = a;
     }
   } else {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < stride; i += (int64_t)gridDim.x * blockDim.x) {
       float a = part[i];
+#pragma unroll
       for (int z = 1; z < S; ++z) a += part[z * stride + i];
       C[row0 * N + i] = a;
     }
@@ -736,16 +764,16 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   float* ahi = blo + N * Kp;
   float* alo = ahi + mrows * Kp;
   {
-    const int64_t n = mrows * Kp;
-    int64_t blocks = (n + 255) / 256;
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    split_rows<<<(unsigned)blocks, 256, 0, s>>>(A, ahi, alo, K, Kp, r0, mrows);
+    // one launch splits A's rows and (unless cached) B
+    const int64_t na = (K == Kp && (K & 3) == 0) ? mrows * K / 4 : mrows * Kp;
+    const int nblk_a = (int)std::min<int64_t>((na + 1023) / 1024, 148 * 8);
     // B is the same whole operand for every row range of this run: split it
     // once per run on this device (only if the app never writes it).
     const bool cached = b_readonly && scr->b_src == B && scr->b_K == K && scr->b_N == N && scr->b_epoch == scr->epoch;
+    const int ntn = (int)((N + 31) / 32);
+    const int64_t nblk_b = cached ? 0 : (int64_t)ntn * ((Kp + 31) / 32);
+    split_ab<<<(unsigned)(nblk_a + nblk_b), 256, 0, s>>>(A, ahi, alo, B, bhi, blo, K, N, Kp, r0, mrows, nblk_a, ntn);
     if (!cached) {
-      dim3 g((unsigned)((N + 31) / 32), (unsigned)((Kp + 31) / 32));
-      split_transpose<<<g, dim3(32, 8), 0, s>>>(B, bhi, blo, K, N, Kp);
       scr->b_src = b_readonly ? B : nullptr;
       scr->b_K = K;
       scr->b_N = N;
@@ -779,9 +807,10 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
         cudaSuccess)
       return e;
     const int64_t work = (N & 3) == 0 ? mrows * N / 4 : mrows * N;
-    int64_t blocks = (work + 255) / 256;
-    if (blocks > 148 * 8) blocks = 148 * 8;
-    split_k_reduce<<<(unsigned)blocks, 256, 0, s>>>(part, C, N, r0, mrows, S);
+    const unsigned blocks = (unsigned)std::min<int64_t>((work + 255) / 256, 148 * 8);
+    if (S == 2) split_k_reduce<2><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
+    else if (S == 3) split_k_reduce<3><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
+    else split_k_reduce<4><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
     return cudaGetLastError();
   }
   const bool narrow = ((mrows + BM - 1) / BM) * ((N + BN - 1) / BN) < cap;   // fewer 128x256 tiles than SMs

@@ -247,6 +247,28 @@ def test_sgemm(R, variant, G, shape):
             assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-4
 
 
+def test_sgemm_splitk_repeat_and_graph(R):
+    """Split-K SGEMM (1024^3: the last arrival per tile sums the K partials in
+    split order inside the GEMM) gives the same bits on every eager run and
+    every CUDA-graph replay of the same session (the arrival counters are
+    cleared by the last arrival; graph replays reuse the captured launch tag)."""
+    mm, runner = R
+    M = N = K = 1024
+    Au, Bu = synthgen.matmul_uniform(M, K, N)
+    ref = on.sgemm(Au, Bu)
+    outs = []
+    with runner.session(mm.MM_APP_SGEMM, [M, N, K, 2, 16, 1], G=1) as s:
+        s.fill(integer=False)
+        plan = s.plan(1, rand_profile(mm, 1, 1, 9))
+        for graph in (False, False, True, True, True, False):
+            s.bufs[(2, 0)].fill_(float("nan"))
+            s.run(plan, use_graph=graph)
+            outs.append(s.collect(plan, 2).reshape(M, N))
+    assert np.max(np.abs(outs[0] - ref) / np.abs(ref)) <= 1e-4
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0])
+
+
 def test_stream_full_size_sampled(R):
     """BASELINE configs[1] size (2^28) in the bench's launch configuration
     (1 logical device, SP-Unified, CUDA graph): sampled outputs vs the oracle
