@@ -25,6 +25,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <utility>
 #include <vector>
 
 #include "kernels.h"
@@ -243,6 +244,11 @@ __device__ __forceinline__ void gemm_body(const CUtensorMap& tAhi, const CUtenso
   if (PAIR) cluster_sync_all();   // both CTAs' barriers initialised before any cross-CTA traffic
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tslot;
+  // programmatic dependent launch (SGEMM chain): the set-up above overlaps the
+  // producer kernel's tail; no global access before its results are visible.
+  // No-ops when launched without the PDL attribute (the Cholesky launches).
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
   if (warp == 0) {
     if (lane == 0) {  // ===== TMA producer (both CTAs in PAIR mode)
@@ -443,6 +449,7 @@ __global__ void __launch_bounds__(256) split_ab(const float* __restrict__ A, flo
                                                 int64_t N, int64_t Kp, int64_t r0, int64_t mrows, int nblk_a,
                                                 int ntn) {
   __shared__ float t[32][33];
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");   // the GEMM may start its set-up
   if ((int)blockIdx.x < nblk_a) {
     const int64_t stride = (int64_t)nblk_a * 256;
     if (K == Kp && (K & 3) == 0) {
@@ -535,6 +542,24 @@ cudaError_t set_gemm_smem() {
   });
 }
 
+// Launch with programmatic stream serialization (PDL): the kernel may start
+// while the previous kernel on the stream finishes; it orders itself with
+// griddepcontrol.wait.
+template <typename... P, typename... A>
+cudaError_t launch_pdl(void (*kern)(P...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, A&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<A>(args)...);
+}
+
 // 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0
 // turns it off).
 // The 128x64 narrow tiles of small SGEMMs stay single-SM (measured faster).
@@ -551,7 +576,7 @@ bool use_mc(const GemmJob& job, int bn = BN) { return use_mc_env() && bn == BN &
 template <int BN_>
 cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, const CUtensorMap& tb_hi,
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
-                        const GemmJob& job, int cap, cudaStream_t s) {
+                        const GemmJob& job, int cap, cudaStream_t s, bool pdl = false) {
   const bool mc = use_mc(job, BN_);
   const int ntiles = job.mblk * job.nblk * (job.mode >= 1 ? job.n : 1);
   if (ntiles <= 0) return cudaSuccess;
@@ -560,9 +585,15 @@ cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, cons
   int grid;
   if (cap > 0) grid = std::min(units, mc ? cap / 2 : cap);
   else grid = std::max(std::min(units, slots), (units + 3) / 4);
+  if (mc && pdl)
+    return launch_pdl(gemm_tf32x3_pair<BN_>, dim3(2 * grid), dim3(kThreadsGemm), gemm_smem<BN_, true>(), s, ta_hi,
+                      ta_lo, tb_hi, tb_lo, C, N, row0, mrows, nkb, units, job);
   if (mc)
     gemm_tf32x3_pair<BN_><<<2 * grid, kThreadsGemm, gemm_smem<BN_, true>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N,
                                                                                row0, mrows, nkb, units, job);
+  else if (pdl)
+    return launch_pdl(gemm_tf32x3<BN_>, dim3(grid), dim3(kThreadsGemm), gemm_smem<BN_, false>(), s, ta_hi, ta_lo,
+                      tb_hi, tb_lo, C, N, row0, mrows, nkb, units, job);
   else
     gemm_tf32x3<BN_><<<grid, kThreadsGemm, gemm_smem<BN_, false>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0,
                                                                          mrows, nkb, units, job);
@@ -707,6 +738,7 @@ namespace {
 template <int S>
 __global__ void __launch_bounds__(256) split_k_reduce(const float* __restrict__ part, float* __restrict__ C, int64_t N,
                                                       int64_t row0, int64_t mrows) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");   // PDL: the GEMM's partials are complete
   const int64_t stride = mrows * N;
   if ((N & 3) == 0) {
     const int64_t n4 = stride / 4;
@@ -803,15 +835,14 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
     job.ncols = BN;
     job.mblk = probe.mblk;
     job.nblk = (int32_t)((N + BN - 1) / BN);
-    if ((e = launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, part, N, 0, mrows, (int)(Kp / S / BK), job, cap, s)) !=
-        cudaSuccess)
+    if ((e = launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, part, N, 0, mrows, (int)(Kp / S / BK), job, cap, s,
+                             true)) != cudaSuccess)
       return e;
     const int64_t work = (N & 3) == 0 ? mrows * N / 4 : mrows * N;
-    const unsigned blocks = (unsigned)std::min<int64_t>((work + 255) / 256, 148 * 8);
-    if (S == 2) split_k_reduce<2><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
-    else if (S == 3) split_k_reduce<3><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
-    else split_k_reduce<4><<<blocks, 256, 0, s>>>(part, C, N, r0, mrows);
-    return cudaGetLastError();
+    const dim3 blocks((unsigned)std::min<int64_t>((work + 255) / 256, 148 * 8));
+    if (S == 2) return launch_pdl(split_k_reduce<2>, blocks, dim3(256), 0, s, (const float*)part, C, N, r0, mrows);
+    if (S == 3) return launch_pdl(split_k_reduce<3>, blocks, dim3(256), 0, s, (const float*)part, C, N, r0, mrows);
+    return launch_pdl(split_k_reduce<4>, blocks, dim3(256), 0, s, (const float*)part, C, N, r0, mrows);
   }
   const bool narrow = ((mrows + BM - 1) / BM) * ((N + BN - 1) / BN) < cap;   // fewer 128x256 tiles than SMs
   const uint32_t bn = narrow ? 64 : BN;
@@ -829,8 +860,8 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
   job.ncols = BN;
   job.mblk = (int32_t)((mrows + BM - 1) / BM);
   job.nblk = (int32_t)((N + bn - 1) / bn);
-  if (narrow) return launch_gemm<64>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s);
-  return launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s);
+  if (narrow) return launch_gemm<64>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s, true);
+  return launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, r0, mrows, (int)(Kp / BK), job, cap, s, true);
   return cudaGetLastError();
 }
 
