@@ -247,6 +247,30 @@ def test_sgemm(R, variant, G, shape):
             assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-4
 
 
+@pytest.mark.parametrize("strategy", [4, 5, 7])
+@pytest.mark.parametrize("shape", [(520, 300, 77), (1024, 512, 256)])
+def test_sgemm_dp_chunks(R, strategy, shape):
+    """DP-Perf / DP-Dep / DP-Static chunk the rows of one SGEMM over 2 logical
+    devices: every chunk after a device's first reuses that device's cached
+    B split (the split launch then covers A only); ragged K exercises the
+    scalar split path.  Integer inputs: bit-exact; uniform: 1e-4."""
+    mm, runner = R
+    M, N, K = shape
+    for integer in (True, False):
+        A, B = (synthgen.matmul_integer if integer else synthgen.matmul_uniform)(M, K, N)
+        ref = on.sgemm(A, B)
+        with runner.session(mm.MM_APP_SGEMM, [M, N, K, 2, 16, 1], G=2) as s:
+            s.fill(integer=integer)
+            plan = s.plan(strategy, rand_profile(mm, 2, 1, 5), chunks_per_dev=4)
+            s.run(plan)
+            s.run(plan)
+            got = s.collect(plan, 2).reshape(M, N)
+        if integer:
+            assert np.array_equal(got, ref)
+        else:
+            assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-4
+
+
 def test_sgemm_splitk_repeat_and_graph(R):
     """Split-K SGEMM (1024^3: the last arrival per tile sums the K partials in
     split order inside the GEMM) gives the same bits on every eager run and
