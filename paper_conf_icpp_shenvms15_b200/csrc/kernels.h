@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <atomic>
 #include <cstdint>
+#include <utility>
 #include <vector>
 
 namespace mm {
@@ -21,6 +22,24 @@ cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
   e = set();
   if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
   return e;
+}
+
+// Launch with programmatic stream serialization (PDL): the kernel may start
+// while the previous kernel on the stream finishes; it orders itself with
+// griddepcontrol.wait.
+template <typename... P, typename... A>
+cudaError_t launch_pdl(void (*kern)(P...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, A&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<A>(args)...);
 }
 
 struct Kernel;
@@ -97,7 +116,8 @@ cudaError_t chol_trsm_prepare(float* A, int64_t T, int64_t b, int32_t k, cudaStr
                               float** hi, float** lo, int32_t* slot0);
 void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, int32_t n);
 cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n,
-                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr);
+                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr,
+                                bool pdl = false);   // pdl: launched as a programmatic dependent of a leaf
 
 // Nbody step for bodies [r0, r1) (kernels_nbody.cu); float4 bodies.
 cudaError_t nbody_rows_launch(const float* pin, const float* vin, float* pout, float* vout, int64_t n, int64_t r0,

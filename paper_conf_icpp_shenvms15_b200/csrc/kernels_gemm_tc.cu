@@ -25,7 +25,6 @@
 
 #include <algorithm>
 #include <cstdlib>
-#include <utility>
 #include <vector>
 
 #include "kernels.h"
@@ -542,24 +541,6 @@ cudaError_t set_gemm_smem() {
   });
 }
 
-// Launch with programmatic stream serialization (PDL): the kernel may start
-// while the previous kernel on the stream finishes; it orders itself with
-// griddepcontrol.wait.
-template <typename... P, typename... A>
-cudaError_t launch_pdl(void (*kern)(P...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, A&&... args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, kern, std::forward<A>(args)...);
-}
-
 // 2-SM pairs (cta_group::2) when the task's m-blocks pair up (MM_GEMM_PAIR=0
 // turns it off).
 // The 128x64 narrow tiles of small SGEMMs stay single-SM (measured faster).
@@ -701,7 +682,7 @@ void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, i
 // TRSM block update over a batch: columns [n0, b) of tiles (ti[q], k) -=
 // X_i[:, kx0:kx0+K] L_kk[n0:b, kx0:kx0+K]^T (3xTF32, split operands in slots).
 cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n,
-                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr) {
+                                int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr, bool pdl) {
   if (n <= 0 || n0 >= b) return cudaSuccess;
   CUtensorMap ta_hi, ta_lo, tb_hi, tb_lo;
   cudaError_t e;
@@ -726,7 +707,8 @@ cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const
     }
     job.mblk = (int32_t)(b / BM);
     job.nblk = (int32_t)((b - n0 + BN - 1) / BN);
-    launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job, 0, s);
+    if ((e = launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, K / BK, job, 0, s, pdl)) != cudaSuccess)
+      return e;
   }
   return cudaGetLastError();
 }
