@@ -42,7 +42,7 @@ cudaError_t chol_trsm_prepare(float*, int64_t, int64_t, int32_t, cudaStream_t, S
 }
 void chol_mark_split(Scratch*, int64_t, int32_t, const int32_t*, int32_t) {}
 cudaError_t chol_trsm_update_tc(float*, int64_t, int64_t, int32_t, const int32_t*, int32_t, int32_t, int32_t, int32_t,
-                                cudaStream_t, Scratch*) {
+                                cudaStream_t, Scratch*, bool) {
   return cudaErrorNotSupported;
 }
 }  // namespace mm
