@@ -180,6 +180,14 @@ mm_status mm_app_set_lane(mm_app* app, int32_t kernel, int32_t lane);
 mm_status mm_app_set_unstable(mm_app* app, int32_t unstable);
 /* Explicit task (MK-DAG).  Tasks are kept in creation order. */
 mm_status mm_app_add_task(mm_app* app, const mm_task_desc* task);
+/* Freeze the description of an app (P53 §III-A: "an application ... its
+ * kernels and execution flow" is the input of the method).
+ * Validates what the single calls cannot (>= 1 kernel, no loop over an
+ * explicit-task DAG, every reference in range) and makes every later
+ * mm_app_add_* / mm_app_set_* call on this app return MM_ESTATE.  Optional:
+ * classify / split / plan also accept an unfinalized app.  Idempotent.
+ * Errors: MM_EINVAL (null or invalid description; the app stays mutable). */
+mm_status mm_app_finalize(mm_app* app);
 
 /* Built-in apps of the paper (Table II) and of BASELINE.json configs. */
 typedef enum {
@@ -317,6 +325,25 @@ void      mm_ctx_destroy(mm_ctx* ctx);
 mm_status mm_ctx_stream(mm_ctx* ctx, int32_t d, void** stream);
 /* SMs actually granted to logical device d. */
 mm_status mm_ctx_sm_count(mm_ctx* ctx, int32_t d, int32_t* sms);
+/* PyTorch stream interop (SURVEY §8(b) mm_ctx_set_stream): order the runs of
+ * logical device d with a caller stream (e.g. torch.cuda.current_stream()
+ * .cuda_stream).  mm_run then makes all of d's library streams wait for the
+ * work already enqueued on `stream`, and `stream` wait for the run's last
+ * kernel, so caller kernels before / after mm_run see its inputs / results
+ * without a host synchronisation.  The stream stays caller-owned (never
+ * destroyed by the library); NULL clears it.  Errors: MM_EINVAL (bad device
+ * or a device another rank owns), MM_ESTATE (poisoned ctx). */
+mm_status mm_ctx_set_stream(mm_ctx* ctx, int32_t d, void* stream);
+/* Register one app buffer (SURVEY §8(b) mm_buffer_register): dev_ptrs[G] are
+ * caller-owned device pointers of elem_bytes x n_elems, one full-size copy per
+ * logical device (NULL for devices another rank owns); never freed by the
+ * library.  The i-th registration stands for app buffer slot i: mm_run and
+ * mm_collect called with buffers == NULL use the registered pointers, after
+ * checking that every slot's element size and length match the plan's app.
+ * Errors: MM_EINVAL (null / missing pointer of an owned device, bad size,
+ * more than MM_MAX_BUF buffers), MM_ENOMEM. */
+mm_status mm_buffer_register(mm_ctx* ctx, int32_t elem_bytes, int64_t n_elems, void* const* dev_ptrs,
+                             int32_t* buf_id);
 
 /* Device generator = synthgen.uniform (counter hash):
  * x[i] = lo + (hi-lo)*u(seed, array_id, start+i) for i in [0,n) into the
@@ -385,7 +412,9 @@ typedef struct {
 } mm_run_stats;
 
 /* Execute the plan's op program (blocking: returns when this process's
- * devices are done).  buffers as in mm_profile_run. */
+ * devices are done).  buffers as in mm_profile_run, or NULL for the buffers
+ * registered with mm_buffer_register; runs are ordered with the streams set
+ * by mm_ctx_set_stream. */
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan, void* const* buffers, const mm_run_opts* opts,
                  mm_run_stats* stats);
 
@@ -408,7 +437,8 @@ mm_status mm_run_decisions(const mm_plan* plan, mm_decision* out, int64_t cap, i
 
 /* Assemble buffer `slot` after a run: every element range is copied from the
  * device that holds its final value into `dst` (device memory of logical
- * device `dst_device`, or host memory if dst_device < 0).  In-process only. */
+ * device `dst_device`, or host memory if dst_device < 0).  In-process only.
+ * buffers == NULL: the registered buffers (mm_buffer_register). */
 mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan, void* const* buffers, int32_t slot,
                      void* dst, int32_t dst_device);
 

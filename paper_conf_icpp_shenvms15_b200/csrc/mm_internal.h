@@ -120,5 +120,8 @@ void plan_runtime_free(Plan* plan);
 
 }  // namespace mm
 
-struct mm_app { mm::App a; };
+struct mm_app {
+  mm::App a;
+  bool frozen = false;   // mm_app_finalize: no further mutation
+};
 struct mm_plan { mm::Plan p; };

@@ -148,6 +148,12 @@ struct mm_ctx {
   float* bar_buf = nullptr;        // NCCL barrier scratch (1 float)
   std::vector<void*> flush_scratch;  // per buffer slot, pinned (lazily)
   std::vector<size_t> flush_scratch_bytes;
+  // mm_buffer_register: caller-owned per-device pointers, slot = registration order
+  std::vector<std::vector<void*>> reg;
+  std::vector<std::pair<int32_t, int64_t>> reg_shape;
+  // mm_ctx_set_stream: caller streams the runs of a device are ordered with
+  std::vector<cudaStream_t> ext;
+  std::vector<cudaEvent_t> ext_ev;
 };
 
 namespace {
@@ -1211,6 +1217,8 @@ void mm_ctx_destroy(mm_ctx* ctx) {
       else cudaStreamDestroy(st);
     }
     if (r.scr.ptr) cudaFree(r.scr.ptr);
+    const size_t d = (size_t)(&r - ctx->dev.data());
+    if (d < ctx->ext_ev.size() && ctx->ext_ev[d]) cudaEventDestroy(ctx->ext_ev[d]);
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);
   }
   if (ctx->comm) nccl().CommDestroy(ctx->comm);
@@ -1230,6 +1238,37 @@ mm_status mm_ctx_stream(mm_ctx* ctx, int32_t d, void** stream) {
 mm_status mm_ctx_sm_count(mm_ctx* ctx, int32_t d, int32_t* sms) {
   if (!ctx || !sms || d < 0 || d >= ctx->G) MM_FAIL(MM_EINVAL, "ctx_sm_count: bad arguments");
   *sms = ctx->dev[d].sms;
+  return MM_OK;
+}
+
+mm_status mm_ctx_set_stream(mm_ctx* ctx, int32_t d, void* stream) {
+  if (!ctx || d < 0 || d >= ctx->G) MM_FAIL(MM_EINVAL, "ctx_set_stream: bad arguments");
+  if (!ctx->dev[d].mine) MM_FAIL(MM_EINVAL, "ctx_set_stream: device %d not owned by this rank", d);
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  if (ctx->ext.size() != (size_t)ctx->G) {
+    ctx->ext.assign((size_t)ctx->G, nullptr);
+    ctx->ext_ev.assign((size_t)ctx->G, nullptr);
+  }
+  ctx->ext[d] = static_cast<cudaStream_t>(stream);
+  return MM_OK;
+}
+
+mm_status mm_buffer_register(mm_ctx* ctx, int32_t elem_bytes, int64_t n_elems, void* const* dev_ptrs,
+                             int32_t* buf_id) {
+  if (!ctx || !dev_ptrs || !buf_id) MM_FAIL(MM_EINVAL, "buffer_register: null argument");
+  if (!(elem_bytes == 1 || elem_bytes == 2 || elem_bytes == 4 || elem_bytes == 8) || n_elems < 0)
+    MM_FAIL(MM_EINVAL, "buffer_register: elem_bytes %d n %lld", elem_bytes, (long long)n_elems);
+  if ((int32_t)ctx->reg.size() >= MM_MAX_BUF) MM_FAIL(MM_EINVAL, "buffer_register: too many buffers");
+  for (int32_t d = 0; d < ctx->G; ++d)
+    if (ctx->dev[d].mine && n_elems > 0 && !dev_ptrs[d])
+      MM_FAIL(MM_EINVAL, "buffer_register: no pointer for owned device %d", d);
+  try {
+    ctx->reg.emplace_back(dev_ptrs, dev_ptrs + ctx->G);
+    ctx->reg_shape.push_back({elem_bytes, n_elems});
+  } catch (...) {
+    MM_FAIL(MM_ENOMEM, "buffer_register: out of host memory");
+  }
+  *buf_id = (int32_t)ctx->reg.size() - 1;
   return MM_OK;
 }
 
@@ -1266,8 +1305,49 @@ mm_status mm_fill_spd_tiles(mm_ctx* ctx, int32_t d, float* dst, int64_t n, int64
   return MM_OK;
 }
 
+namespace {
+// buffers == NULL: the registered buffers (slot i = i-th registration), which
+// must match the plan's buffer shapes
+mm_status resolve_buffers(mm_ctx* ctx, const Plan& plan, void* const*& buffers, std::vector<void*>& tmp) {
+  if (buffers) return MM_OK;
+  const size_t nb = plan.app.buffers.size();
+  if (ctx->reg.size() < nb) MM_FAIL(MM_EINVAL, "run: %zu buffers registered, the app has %zu", ctx->reg.size(), nb);
+  tmp.assign(nb * (size_t)ctx->G, nullptr);
+  for (size_t i = 0; i < nb; ++i) {
+    if (ctx->reg_shape[i] != plan.app.buffers[i])
+      MM_FAIL(MM_EINVAL, "run: registered buffer %zu (%d B x %lld) differs from app slot %zu", i,
+              ctx->reg_shape[i].first, (long long)ctx->reg_shape[i].second, i);
+    for (int32_t d = 0; d < ctx->G; ++d) tmp[i * (size_t)ctx->G + d] = ctx->reg[i][(size_t)d];
+  }
+  buffers = tmp.data();
+  return MM_OK;
+}
+
+// mm_ctx_set_stream: order device d's streams after the work already on the
+// caller's stream (before), or the caller's stream after the run (after)
+mm_status join_external(mm_ctx* ctx, bool before) {
+  for (int32_t d = 0; d < (int32_t)ctx->ext.size(); ++d) {
+    if (!ctx->ext[d] || !ctx->dev[d].mine) continue;
+    DevRt& r = ctx->dev[d];
+    CU_OK(set_dev(ctx, d));
+    if (!ctx->ext_ev[d]) CU_OK(cudaEventCreateWithFlags(&ctx->ext_ev[d], cudaEventDisableTiming));
+    if (before) {
+      CU_OK(cudaEventRecord(ctx->ext_ev[d], ctx->ext[d]));
+      for (cudaStream_t st : {r.stream, r.h2d, r.d2h, r.lane1})
+        if (st) CU_OK(cudaStreamWaitEvent(st, ctx->ext_ev[d], 0));
+    } else {
+      CU_OK(cudaEventRecord(ctx->ext_ev[d], r.stream));
+      CU_OK(cudaStreamWaitEvent(ctx->ext[d], ctx->ext_ev[d], 0));
+    }
+  }
+  return MM_OK;
+}
+}  // namespace
+
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_run_opts* o, mm_run_stats* st) {
-  if (!ctx || !plan_h || !buffers) MM_FAIL(MM_EINVAL, "run: null argument");
+  if (!ctx || !plan_h) MM_FAIL(MM_EINVAL, "run: null argument");
+  std::vector<void*> reg_bufs;
+  if (mm_status rb = resolve_buffers(ctx, plan_h->p, buffers, reg_bufs)) return rb;
   if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
   Plan& plan = plan_h->p;
   if (plan.G != ctx->G) MM_FAIL(MM_EINVAL, "run: plan has G=%d, ctx has G=%d", plan.G, ctx->G);
@@ -1278,6 +1358,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   const bool graph = o && o->use_graph && !timing && ctx->world == 1;
   mm_status r = ensure_rt(ctx, plan, timing);
   if (r) return r;
+  if ((r = join_external(ctx, true))) return r;
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
   for (auto& dv : ctx->dev) dv.scr.epoch++;   // operand-split caches are per run
   const int32_t root = first_owned(ctx);
@@ -1350,6 +1431,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   }
   CU_OK(cudaEventSynchronize(rt->t_stop));
   auto t1 = std::chrono::steady_clock::now();
+  if ((r = join_external(ctx, false))) return r;
   S->wall_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
   float ms = 0.f;
   CU_OK(cudaEventElapsedTime(&ms, rt->t_start, rt->t_stop));
@@ -1436,7 +1518,9 @@ mm_status mm_tune_chunks(mm_ctx* ctx, const mm_app* app, const mm_profile* prof,
 
 mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan_h, void* const* buffers, int32_t slot, void* dst,
                      int32_t dst_device) {
-  if (!ctx || !plan_h || !buffers || !dst) MM_FAIL(MM_EINVAL, "collect: null argument");
+  if (!ctx || !plan_h || !dst) MM_FAIL(MM_EINVAL, "collect: null argument");
+  std::vector<void*> reg_bufs;
+  if (mm_status rb = resolve_buffers(ctx, plan_h->p, buffers, reg_bufs)) return rb;
   const PlanRt* prt = static_cast<const PlanRt*>(plan_h->p.rt);
   const Plan& plan = (prt && prt->last_adaptive && prt->ad) ? prt->ad->ap : plan_h->p;
   if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "collect: in-process contexts only");

@@ -179,6 +179,9 @@ _SIGS = {
     "mm_ctx_create": [C.POINTER(mm_device_spec), C.c_int32, C.c_int32, C.c_int32, C.c_void_p, C.POINTER(_P)],
     "mm_ctx_stream": [_P, C.c_int32, C.POINTER(_P)],
     "mm_ctx_sm_count": [_P, C.c_int32, C.POINTER(C.c_int32)],
+    "mm_ctx_set_stream": [_P, C.c_int32, C.c_void_p],
+    "mm_buffer_register": [_P, C.c_int32, C.c_int64, C.POINTER(_P), C.POINTER(C.c_int32)],
+    "mm_app_finalize": [_P],
     "mm_fill_uniform": [_P, C.c_int32, C.c_void_p, C.c_int64, C.c_uint64, C.c_int32, C.c_int64, C.c_float,
                         C.c_float],
     "mm_fill_integers": [_P, C.c_int32, C.c_void_p, C.c_int64, C.c_uint64, C.c_int32, C.c_int64, C.c_int32,
@@ -487,6 +490,22 @@ def mm_ctx_sm_count(ctx: int, d: int) -> int:
     return s.value
 
 
+def mm_ctx_set_stream(ctx: int, d: int, stream: int):
+    """Order device d's runs with a caller stream (torch ``Stream.cuda_stream``); 0 clears it."""
+    _call("mm_ctx_set_stream", ctx, d, stream or None)
+
+
+def mm_buffer_register(ctx: int, elem_bytes: int, n_elems: int, dev_ptrs: Sequence[int]) -> int:
+    """Register app buffer slot i (i-th call): one caller-owned device pointer per logical device."""
+    b = C.c_int32()
+    _call("mm_buffer_register", ctx, elem_bytes, n_elems, _ptr_array(dev_ptrs), C.byref(b))
+    return b.value
+
+
+def mm_app_finalize(app: int):
+    _call("mm_app_finalize", app)
+
+
 def mm_fill_uniform(ctx: int, d: int, ptr: int, n: int, seed: int, array_id: int, start: int,
                     lo: float, hi: float):
     _call("mm_fill_uniform", ctx, d, ptr, n, seed, array_id, start, lo, hi)
@@ -513,7 +532,7 @@ def mm_profile_run(ctx: int, app: int, buffers: Sequence[int], reps: int = 5, dp
     return p
 
 
-def mm_run(ctx: int, plan: int, buffers: Sequence[int], use_graph: bool = False, time_kernels: bool = False,
+def mm_run(ctx: int, plan: int, buffers: Optional[Sequence[int]], use_graph: bool = False, time_kernels: bool = False,
            host: Optional[Sequence[int]] = None, adaptive: bool = False, max_inflight: int = 0) -> mm_run_stats:
     o = mm_run_opts()
     o.use_graph = int(use_graph)
@@ -524,7 +543,7 @@ def mm_run(ctx: int, plan: int, buffers: Sequence[int], use_graph: bool = False,
         harr = _ptr_array(host)
         o.host = C.cast(harr, C.POINTER(C.c_void_p))
     st = mm_run_stats()
-    _call("mm_run", ctx, plan, _ptr_array(buffers), C.byref(o), C.byref(st))
+    _call("mm_run", ctx, plan, None if buffers is None else _ptr_array(buffers), C.byref(o), C.byref(st))
     return st
 
 
@@ -547,8 +566,8 @@ def mm_run_decisions(plan: int) -> List[mm_decision]:
     return list(out[:n.value])
 
 
-def mm_collect(ctx: int, plan: int, buffers: Sequence[int], slot: int, dst: int, dst_device: int = -1):
-    _call("mm_collect", ctx, plan, _ptr_array(buffers), slot, dst, dst_device)
+def mm_collect(ctx: int, plan: int, buffers: Optional[Sequence[int]], slot: int, dst: int, dst_device: int = -1):
+    _call("mm_collect", ctx, plan, None if buffers is None else _ptr_array(buffers), slot, dst, dst_device)
 
 
 def mm_kernel_launch_count() -> int:
