@@ -259,6 +259,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
     ap.add_argument("--no-profile", action="store_true",
                     help="use an equal synthetic profile instead of measuring one (ncu runs)")
+    ap.add_argument("--kernel-timing", default="last", choices=["all", "last", "none"],
+                    help="per-kernel CUDA events in the timed steps: every step, the last ceil(K/5) steps, or none")
     ap.add_argument("--logical", type=int, default=0,
                     help="virtual mode: run G logical devices on this one GPU (G = --logical)")
     args = ap.parse_args()
@@ -316,26 +318,49 @@ def main():
             mm.mm_split(sess.app, prof, best)
         return sess.run(p, **kw)
 
+    # MK-DAG factors A in place: every step starts from the same SPD matrix,
+    # restored from a pristine copy between steps, outside the timed spans
+    # (each step is then bracketed by its own barrier + synchronize); the
+    # other apps' steps are timed back to back
+    pristine = {}
+    if args.app == "cholesky":
+        pristine = {d: sess.bufs[(0, d)].clone() for d in range(G) if sess.mine[d]}
+
+    def restore():
+        for d, t in pristine.items():
+            sess.bufs[(0, d)].copy_(t)
+        if pristine:
+            torch.cuda.synchronize()
+
     for _ in range(args.warmup):
+        restore()
         step(plan, time_kernels=True)
     barrier()
     l0 = mm.mm_kernel_launch_count()
     stream = sess.stream(rank if world > 1 else 0)
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     kms = [[0.0] * K for _ in range(G)]
     launches = 0
+    spans = []
+    n_last = max(1, (args.steps + 4) // 5)   # --kernel-timing last: the last ceil(K/5) timed steps
     with ClockSampler(local) as clk:
-        barrier()
-        ev0.record(stream)
-        for _ in range(args.steps):
-            st = step(plan, time_kernels=True)
+        for i in range(args.steps):
+            if pristine or i == 0:
+                restore()
+                barrier()
+                ev0 = torch.cuda.Event(enable_timing=True)
+                ev0.record(stream)
+            kt = args.kernel_timing == "all" or (args.kernel_timing == "last" and i >= args.steps - n_last)
+            st = step(plan, time_kernels=kt)
             for d in range(G):
                 for k in range(K):
                     kms[d][k] += st.kernel_ms[d][k]
             launches += st.n_launches
-        ev1.record(stream)
-        barrier()
-    ms_total = ev0.elapsed_time(ev1)
+            if pristine or i == args.steps - 1:
+                ev1 = torch.cuda.Event(enable_timing=True)
+                ev1.record(stream)
+                barrier()
+                spans.append((ev0, ev1))
+    ms_total = sum(a.elapsed_time(b) for a, b in spans)
     gpu_launches = mm.mm_kernel_launch_count() - l0
     if world > 1:
         t = torch.tensor([ms_total], dtype=torch.float64)
@@ -361,20 +386,21 @@ def main():
     kid = kname_map.index(dom)
     my = [d for d in range(G) if sess.mine[d]]
     dom_ms = sum(kms[d][kid] for d in my)
-    dom_launch = sum(st.kernel_launches[d][kid] for d in my) * args.steps
+    timed_steps = {"all": args.steps, "last": n_last, "none": 0}[args.kernel_timing]
+    dom_launch = sum(st.kernel_launches[d][kid] for d in my) * timed_steps
     items = sum(info.items[d][kid] for d in my)
     if bpi is None:
         bpi = {"hotspot": 12 * iparam[1], "stencil": 12 * iparam[1]}.get(args.app)
     roof = None
     if dom_launch and dom_ms > 0:
         per_launch_ms = dom_ms / dom_launch
-        launches_per_step = dom_launch / args.steps
+        launches_per_step = dom_launch / timed_steps
         if args.app == "nbody":
             # FP32-pipe-bound all-pairs: 20 flop per interaction (usual count);
             # the kernel needs 12 FP32 lane-ops per interaction, so the ceiling
             # is 148 SMs x 128 lanes x 1.965 GHz / 12 interactions/s x 20 flop
             n_b = iparam[0]
-            ach = 20 * n_b * items * args.steps / (dom_ms * 1e-3) / 1e12
+            ach = 20 * n_b * items * timed_steps / (dom_ms * 1e-3) / 1e12
             pk = 148 * 128 * 1.965e9 / 12 * 20 / 1e12
             roof = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
                     "traffic": None, "kernel": "nbody (all pairs, smem tiles, 2 bodies/thread in f32x2)",
@@ -386,7 +412,7 @@ def main():
             # (the step runs ~75 ms back to back under the power cap, so the
             # denominator is the sustained figure; burst reported beside it)
             b = iparam[1]
-            ach = 2 * b ** 3 * items * args.steps / (dom_ms * 1e-3) / 1e12
+            ach = 2 * b ** 3 * items * timed_steps / (dom_ms * 1e-3) / 1e12
             sus, sus_kind = load_sustained_bf16()
             burst = tf_peak * 0.5 / 3.0
             pk = sus * 0.5 / 3.0 if sus else burst
@@ -451,17 +477,26 @@ def main():
         for s in range(nbuf):
             eb, n = mm.mm_app_buffer_info(sess.app, s)
             h = torch.empty(max(n, 1), dtype=runner._DT[eb], pin_memory=True)
-            h.copy_(sess.bufs[(s, my[0])].cpu()) if n <= (1 << 29) else None
+            src = pristine[my[0]] if (s == 0 and pristine) else sess.bufs[(s, my[0])]
+            if n <= (1 << 29) or pristine:
+                h[:n].copy_(src[:n])
             host.append(h)
+
+        def restore_host():   # MK-DAG: the staged run writes L back over host A
+            if pristine:
+                host[0].copy_(pristine[my[0]])
+                torch.cuda.synchronize()
         # staged pipeline (R24): sub-chunks overlap H2D, kernels and D2H on
         # separate streams (applies to pointwise apps; ignored otherwise)
         splan = sess.plan(best, prof, staged=True, pipeline=args.pipeline)
+        restore_host()
         step(splan, host=[h.data_ptr() for h in host])  # warm-up
         barrier()
         e0 = time.perf_counter()
         tot = []
         hb = db = 0
         for _ in range(max(1, min(args.steps, 5))):
+            restore_host()
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             st = step(splan, host=[h.data_ptr() for h in host])
@@ -492,16 +527,22 @@ def main():
         for s_id in list(ranked) + [x for x in extras if x not in ranked]:
             try:
                 p = sess.plan(s_id, prof)
+                restore()
                 step(p)
                 barrier()
                 ts = []
                 for _ in range(3):
+                    restore()
                     st = sess.run(p)
                     ts.append(st.device_ms)
                 ms = statistics.median(ts)
                 if world == 1:   # the same op program captured once and replayed as a CUDA graph
+                    restore()
                     sess.run(p, use_graph=True)
-                    tg = [sess.run(p, use_graph=True).device_ms for _ in range(3)]
+                    tg = []
+                    for _ in range(3):
+                        restore()
+                        tg.append(sess.run(p, use_graph=True).device_ms)
                     strategies_graph[mm.mm_strategy_name(s_id)] = round(statistics.median(tg), 4)
                 if world > 1:
                     t = torch.tensor([ms], dtype=torch.float64)
@@ -523,11 +564,14 @@ def main():
             "config": {"workload": APPS[args.app][3], "app": args.app, "class": mm.mm_class_name(cls),
                        "strategy": mm.mm_strategy_name(best), "logical_devices": G,
                        "l2": "inputs larger than L2 (1 GiB arrays); no flush",
+                       "kernel_timing": {"all": "per-kernel CUDA events in every timed step",
+                                         "last": f"per-kernel CUDA events in the last {n_last} of {args.steps} timed steps",
+                                         "none": "no per-kernel events"}[args.kernel_timing],
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
                        **({"temporal_block": tb} if args.app == "hotspot" else {})},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
             "clocks": clk.summary(), "strategies_ms": strategies, "strategies_graph_ms": strategies_graph,
-            "kernel_ms_per_step": {kname_map[k]: round(sum(kms[d][k] for d in my) / args.steps, 4)
+            "kernel_ms_per_step": {kname_map[k]: round(sum(kms[d][k] for d in my) / max(1, timed_steps), 4)
                                    for k in range(K)},
             "ranking": [mm.mm_strategy_name(s) for s in ranked],
         }
