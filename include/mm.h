@@ -340,6 +340,8 @@ mm_status mm_ctx_set_stream(mm_ctx* ctx, int32_t d, void* stream);
  * library.  The i-th registration stands for app buffer slot i: mm_run and
  * mm_collect called with buffers == NULL use the registered pointers, after
  * checking that every slot's element size and length match the plan's app.
+ * Registrations last for the ctx's lifetime (extra registrations beyond the
+ * app's buffer count are ignored by its runs).
  * Errors: MM_EINVAL (null / missing pointer of an owned device, bad size,
  * more than MM_MAX_BUF buffers), MM_ENOMEM. */
 mm_status mm_buffer_register(mm_ctx* ctx, int32_t elem_bytes, int64_t n_elems, void* const* dev_ptrs,
