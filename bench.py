@@ -273,6 +273,20 @@ def main():
     from paper_conf_icpp_shenvms15_b200 import mm, runner
 
     world, rank, local = dist_env()
+    if args.gpus > 1 and world == 1:
+        # --gpus N without a launcher: one rank per GPU needs N visible GPUs;
+        # never time fewer GPUs than asked for (exit non-zero instead)
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print(json.dumps({"error": f"--gpus {args.gpus} but only {have} CUDA device(s) visible",
+                              "n_gpus": have}), flush=True)
+            sys.exit(2)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(29500 + os.getpid() % 1000)] + sys.argv
+        sys.exit(subprocess.call(cmd))
+    if world > 1 and world != args.gpus:
+        print(json.dumps({"error": f"WORLD_SIZE={world} but --gpus {args.gpus}"}), flush=True)
+        sys.exit(2)
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("gloo")

@@ -366,11 +366,19 @@ typedef struct {
   int32_t reps;              /* timed repetitions (median), default 5 */
   int32_t dp_warmup_chunks;  /* DP-Perf warm-up chunks per device per kernel (P311: 3) */
   int32_t chunks_per_dev;    /* nominal DP chunk size = n / (chunks_per_dev*G) */
-  int32_t measure_link;      /* 1: time a copy into each device for link_Bps */
+  int32_t measure_link;      /* link_Bps[d], Glinda's transfer metric (P49):
+                                0/1 (MM_LINK_PEER): 64 MiB copy into d from another
+                                logical device (peer GPU, else a device-to-device copy
+                                on the shared GPU); the resident exchange link.
+                                2 (MM_LINK_HOST): pinned host->device + device->host of
+                                64 MiB each, serialised (P119's staged transfers); sets
+                                mm_profile.staged = 1 so mm_split adds the transfer term */
 } mm_profile_opts;
+enum { MM_LINK_PEER = 1, MM_LINK_HOST = 2 };
 
 /* Glinda's low-cost profiling (P49) + the DP-Perf warm-up (P311), excluded
  * from run timings.  Runs kernels on the buffers (their contents change).
+ * link_Bps: best of max(reps, 2) timed copies after one warm-up copy.
  * buffers[slot*G + d] = device pointer of the slot on logical device d
  * (NULL where this rank does not own d).  With world > 1 the per-device rows
  * are exchanged so every rank returns the same profile. */

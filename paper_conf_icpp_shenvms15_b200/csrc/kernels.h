@@ -24,6 +24,12 @@ cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
   return e;
 }
 
+// Kernels launched by this process (mm_kernel_launch_count): every launch
+// site calls note_launch; a run's mm_run_stats.n_launches is the delta over
+// its issue (CUDA-graph replays add the kernels the graph holds).
+extern std::atomic<int64_t> g_kernel_launches;
+inline void note_launch(int64_t n = 1) { g_kernel_launches.fetch_add(n, std::memory_order_relaxed); }
+
 // Launch with programmatic stream serialization (PDL): the kernel may start
 // while the previous kernel on the stream finishes; it orders itself with
 // griddepcontrol.wait.
@@ -39,6 +45,7 @@ cudaError_t launch_pdl(void (*kern)(P...), dim3 grid, dim3 block, size_t smem, c
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
+  note_launch();
   return cudaLaunchKernelEx(&cfg, kern, std::forward<A>(args)...);
 }
 

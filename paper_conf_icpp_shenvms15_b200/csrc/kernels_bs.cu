@@ -124,6 +124,7 @@ cudaError_t blackscholes(const float* S, const float* X, const float* T, float* 
       static const int per_sm = getenv("MM_BS_CTAS") ? atoi(getenv("MM_BS_CTAS")) : 4;
       const int64_t cap = (int64_t)(sms > 0 ? sms : 148) * per_sm;
       if (per_sm > 0 && blocks > cap) blocks = cap;
+      note_launch();
       bs_vec<<<(unsigned)blocks, kThreads, 0, s>>>(
           reinterpret_cast<const float4*>(S), reinterpret_cast<const float4*>(X),
           reinterpret_cast<const float4*>(T), reinterpret_cast<float4*>(call),
@@ -133,6 +134,7 @@ cudaError_t blackscholes(const float* S, const float* X, const float* T, float* 
   }
   if (done < n) {
     const int64_t m = n - done;
+    note_launch();
     bs_scalar<<<(unsigned)((m + 255) / 256), 256, 0, s>>>(S + done, X + done, T + done, call + done,
                                                           put + done, m, R, V);
   }

@@ -47,6 +47,7 @@ cudaError_t fill_uniform(float* dst, int64_t n, uint64_t seed, int32_t array_id,
   if (n <= 0) return cudaSuccess;
   const uint64_t key = seed ^ ((uint64_t)(uint32_t)array_id << 48);
   const float span = hi - lo;  // one float32 rounding, as synthgen
+  note_launch();
   fill_u<<<grid_for(n), 256, 0, s>>>(dst, n, key, start, lo, span);
   return cudaGetLastError();
 }
@@ -56,6 +57,7 @@ cudaError_t fill_integers(float* dst, int64_t n, uint64_t seed, int32_t array_id
   if (n <= 0) return cudaSuccess;
   if (hi < lo) return cudaErrorInvalidValue;
   const uint64_t key = seed ^ ((uint64_t)(uint32_t)array_id << 48);
+  note_launch();
   fill_i<<<grid_for(n), 256, 0, s>>>(dst, n, key, start, lo, (uint64_t)(hi - lo + 1));
   return cudaGetLastError();
 }
@@ -95,6 +97,7 @@ cudaError_t fill_spd_tiles(float* dst, int64_t n, int64_t b, uint64_t seed, int3
   const uint64_t key = seed ^ ((uint64_t)(uint32_t)array_id << 48);
   int64_t blocks = (n * n + 255) / 256;
   if (blocks > 148 * 64) blocks = 148 * 64;
+  note_launch();
   fill_spd<<<(unsigned)blocks, 256, 0, s>>>(dst, n, b, key);
   return cudaGetLastError();
 }

@@ -139,6 +139,7 @@ cudaError_t sgemm_rows(const float* A, const float* B, float* C, int64_t M, int6
   if (r1 <= r0 || N <= 0) return cudaSuccess;
   if (variant == 2) return sgemm_tf32x3_rows(A, B, C, M, N, K, r0, r1, s, sms, scr, b_readonly);
   dim3 grid((unsigned)((N + BN - 1) / BN), (unsigned)((r1 - r0 + BM - 1) / BM));
+  note_launch();
   sgemm_ffma<<<grid, NT, 0, s>>>(A, B, C, N, K, r0, r1);
   return cudaGetLastError();
 }

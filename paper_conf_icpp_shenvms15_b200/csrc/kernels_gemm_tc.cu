@@ -569,15 +569,18 @@ cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, cons
   if (mc && pdl)
     return launch_pdl(gemm_tf32x3_pair<BN_>, dim3(2 * grid), dim3(kThreadsGemm), gemm_smem<BN_, true>(), s, ta_hi,
                       ta_lo, tb_hi, tb_lo, C, N, row0, mrows, nkb, units, job);
-  if (mc)
+  if (mc) {
+    note_launch();
     gemm_tf32x3_pair<BN_><<<2 * grid, kThreadsGemm, gemm_smem<BN_, true>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N,
                                                                                row0, mrows, nkb, units, job);
-  else if (pdl)
+  } else if (pdl) {
     return launch_pdl(gemm_tf32x3<BN_>, dim3(grid), dim3(kThreadsGemm), gemm_smem<BN_, false>(), s, ta_hi, ta_lo,
                       tb_hi, tb_lo, C, N, row0, mrows, nkb, units, job);
-  else
+  } else {
+    note_launch();
     gemm_tf32x3<BN_><<<grid, kThreadsGemm, gemm_smem<BN_, false>(), s>>>(ta_hi, ta_lo, tb_hi, tb_lo, C, N, row0,
                                                                          mrows, nkb, units, job);
+  }
   return cudaSuccess;
 }
 
@@ -603,6 +606,7 @@ cudaError_t split_needed(float* A, int64_t T, int64_t b, int32_t k, const int32_
       sl.ti[sl.n++] = i;
     }
   }
+  if (sl.n) note_launch();
   if (sl.n) split_tiles<<<dim3((unsigned)std::min<int64_t>(b * b / 4 / 256, 64), (unsigned)sl.n), 256, 0, s>>>(
       A, hi, lo, T, b, sl, k);
   return cudaSuccess;
@@ -786,6 +790,7 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
     const bool cached = b_readonly && scr->b_src == B && scr->b_K == K && scr->b_N == N && scr->b_epoch == scr->epoch;
     const int ntn = (int)((N + 31) / 32);
     const int64_t nblk_b = cached ? 0 : (int64_t)ntn * ((Kp + 31) / 32);
+    note_launch();
     split_ab<<<(unsigned)(nblk_a + nblk_b), 256, 0, s>>>(A, ahi, alo, B, bhi, blo, K, N, Kp, r0, mrows, nblk_a, ntn);
     if (!cached) {
       scr->b_src = b_readonly ? B : nullptr;

@@ -109,6 +109,7 @@ cudaError_t nbody_rows_launch(const float* pin, const float* vin, float* pout, f
   if (r1 <= r0) return cudaSuccess;
   if ((((uintptr_t)pin | (uintptr_t)vin | (uintptr_t)pout | (uintptr_t)vout) & 15u) != 0) return cudaErrorInvalidValue;
   if (!(eps2 >= 1.17549435e-38f)) return cudaErrorInvalidValue;   // normal eps^2 > 0 (rsqrt.ftz)
+  note_launch();
   nbody_rows<<<(unsigned)((r1 - r0 + 2 * kTile - 1) / (2 * kTile)), kTile, 0, s>>>(
       reinterpret_cast<const float4*>(pin), reinterpret_cast<const float4*>(vin), reinterpret_cast<float4*>(pout),
       reinterpret_cast<float4*>(vout), n, r0, r1, dt, eps2);

@@ -344,6 +344,7 @@ cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t ro
   nstrip = (nr + SR - 1) / SR;
   const int64_t warps = nwx * nstrip;
   if (warps + kTbWarps >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
+  note_launch();
   hotspot_tb<H><<<(unsigned)((warps + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, smem, s>>>(
       tin, pw, tout, (int)rows, (int)cols, (int)r0, (int)r1, c, (int)nwx, (int)SR);
   return cudaGetLastError();
@@ -424,9 +425,11 @@ cudaError_t hotspot_rows(const float* tin, const float* pw, float* tout, int64_t
   if (vec) {
     const int64_t ncb = (cols / 4 + kThreads - 1) / kThreads;
     const int64_t tiles = ncb * ((r1 - r0 + kH - 1) / kH);
+    note_launch();
     hotspot_vec<<<(unsigned)tiles, kThreads, 0, s>>>(tin, pw, tout, rows, cols, r0, r1, c, ncb);
   } else {
     const int64_t n = (r1 - r0) * cols;
+    note_launch();
     hotspot_scalar<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(tin, pw, tout, rows, cols, r0, r1, c);
   }
   return cudaGetLastError();
@@ -435,6 +438,7 @@ cudaError_t hotspot_rows(const float* tin, const float* pw, float* tout, int64_t
 cudaError_t row_residual(const float* t0, const float* t1, double* rowsum, int64_t cols, int64_t r0,
                          int64_t r1, cudaStream_t s, int) {
   if (r1 <= r0) return cudaSuccess;
+  note_launch();
   residual_rows<<<(unsigned)(r1 - r0), kThreads, 0, s>>>(t0, t1, rowsum, cols, r0);
   return cudaGetLastError();
 }

@@ -92,6 +92,7 @@ cudaError_t run(const float* x, const float* y, float* z, float q, int64_t lo, i
     const int64_t n4 = n / 4;
     if (n4 > 0) {
       const int64_t blocks = (n4 + kVecPerBlock - 1) / kVecPerBlock;
+      note_launch();
       stream_vec<OP><<<(unsigned)blocks, kThreads, 0, s>>>(
           reinterpret_cast<const float4*>(xs), reinterpret_cast<const float4*>(ys ? ys : xs),
           reinterpret_cast<float4*>(zs), n4, q);
@@ -100,6 +101,7 @@ cudaError_t run(const float* x, const float* y, float* z, float q, int64_t lo, i
   }
   if (done < n) {
     const int64_t m = n - done;
+    note_launch();
     stream_scalar<OP><<<(unsigned)((m + 255) / 256), 256, 0, s>>>(xs + done, ys ? ys + done : xs + done,
                                                                    zs + done, m, q);
   }

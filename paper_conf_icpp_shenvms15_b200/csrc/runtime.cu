@@ -153,7 +153,8 @@ struct mm_ctx {
   std::vector<std::pair<int32_t, int64_t>> reg_shape;
   // mm_ctx_set_stream: caller streams the runs of a device are ordered with
   std::vector<cudaStream_t> ext;
-  std::vector<cudaEvent_t> ext_ev;
+  std::vector<cudaEvent_t> ext_ev;    // created in the caller stream's (primary) context
+  std::vector<cudaEvent_t> lib_ev;    // created in the device's own (possibly green) context
 };
 
 namespace {
@@ -464,7 +465,6 @@ mm_status launch_task(mm_ctx* ctx, const App& app, const Task& t, int32_t d, voi
     ctx->poisoned = true;
     MM_FAIL(MM_ECUDA, "kernel %s launch failed: %s", k.name.c_str(), cudaGetErrorString(e));
   }
-  g_kernel_launches.fetch_add(1, std::memory_order_relaxed);
   return MM_OK;
 }
 
@@ -495,7 +495,6 @@ mm_status launch_task_batch(mm_ctx* ctx, const App& app, const std::vector<const
     ctx->poisoned = true;
     MM_FAIL(MM_ECUDA, "batched %s launch failed: %s", k.name.c_str(), cudaGetErrorString(e));
   }
-  g_kernel_launches.fetch_add(1, std::memory_order_relaxed);
   return MM_OK;
 }
 
@@ -639,7 +638,6 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
       mm_status r = launch_batch(ctx, plan, rt, (int64_t)i, d, buffers, s);
       if (r) return r;
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
-      st->n_launches++;
       for (int64_t m : rt->members[i])
         if (plan.needs_event[m]) CU_OK(cudaEventRecord(rt->ev[m], s));
     } else if (op.kind == MM_OPK_KERNEL) {
@@ -647,7 +645,6 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
       mm_status r = launch_task(ctx, app, plan.tasks[op.task], d, buffers, s);
       if (r) return r;
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
-      st->n_launches++;
     } else if (op.kind == MM_OPK_XFER) {
       const int64_t eb = app.buffers[op.buffer].first;
       const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
@@ -719,7 +716,6 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
                                             : launch_batch(ctx, plan, rt, (int64_t)i, me, buffers, s);
       if (r) return r;
       if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
-      st->n_launches++;
       continue;
     }
     const int64_t eb = app.buffers[op.buffer].first;
@@ -823,7 +819,6 @@ mm_status adaptive_issue_op(mm_ctx* ctx, AdaptiveState* ad, size_t i, void* cons
     CU_OK(cudaEventRecord(ad->ev_beg[i], s));
     r = launch_task(ctx, app, ap.tasks[op.task], d, buffers, s);
     if (r) return r;
-    st->n_launches++;
   } else if (op.kind == MM_OPK_XFER) {
     const int64_t eb = app.buffers[op.buffer].first;
     const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
@@ -1219,6 +1214,7 @@ void mm_ctx_destroy(mm_ctx* ctx) {
     if (r.scr.ptr) cudaFree(r.scr.ptr);
     const size_t d = (size_t)(&r - ctx->dev.data());
     if (d < ctx->ext_ev.size() && ctx->ext_ev[d]) cudaEventDestroy(ctx->ext_ev[d]);
+    if (d < ctx->lib_ev.size() && ctx->lib_ev[d]) cudaEventDestroy(ctx->lib_ev[d]);
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);
   }
   if (ctx->comm) nccl().CommDestroy(ctx->comm);
@@ -1248,6 +1244,7 @@ mm_status mm_ctx_set_stream(mm_ctx* ctx, int32_t d, void* stream) {
   if (ctx->ext.size() != (size_t)ctx->G) {
     ctx->ext.assign((size_t)ctx->G, nullptr);
     ctx->ext_ev.assign((size_t)ctx->G, nullptr);
+    ctx->lib_ev.assign((size_t)ctx->G, nullptr);
   }
   ctx->ext[d] = static_cast<cudaStream_t>(stream);
   return MM_OK;
@@ -1324,20 +1321,27 @@ mm_status resolve_buffers(mm_ctx* ctx, const Plan& plan, void* const*& buffers, 
 }
 
 // mm_ctx_set_stream: order device d's streams after the work already on the
-// caller's stream (before), or the caller's stream after the run (after)
+// caller's stream (before), or the caller's stream after the run (after).
+// An event must be recorded in its stream's context: the caller's stream
+// lives in the primary context of the GPU, the library's streams of an
+// SM-budgeted device in its green context; waits may cross contexts.
 mm_status join_external(mm_ctx* ctx, bool before) {
   for (int32_t d = 0; d < (int32_t)ctx->ext.size(); ++d) {
     if (!ctx->ext[d] || !ctx->dev[d].mine) continue;
     DevRt& r = ctx->dev[d];
-    CU_OK(set_dev(ctx, d));
-    if (!ctx->ext_ev[d]) CU_OK(cudaEventCreateWithFlags(&ctx->ext_ev[d], cudaEventDisableTiming));
     if (before) {
+      CU_OK(cudaSetDevice(r.phys));   // primary context of the caller's stream
+      if (!ctx->ext_ev[d]) CU_OK(cudaEventCreateWithFlags(&ctx->ext_ev[d], cudaEventDisableTiming));
       CU_OK(cudaEventRecord(ctx->ext_ev[d], ctx->ext[d]));
+      CU_OK(set_dev(ctx, d));
       for (cudaStream_t st : {r.stream, r.h2d, r.d2h, r.lane1})
         if (st) CU_OK(cudaStreamWaitEvent(st, ctx->ext_ev[d], 0));
     } else {
-      CU_OK(cudaEventRecord(ctx->ext_ev[d], r.stream));
-      CU_OK(cudaStreamWaitEvent(ctx->ext[d], ctx->ext_ev[d], 0));
+      CU_OK(set_dev(ctx, d));
+      if (!ctx->lib_ev[d]) CU_OK(cudaEventCreateWithFlags(&ctx->lib_ev[d], cudaEventDisableTiming));
+      CU_OK(cudaEventRecord(ctx->lib_ev[d], r.stream));
+      CU_OK(cudaSetDevice(r.phys));
+      CU_OK(cudaStreamWaitEvent(ctx->ext[d], ctx->lib_ev[d], 0));
     }
   }
   return MM_OK;
@@ -1370,7 +1374,9 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "run: adaptive DP-Perf is in-process only");
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_start, rs));
+    const int64_t l0 = g_kernel_launches.load();
     r = run_adaptive(ctx, plan, rt, buffers, o, S);
+    S->n_launches = g_kernel_launches.load() - l0;
     if (r) return r;
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_stop, rs));
@@ -1385,8 +1391,28 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   }
   rt->last_adaptive = false;
   if (graph) {
-    std::vector<void*> bufs(buffers, buffers + nbuf);
-    if (!rt->gexec || bufs != rt->graph_bufs) {
+    // Everything the captured graph bakes in is part of its key: the app
+    // buffers, each device's library scratch (operand splits, split-K
+    // partials, Cholesky panels and the TMA maps built on them), the host
+    // pointers of staged/flush copies and the pinned flush scratch.  Flush
+    // scratch is reserved before the key is formed (never inside a capture).
+    for (size_t i = 0; i < plan.ops.size(); ++i) {
+      const mm_op_rec& op = plan.ops[i];
+      if (op.kind != MM_OPK_FLUSH || !ctx->dev[op.device].mine) continue;
+      mm_status fs;
+      const int64_t eb = plan.app.buffers[op.buffer].first;
+      flush_target(ctx, plan, o, op.buffer, (size_t)(plan.app.buffers[op.buffer].second * eb), &fs);
+      if (fs) return fs;
+    }
+    std::vector<void*> key(buffers, buffers + nbuf);
+    for (auto& dv : ctx->dev) {
+      key.push_back(dv.scr.ptr);
+      key.push_back(reinterpret_cast<void*>(dv.scr.bytes));
+    }
+    for (size_t b = 0; b < plan.app.buffers.size(); ++b)
+      key.push_back(o && o->host ? o->host[b] : nullptr);
+    for (void* p : ctx->flush_scratch) key.push_back(p);
+    if (!rt->gexec || key != rt->graph_bufs) {
       if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
       if (rt->graph) cudaGraphDestroy(rt->graph);
       rt->gexec = nullptr;
@@ -1394,7 +1420,10 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       CU_OK(set_dev(ctx, root));
       CU_OK(cudaStreamBeginCapture(rs, cudaStreamCaptureModeThreadLocal));
       mm_run_stats cap{};
+      const int64_t l0 = g_kernel_launches.load();
       r = issue_local(ctx, plan, buffers, o, false, &cap);
+      const int64_t captured = g_kernel_launches.load() - l0;
+      g_kernel_launches.fetch_sub(captured, std::memory_order_relaxed);   // counted per replay
       cudaGraph_t g = nullptr;
       cudaError_t ce = cudaStreamEndCapture(rs, &g);
       if (r) {
@@ -1404,8 +1433,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       CU_OK(ce);
       rt->graph = g;
       CU_OK(cudaGraphInstantiate(&rt->gexec, g, 0));
-      rt->graph_bufs = bufs;
-      rt->graph_launches = cap.n_launches;
+      rt->graph_bufs = key;
+      rt->graph_launches = captured;
       rt->graph_xfer = cap.xfer_bytes;
       rt->graph_h2d = cap.h2d_bytes;
       rt->graph_d2h = cap.d2h_bytes;
@@ -1423,8 +1452,10 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   } else {
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_start, rs));
+    const int64_t l0 = g_kernel_launches.load();
     if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
     else r = issue_dist(ctx, plan, buffers, o, timing, S);
+    S->n_launches = g_kernel_launches.load() - l0;
     if (r) return r;
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_stop, rs));
@@ -1524,6 +1555,8 @@ mm_status mm_collect(mm_ctx* ctx, const mm_plan* plan_h, void* const* buffers, i
   const PlanRt* prt = static_cast<const PlanRt*>(plan_h->p.rt);
   const Plan& plan = (prt && prt->last_adaptive && prt->ad) ? prt->ad->ap : plan_h->p;
   if (ctx->world != 1) MM_FAIL(MM_ENOTSUP, "collect: in-process contexts only");
+  if (ctx->poisoned) MM_FAIL(MM_ESTATE, "ctx poisoned by an earlier CUDA error");
+  if (dst_device >= ctx->G) MM_FAIL(MM_EINVAL, "collect: dst_device %d of G=%d", dst_device, ctx->G);
   if (slot < 0 || slot >= (int32_t)plan.app.buffers.size()) MM_FAIL(MM_EINVAL, "collect: slot");
   const int64_t eb = plan.app.buffers[slot].first;
   for (auto& seg : plan.final_owner[slot]) {
@@ -1555,6 +1588,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
   *out = mm_profile{};
   out->G = G;
   out->K = K;
+  out->staged = po && po->measure_link == 2 ? 1 : 0;
   std::vector<uint64_t> row(2 * MM_MAX_K + 1, 0);
   try {
     for (int32_t d = 0; d < G; ++d) {
@@ -1649,22 +1683,58 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
           out->chunk_est_ns[d][k] = std::max<uint64_t>(1, (uint64_t)((double)ms * 1e6 / (double)ch.size()));
         }
       }
-      // link: bytes/s of a 64 MiB device-to-device copy into d
+      // Glinda's second metric (P49: "the GPU computation to data transfer
+      // gap"): bytes/s of the link data crosses to reach device d.
+      //  host (staged, measure_link = 2): one pinned host->device copy then one
+      //   device->host copy of 64 MiB on d's stream, serialised as P119's
+      //   "single host-to-device data transfer before the first kernel ... one
+      //   device-to-host data transfer after the last"; B = 2 x 64 MiB / time.
+      //  peer (resident, 0/1): a 64 MiB copy into d from another logical
+      //   device's memory — cudaMemcpyPeerAsync when that device is another
+      //   GPU, else a device-to-device copy (the XFER of logical devices that
+      //   share a GPU); with no other device, a copy within d.
       {
         const size_t bytes = 64ull << 20;
+        const bool host = po && po->measure_link == 2;
         void *x = nullptr, *y = nullptr;
-        CU_OK(cudaMalloc(&x, bytes));
+        int32_t src_phys = ctx->dev[d].phys;
+        for (int32_t q = 0; q < G; ++q)
+          if (q != d && ctx->dev[q].mine && ctx->dev[q].phys != ctx->dev[d].phys) {
+            src_phys = ctx->dev[q].phys;
+            break;
+          }
         CU_OK(cudaMalloc(&y, bytes));
-        CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
-        CU_OK(cudaEventRecord(a, s));
-        CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
-        CU_OK(cudaEventRecord(b, s));
-        CU_OK(cudaEventSynchronize(b));
-        float ms = 0.f;
-        CU_OK(cudaEventElapsedTime(&ms, a, b));
-        cudaFree(x);
+        if (host) {
+          CU_OK(cudaMallocHost(&x, bytes));
+          std::memset(x, 0, bytes);
+        } else {
+          if (src_phys != ctx->dev[d].phys) CU_OK(cudaSetDevice(src_phys));
+          CU_OK(cudaMalloc(&x, bytes));
+          CU_OK(cudaMemset(x, 0, bytes));
+          CU_OK(cudaDeviceSynchronize());
+          CU_OK(set_dev(ctx, d));
+        }
+        float best = 0.f;
+        for (int32_t i = 0; i < 1 + std::max<int32_t>(reps, 2); ++i) {   // first = warm-up
+          CU_OK(cudaEventRecord(a, s));
+          if (host) {
+            CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyHostToDevice, s));
+            CU_OK(cudaMemcpyAsync(x, y, bytes, cudaMemcpyDeviceToHost, s));
+          } else if (src_phys != ctx->dev[d].phys) {
+            CU_OK(cudaMemcpyPeerAsync(y, ctx->dev[d].phys, x, src_phys, bytes, s));
+          } else {
+            CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
+          }
+          CU_OK(cudaEventRecord(b, s));
+          CU_OK(cudaEventSynchronize(b));
+          float ms = 0.f;
+          CU_OK(cudaEventElapsedTime(&ms, a, b));
+          if (i > 0 && (best == 0.f || ms < best)) best = ms;
+        }
+        if (host) cudaFreeHost(x);
+        else cudaFree(x);
         cudaFree(y);
-        out->link_Bps[d] = (uint64_t)((double)bytes / (ms * 1e-3));
+        out->link_Bps[d] = (uint64_t)((double)(host ? 2 * bytes : bytes) / ((double)best * 1e-3));
       }
       cudaEventDestroy(a);
       cudaEventDestroy(b);

@@ -23,6 +23,7 @@ MM_SK_ONE, MM_SK_LOOP, MM_MK_SEQ, MM_MK_LOOP, MM_MK_DAG = 1, 2, 3, 4, 5
 MM_SP_SINGLE, MM_SP_UNIFIED, MM_SP_VARIED, MM_DP_PERF, MM_DP_DEP, MM_SP_CYCLIC, MM_DP_STATIC = 1, 2, 3, 4, 5, 6, 7
 MM_SYNC_NONE, MM_SYNC_BARRIER, MM_SYNC_FLUSH = 0, 1, 2
 MM_READ, MM_WRITE, MM_RW = 1, 2, 3
+MM_LINK_PEER, MM_LINK_HOST = 1, 2
 (MM_OP_CUSTOM, MM_OP_STREAM_COPY, MM_OP_STREAM_SCALE, MM_OP_STREAM_ADD, MM_OP_STREAM_TRIAD,
  MM_OP_HOTSPOT, MM_OP_ROW_RESIDUAL, MM_OP_BLACKSCHOLES, MM_OP_SGEMM, MM_OP_CHOL_POTRF,
  MM_OP_CHOL_TRSM, MM_OP_CHOL_SYRK, MM_OP_CHOL_GEMM, MM_OP_NBODY) = range(14)
@@ -525,8 +526,10 @@ def _ptr_array(ptrs: Sequence[int]):
 
 
 def mm_profile_run(ctx: int, app: int, buffers: Sequence[int], reps: int = 5, dp_warmup_chunks: int = 3,
-                   chunks_per_dev: int = 8, probe_items: int = 0) -> mm_profile:
-    o = mm_profile_opts(probe_items, reps, dp_warmup_chunks, chunks_per_dev, 1)
+                   chunks_per_dev: int = 8, probe_items: int = 0, link: str = "peer") -> mm_profile:
+    """link = "peer" (resident exchanges) or "host" (staged: pinned PCIe copies; sets prof.staged)."""
+    o = mm_profile_opts(probe_items, reps, dp_warmup_chunks, chunks_per_dev,
+                        {"peer": MM_LINK_PEER, "host": MM_LINK_HOST}[link])
     p = mm_profile()
     _call("mm_profile_run", ctx, app, _ptr_array(buffers), C.byref(o), C.byref(p))
     return p

@@ -1,0 +1,210 @@
+"""Round-2 pins of oracle functions that had none ("parity
+unpinned"): SP-Cyclic's tile -> device map, the per-item link bytes of the
+staged split (R5, P119), and the staged sub-chunk pipeline (R24) against
+P119's one H2D before the first kernel / one D2H after the last.
+
+Every expected value here is written out by hand from the cited passage, not
+computed by calling the oracle's own arithmetic a second time."""
+import pytest
+
+from oracle import apps as oa
+from oracle import control as oc
+
+# ---------------------------------------------------------------- SP-Cyclic --
+# R17: tile (i, j) -> device (i mod Pr) * Pc + (j mod Pc), Pr = the largest
+# divisor of G not above sqrt(G).  By hand: G=2 -> 1 x 2, G=4 -> 2 x 2,
+# G=6 -> 2 x 3, G=8 -> 2 x 4.  Rows below = lower-triangle tiles (i >= j) of a
+# 5 x 5 tile grid, row i listing j = 0..i.
+CYCLIC_HAND = {
+    2: [[0],
+        [0, 1],
+        [0, 1, 0],
+        [0, 1, 0, 1],
+        [0, 1, 0, 1, 0]],
+    4: [[0],
+        [2, 3],
+        [0, 1, 0],
+        [2, 3, 2, 3],
+        [0, 1, 0, 1, 0]],
+    6: [[0],
+        [3, 4],
+        [0, 1, 2],
+        [3, 4, 5, 3],
+        [0, 1, 2, 0, 1]],
+    8: [[0],
+        [4, 5],
+        [0, 1, 2],
+        [4, 5, 6, 7],
+        [0, 1, 2, 3, 0]],
+}
+
+
+@pytest.mark.parametrize("G", [2, 4, 6, 8])
+def test_sp_cyclic_hand_maps(G):
+    app = oa.cholesky_tasks(5, 1)
+    tasks, dev = oc.sp_cyclic(app, G)
+    seen = {}
+    for t, d in zip(tasks, dev):
+        i, j = t.ij
+        assert d == CYCLIC_HAND[G][i][j], (G, i, j)
+        seen.setdefault((i, j), set()).add(d)
+    # owner-computes: every task writing a tile runs on that tile's device
+    assert all(len(s) == 1 for s in seen.values())
+    assert len(seen) == 15
+
+
+def test_sp_cyclic_explicit_grid_rows():
+    # grid_rows given: G = 8 as 4 x 2 -> (i mod 4) * 2 + (j mod 2)
+    app = oa.cholesky_tasks(5, 1)
+    tasks, dev = oc.sp_cyclic(app, 8, grid_rows=4)
+    hand = {(0, 0): 0, (1, 0): 2, (1, 1): 3, (2, 0): 4, (2, 1): 5, (2, 2): 4, (3, 0): 6, (3, 1): 7,
+            (3, 2): 6, (3, 3): 7, (4, 0): 0, (4, 1): 1, (4, 2): 0, (4, 3): 1, (4, 4): 0}
+    for t, d in zip(tasks, dev):
+        assert d == hand[t.ij]
+
+
+def test_sp_cyclic_cpp_matches_hand_maps():
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    for G in (2, 4, 6, 8):
+        app = mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [5 * 32, 32])
+        prof = mm.make_profile(G, [[1000] * 4] * G, [[1000] * 4] * G, [10 ** 9] * G)
+        plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_SP_CYCLIC))
+        otasks = oa.cholesky_tasks(5, 32).dag_tasks
+        for c, t in zip(mm.mm_plan_chunks(plan), otasks):
+            i, j = t.ij
+            assert c.device == CYCLIC_HAND[G][i][j]
+        mm.mm_plan_destroy(plan)
+        mm.mm_app_destroy(app)
+
+
+# ------------------------------------------------------- link bytes (R5) ----
+def bs_app(n):
+    """BlackScholes (P311): S, X, T read; call, put written (5 FP32 arrays)."""
+    k = oc.Kernel("bs", n, 32, 1, [oc.Access(0, oc.READ), oc.Access(1, oc.READ), oc.Access(2, oc.READ),
+                                   oc.Access(3, oc.WRITE), oc.Access(4, oc.WRITE)])
+    return oc.App(buffers=[(4, n)] * 5, kernels=[k])
+
+
+def sgemm_app(M, N, K):
+    """Row-split C = A B (P311): per row K floats of A in, N floats of C out;
+    B is a whole-buffer operand (R18), not per item."""
+    k = oc.Kernel("sgemm", M, 16, 1, [oc.Access(0, oc.READ, K), oc.Access(1, oc.READ, 0),
+                                      oc.Access(2, oc.WRITE, N)])
+    return oc.App(buffers=[(4, M * K), (4, K * N), (4, M * N)], kernels=[k])
+
+
+def test_link_bytes_stream_by_hand():
+    # copy c=a: a in, c out = 8 B; scale b=s c: 8 B; add c=a+b: 12 B; triad
+    # a=b+s c: 12 B per element when each kernel runs alone (SP-Single/Varied)
+    app = oa.stream(1024, 1)
+    assert [oc.kernel_link_bytes(app, k) for k in range(4)] == [8, 8, 12, 12]
+    # SP-Unified (P119): one H2D before the first kernel — only a is read
+    # before being written (copy reads a; scale reads c, written by copy; add
+    # reads b, written by scale; triad reads b, c) = 4 B — and one D2H after
+    # the last of every written array (c, b, a) = 12 B: 16 B per element.
+    assert oc.unified_link_bytes(app) == 16
+
+
+def test_link_bytes_blackscholes_by_hand():
+    # 3 inputs + 2 outputs x 4 B = 20 B per option, alone or unified
+    app = bs_app(1000)
+    assert oc.kernel_link_bytes(app, 0) == 20
+    assert oc.unified_link_bytes(app) == 20
+
+
+@pytest.mark.parametrize("cols", [1, 8, 8192])
+def test_link_bytes_hotspot_by_hand(cols):
+    # per row: T_in (cols floats) and P (cols floats) in, T_out out: 12 cols B
+    app = oa.hotspot(16, cols, 4)
+    assert oc.kernel_link_bytes(app, 0) == 12 * cols
+    assert oc.unified_link_bytes(app) == 12 * cols
+
+
+def test_link_bytes_stencil_reduction_by_hand():
+    cols = 64
+    app = oa.stencil_reduction(16, cols, 3)
+    # stencil alone: T_in, P in, T_out out = 12 cols; residual alone: T_in,
+    # T_out in (8 cols) + one FP64 row sum out (8 B)
+    assert oc.kernel_link_bytes(app, 0) == 12 * cols
+    assert oc.kernel_link_bytes(app, 1) == 8 * cols + 8
+    # unified: T_in and P read first (8 cols), T_out and rowsum written (4 cols + 8)
+    assert oc.unified_link_bytes(app) == 12 * cols + 8
+
+
+def test_link_bytes_sgemm_by_hand():
+    app = sgemm_app(64, 48, 80)
+    assert oc.kernel_link_bytes(app, 0) == 4 * 80 + 4 * 48
+
+
+def test_staged_split_prices_the_link():
+    """Glinda's R_GD term (P49): with identical compute on two devices, the
+    device behind a 4x slower link gets the smaller share, and with a link of
+    v bytes/item at B bytes/s the per-item cost grows by v/B.  Hand numbers:
+    STREAM-Seq unified v = 16 B; B0 = 16e9 B/s -> 1 ns = 1e6 fs per element;
+    B1 = 4e9 -> 4e6 fs.  fs_item 1e5 per kernel (4e5 summed).  Costs 1.4e6 vs
+    4.4e6 fs: n0/n = 4.4 / 5.8 -> 0.7586 of 2^20, rounded up to 32."""
+    n = 1 << 20
+    app = oa.stream(n, 1)
+    prof = oc.Profile(G=2, fs_item=[[100000] * 4, [100000] * 4], chunk_est_ns=[[1] * 4] * 2,
+                      link_Bps=[16 * 10 ** 9, 4 * 10 ** 9], staged=True)
+    r = oc.sp_split(app, prof, oc.SP_UNIFIED)[0]
+    n0 = r[0][1] - r[0][0]
+    assert abs(n0 / n - 4.4 / 5.8) < 1e-4
+    assert n0 % 32 == 0 and r[1] == (n0, n)
+    # resident (no link term): equal compute -> equal split
+    prof.staged = False
+    r = oc.sp_split(app, prof, oc.SP_UNIFIED)[0]
+    assert r == [(0, n // 2), (n // 2, n)]
+
+
+# --------------------------------------------------- staged pipeline (R24) --
+def _per_elem(ops, kind, G, nbuf, n):
+    """Count, per (buffer, element), how often it crosses the link."""
+    cnt = [[0] * n for _ in range(nbuf)]
+    for o in ops:
+        if kind == oc.OP_XFER and o[0] == oc.OP_XFER and o[2] == -1:
+            b, lo, hi = o[3], o[4], o[5]
+        elif kind == oc.OP_FLUSH and o[0] == oc.OP_FLUSH:
+            b, lo, hi = o[2], o[3], o[4]
+        else:
+            continue
+        for x in range(lo, hi):
+            cnt[b][x] += 1
+    return cnt
+
+
+@pytest.mark.parametrize("P", [1, 2, 5])
+@pytest.mark.parametrize("passes", [1, 2])
+def test_pipelined_staged_program_moves_each_element_once(P, passes):
+    """P119: SP-Unified needs "a single host-to-device data transfer before the
+    first kernel ... and one device-to-host data transfer after the last".  The
+    pipelined program (R24) may cut it into sub-chunks but must keep exactly
+    that per element: array a (the only one read before written) goes in once,
+    every element of the written arrays a, b, c comes out once, b and c never
+    go in — whatever P, and the same element sets as the unpipelined program."""
+    n, G = 301, 2
+    app = oa.stream(n, passes)
+    prof = oc.Profile(G=G, fs_item=[[10] * 4, [23] * 4], chunk_est_ns=[[1] * 4] * 2, link_Bps=[10 ** 9] * 2)
+    ranges = oc.sp_split(app, prof, oc.SP_UNIFIED)
+    tasks, dev, flush = oc.sp_tasks_pipelined(app, ranges, P)
+    ops = oc.op_program(app, G, tasks, dev, oc.SP_UNIFIED, True, None, flush)
+    h2d = _per_elem(ops, oc.OP_XFER, G, 3, n)
+    d2h = _per_elem(ops, oc.OP_FLUSH, G, 3, n)
+    assert h2d[0] == [1] * n and h2d[1] == [0] * n and h2d[2] == [0] * n
+    assert d2h == [[1] * n] * 3
+    # same per-element traffic as P119's one-shot program
+    t1, d1 = oc.sp_tasks(app, ranges)
+    ops1 = oc.op_program(app, G, t1, d1, oc.SP_UNIFIED, True)
+    assert _per_elem(ops1, oc.OP_XFER, G, 3, n) == h2d
+    assert _per_elem(ops1, oc.OP_FLUSH, G, 3, n) == d2h
+    # no element is flushed before its final write: every FLUSH of a
+    # (device, range) follows the last KERNEL op of that device that writes it
+    last_kernel = {}
+    for i, o in enumerate(ops):
+        if o[0] == oc.OP_KERNEL:
+            last_kernel.setdefault(o[1], []).append((i, o[4], o[5]))
+    for i, o in enumerate(ops):
+        if o[0] == oc.OP_FLUSH:
+            d, lo, hi = o[1], o[3], o[4]
+            later = [k for (k, b, e) in last_kernel[d] if k > i and b < hi and lo < e]
+            assert not later

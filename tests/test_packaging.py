@@ -26,6 +26,8 @@ def test_product_package_does_not_import_oracle():
         for f in files:
             if f.endswith((".py", ".cu", ".cpp", ".h")):
                 src = open(os.path.join(dirpath, f)).read()
-                assert "oracle" not in src.replace("oracle/", "").split("\n")[0] or True
+                # comments may cite the oracle; code may not name its module or library
+                code = "\n".join(ln.split("//")[0].split("#")[0] for ln in src.split("\n"))
+                assert "oracle" not in code, f
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "or_stream" not in src and "_numeric" not in src, f
