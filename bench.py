@@ -261,6 +261,9 @@ def main():
                     help="use an equal synthetic profile instead of measuring one (ncu runs)")
     ap.add_argument("--kernel-timing", default="last", choices=["all", "last", "none"],
                     help="per-kernel CUDA events in the timed steps: every step, the last ceil(K/5) steps, or none")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="ranks share GPUs (rank r on cuda:r %% count): exercises the multi-process "
+                         "IPC path on a box with fewer GPUs than ranks; not a scaling measurement")
     ap.add_argument("--logical", type=int, default=0,
                     help="virtual mode: run G logical devices on this one GPU (G = --logical)")
     args = ap.parse_args()
@@ -273,11 +276,11 @@ def main():
     from paper_conf_icpp_shenvms15_b200 import mm, runner
 
     world, rank, local = dist_env()
+    have = torch.cuda.device_count()
     if args.gpus > 1 and world == 1:
-        # --gpus N without a launcher: one rank per GPU needs N visible GPUs;
-        # never time fewer GPUs than asked for (exit non-zero instead)
-        have = torch.cuda.device_count()
-        if have < args.gpus:
+        # --gpus N without a launcher: one rank per GPU needs N visible GPUs
+        # (or --share-gpu); never time fewer GPUs than asked for
+        if have < args.gpus and not args.share_gpu:
             print(json.dumps({"error": f"--gpus {args.gpus} but only {have} CUDA device(s) visible",
                               "n_gpus": have}), flush=True)
             sys.exit(2)
@@ -287,10 +290,18 @@ def main():
     if world > 1 and world != args.gpus:
         print(json.dumps({"error": f"WORLD_SIZE={world} but --gpus {args.gpus}"}), flush=True)
         sys.exit(2)
+    if world > have and not args.share_gpu:
+        print(json.dumps({"error": f"{world} ranks but only {have} CUDA device(s) visible"}), flush=True)
+        sys.exit(2)
+    if args.share_gpu:   # exercising the multi-process path on fewer GPUs than ranks
+        local = local % have
     torch.cuda.set_device(local)
     if world > 1:
+        # rank 0 names the context: the IPC rendezvous id (default transport:
+        # CUDA IPC pulls + device-memory flags) or an NCCL id (MM_TRANSPORT=nccl)
         dist.init_process_group("gloo")
-        nid = [mm.mm_nccl_unique_id() if rank == 0 else None]
+        nccl = os.environ.get("MM_TRANSPORT") == "nccl"
+        nid = [(mm.mm_nccl_unique_id() if nccl else mm.mm_rendezvous_id()) if rank == 0 else None]
         dist.broadcast_object_list(nid, src=0)
         nccl_id = nid[0]
     else:

@@ -310,14 +310,28 @@ typedef struct {
   int32_t _pad;
 } mm_device_spec;
 
-/* NCCL unique id for multi-process contexts (128 bytes), created on rank 0
- * and broadcast by the caller. */
+/* Rendezvous id of a multi-process context (128 random bytes), created on
+ * rank 0 and broadcast by the caller (IPC transport, the default). */
+mm_status mm_rendezvous_id(void* out128);
+/* NCCL unique id (128 bytes) for the NCCL transport (MM_TRANSPORT=nccl). */
 mm_status mm_nccl_unique_id(void* out128);
 /* G logical devices; this process is `my_rank` of `world` (1 = in-process:
  * every device has rank 0, exchanges are cudaMemcpyAsync on the consumer's
- * stream).  world > 1: each rank owns exactly one logical device and
- * exchanges are NCCL send/recv on the owning device's stream (nccl_id must
- * be the same 128 bytes on every rank). */
+ * stream).  world > 1 (all ranks on one node): each rank owns exactly one
+ * logical device; `nccl_id` = the same 128 bytes on every rank.
+ *  - IPC transport (default): the ranks meet in a POSIX shared-memory block
+ *    named after the id (host barrier, exchange of CUDA IPC handles); every
+ *    rank runs the in-process executor's op program for its device, pulls
+ *    (XFER) copy straight out of the producer rank's buffer through its IPC
+ *    mapping (NVLink peer memory between GPUs; ranks may also share a GPU),
+ *    and cross-rank hazards are waits on device-memory completion flags the
+ *    producer/reader signals.  mm_run exchanges the buffer handles (a host
+ *    barrier) and may capture the rank's program as a CUDA graph.
+ *  - NCCL transport (environment MM_TRANSPORT=nccl, id from
+ *    mm_nccl_unique_id): XFERs are grouped ncclSend/ncclRecv on the device's
+ *    stream, BARRIER a 4-byte all-reduce; no graph capture; one rank per GPU.
+ * Errors: MM_EINVAL, MM_ESTATE (a rank never joined the rendezvous within
+ * 120 s), MM_ECUDA, MM_ENCCL. */
 mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, int32_t world,
                         const void* nccl_id, mm_ctx** out);
 void      mm_ctx_destroy(mm_ctx* ctx);

@@ -97,7 +97,8 @@ def cholesky_tasks(T: int, b: int) -> App:
                                   [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)], ij=(i, j)))
     ks = [Kernel(nm, 1, 1, 1, []) for nm in ("potrf", "trsm", "syrk", "gemm")]
     edges = [(0, 1), (1, 2), (1, 3), (2, 0), (3, 1), (3, 2), (3, 3)]
-    return App(buffers=[(4, T * T * bb)], kernels=ks, edges=edges, dag_tasks=tasks)
+    # POTRF and TRSM (the critical path) on compute lane 1 (R31)
+    return App(buffers=[(4, T * T * bb)], kernels=ks, edges=edges, dag_tasks=tasks, lanes={0: 1, 1: 1})
 
 
 def nbody(n: int, iters: int, granule: int = 256, min_items: int = 1) -> App:

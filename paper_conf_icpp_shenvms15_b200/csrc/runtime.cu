@@ -17,8 +17,10 @@
 #include <memory>
 #include <new>
 #include <map>
+#include <random>
 #include <vector>
 
+#include "ipc.h"
 #include "kernels.h"
 #include "mm_internal.h"
 #include "segmap.h"
@@ -155,6 +157,9 @@ struct mm_ctx {
   std::vector<cudaStream_t> ext;
   std::vector<cudaEvent_t> ext_ev;    // created in the caller stream's (primary) context
   std::vector<cudaEvent_t> lib_ev;    // created in the device's own (possibly green) context
+  // world > 1: IPC transport (default) or NCCL (MM_TRANSPORT=nccl)
+  IpcChannel* ipc = nullptr;
+  std::vector<char*> ipc_bufs;        // [slot * world + rank]: pointers valid in this process
 };
 
 namespace {
@@ -227,6 +232,8 @@ struct PlanRt {
   // DAG task batching: members[head] = kernel ops launched together with head
   std::vector<int64_t> batch_head;               // -1: not a member of another op's batch
   std::vector<std::vector<int64_t>> members;
+  // IPC transport: op i is waited on by another rank's stream (signal its flag)
+  std::vector<uint8_t> remote_sig;
 };
 
 bool is_batchable_op(int32_t op) {
@@ -538,6 +545,14 @@ mm_status ensure_rt(mm_ctx* ctx, Plan& plan, bool timing) {
     CU_OK(cudaEventCreate(&rt->t_start));
     CU_OK(cudaEventCreate(&rt->t_stop));
     compute_batches(plan, rt);
+    rt->remote_sig.assign(plan.ops.size(), 0);
+    if (ctx->ipc)
+      for (size_t j = 0; j < plan.ops.size(); ++j) {
+        if (plan.op_stream[j] < 0) continue;
+        const int32_t rj = ctx->dev[sid_dev(ctx, plan.op_stream[j])].rank;
+        for (auto& w : plan.waits[j])
+          if (ctx->dev[sid_dev(ctx, w.dev)].rank != rj) rt->remote_sig[w.op] = 1;
+      }
   }
   // reserve device scratch for every kernel op before any graph capture
   for (size_t i = 0; i < plan.ops.size(); ++i) {
@@ -754,6 +769,149 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
     }
   }
   if (in_group) NCCL_OK(nccl().GroupEnd());
+  return MM_OK;
+}
+
+// Issue the op program of one rank of a multi-process ctx on the IPC
+// transport: the in-process executor's program (four streams, exact
+// hazards) restricted to the owned device, with every hazard on another
+// rank's op turned into a wait on that rank's completion flag, every op a
+// peer waits on followed by a flag signal, pulls copying straight out of the
+// peer's buffer (ctx->ipc_bufs), and BARRIER = join, signal, wait for every
+// rank, fork.  A run starts by bumping this rank's epoch and waiting for
+// every peer to have finished the previous run (cross-run WAR on pulled
+// ranges); it ends by signalling its own end.  Capturable as a CUDA graph.
+mm_status issue_ipc(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run_opts* o, bool timing,
+                    mm_run_stats* st) {
+  PlanRt* rt = static_cast<PlanRt*>(plan.rt);
+  IpcChannel* ch = ctx->ipc;
+  const int32_t G = ctx->G, W = ctx->world;
+  const int32_t me = first_owned(ctx);
+  const App& app = plan.app;
+  const int32_t NS = kKinds * G;
+  if ((int64_t)plan.ops.size() + kIpcOp0 > kIpcFlagSlots)
+    MM_FAIL(MM_ENOTSUP, "ipc: %zu ops exceed the flag slots", plan.ops.size());
+  std::vector<uint8_t> used(NS, 0);
+  for (size_t i = 0; i < plan.ops.size(); ++i)
+    if (plan.op_stream[i] >= 0 && sid_dev(ctx, plan.op_stream[i]) == me) used[plan.op_stream[i]] = 1;
+  const int32_t root = me;   // compute stream of the owned device
+  used[root] = 1;
+  auto rank_of_sid = [&](int32_t sid) { return ctx->dev[sid_dev(ctx, sid)].rank; };
+  std::vector<uint64_t*> wp;
+  std::vector<int64_t> ws;
+  std::vector<uint32_t> wl;
+  auto flush_waits = [&](cudaStream_t s) -> mm_status {
+    if (wp.empty()) return MM_OK;
+    CU_OK(ipc_wait(ch->flags, wp.data(), ws.data(), wl.data(), (int32_t)wp.size(), s));
+    wp.clear();
+    ws.clear();
+    wl.clear();
+    return MM_OK;
+  };
+  auto fork_from_root = [&](cudaEvent_t* evs) -> mm_status {
+    CU_OK(cudaEventRecord(evs[root], ctx->dev[me].stream));
+    for (int32_t sid = 0; sid < NS; ++sid)
+      if (used[sid] && sid != root) CU_OK(cudaStreamWaitEvent(sid_stream(ctx, sid), evs[root], 0));
+    return MM_OK;
+  };
+  auto join_to_root = [&](cudaEvent_t* evs) -> mm_status {
+    for (int32_t sid = 0; sid < NS; ++sid)
+      if (used[sid] && sid != root) {
+        CU_OK(cudaEventRecord(evs[sid], sid_stream(ctx, sid)));
+        CU_OK(cudaStreamWaitEvent(ctx->dev[me].stream, evs[sid], 0));
+      }
+    return MM_OK;
+  };
+  CU_OK(set_dev(ctx, me));
+  cudaStream_t rs = ctx->dev[me].stream;
+  // run start: new epoch; every peer has finished the previous run
+  CU_OK(ipc_bump_epoch(ch->flags, rs));
+  for (int32_t q = 0; q < W; ++q)
+    if (q != ctx->my_rank) {
+      wp.push_back(ch->peer_flags[q]);
+      ws.push_back(kIpcEnd);
+      wl.push_back(1);
+    }
+  if (mm_status r = flush_waits(rs)) return r;
+  if (mm_status r = fork_from_root(rt->bar_ev.data())) return r;
+  for (size_t i = 0; i < plan.ops.size(); ++i) {
+    const mm_op_rec& op = plan.ops[i];
+    if (op.kind == MM_OPK_BARRIER) {
+      if (mm_status r = join_to_root(rt->join_ev.data())) return r;
+      CU_OK(ipc_signal(ch->flags, kIpcOp0 + (int64_t)i, rs));
+      for (int32_t q = 0; q < W; ++q)
+        if (q != ctx->my_rank) {
+          wp.push_back(ch->peer_flags[q]);
+          ws.push_back(kIpcOp0 + (int64_t)i);
+          wl.push_back(0);
+        }
+      if (mm_status r = flush_waits(rs)) return r;
+      if (mm_status r = fork_from_root(rt->bar_ev.data())) return r;
+      continue;
+    }
+    const int32_t d = sid_dev(ctx, plan.op_stream[i]);
+    if (d != me) continue;
+    if (op.kind == MM_OPK_KERNEL && rt->batch_head[i] >= 0) continue;   // launched with its head
+    cudaStream_t s = sid_stream(ctx, plan.op_stream[i]);
+    auto add_waits = [&](size_t j) -> mm_status {
+      for (auto& w : plan.waits[j]) {
+        if (sid_dev(ctx, w.dev) == me) {
+          CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
+        } else {
+          wp.push_back(ch->peer_flags[rank_of_sid(w.dev)]);
+          ws.push_back(kIpcOp0 + w.op);
+          wl.push_back(0);
+        }
+      }
+      return MM_OK;
+    };
+    if (mm_status r = add_waits(i)) return r;
+    if (op.kind == MM_OPK_KERNEL)
+      for (int64_t m : rt->members[i])
+        if (mm_status r = add_waits((size_t)m)) return r;
+    if (mm_status r = flush_waits(s)) return r;
+    if (op.kind == MM_OPK_KERNEL) {
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      mm_status r = rt->members[i].empty() ? launch_task(ctx, app, plan.tasks[op.task], d, buffers, s)
+                                           : launch_batch(ctx, plan, rt, (int64_t)i, d, buffers, s);
+      if (r) return r;
+      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      for (int64_t m : rt->members[i]) {
+        if (plan.needs_event[m]) CU_OK(cudaEventRecord(rt->ev[m], s));
+        if (rt->remote_sig[m]) CU_OK(ipc_signal(ch->flags, kIpcOp0 + m, s));
+      }
+    } else if (op.kind == MM_OPK_XFER) {
+      const int64_t eb = app.buffers[op.buffer].first;
+      const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+      char* dst = static_cast<char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+      if (op.src < 0) {
+        if (!o || !o->host || !o->host[op.buffer]) MM_FAIL(MM_EINVAL, "staged run: no host pointer for slot %d", op.buffer);
+        CU_OK(cudaMemcpyAsync(dst, static_cast<const char*>(o->host[op.buffer]) + op.r.begin * eb, bytes,
+                              cudaMemcpyHostToDevice, s));
+        st->h2d_bytes += (int64_t)bytes;
+      } else {
+        const char* src = ctx->ipc_bufs[(size_t)op.buffer * W + ctx->dev[op.src].rank];
+        if (!src) MM_FAIL(MM_EINVAL, "run: rank %d has no buffer %d", ctx->dev[op.src].rank, op.buffer);
+        CU_OK(cudaMemcpyAsync(dst, src + op.r.begin * eb, bytes, cudaMemcpyDefault, s));
+        st->xfer_bytes += (int64_t)bytes;
+      }
+    } else if (op.kind == MM_OPK_FLUSH) {
+      const int64_t eb = app.buffers[op.buffer].first;
+      const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
+      mm_status fs;
+      char* host = static_cast<char*>(flush_target(ctx, plan, o, op.buffer,
+                                                   (size_t)(app.buffers[op.buffer].second * eb), &fs));
+      if (fs) return fs;
+      const char* src = static_cast<const char*>(buffers[(size_t)op.buffer * G + d]) + op.r.begin * eb;
+      CU_OK(cudaMemcpyAsync(host + op.r.begin * eb, src, bytes, cudaMemcpyDeviceToHost, s));
+      st->d2h_bytes += (int64_t)bytes;
+    }
+    if (plan.needs_event[i]) CU_OK(cudaEventRecord(rt->ev[i], s));
+    if (rt->remote_sig[i]) CU_OK(ipc_signal(ch->flags, kIpcOp0 + (int64_t)i, s));
+  }
+  // run end: every stream joined, then this rank's end flag
+  if (mm_status r = join_to_root(rt->join_ev.data())) return r;
+  CU_OK(ipc_signal(ch->flags, kIpcEnd, rs));
   return MM_OK;
 }
 
@@ -1048,6 +1206,14 @@ mm_status mm_nccl_unique_id(void* out128) {
   return MM_OK;
 }
 
+mm_status mm_rendezvous_id(void* out128) {
+  if (!out128) MM_FAIL(MM_EINVAL, "null out");
+  std::random_device rd;
+  uint32_t* o = static_cast<uint32_t*>(out128);
+  for (int i = 0; i < 32; ++i) o[i] = rd();
+  return MM_OK;
+}
+
 mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, int32_t world,
                         const void* nccl_id, mm_ctx** out) {
   if (!devs || !out || G < 1 || G > MM_MAX_DEV || world < 1 || my_rank < 0 || my_rank >= world)
@@ -1172,7 +1338,17 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       rq.sms = (int32_t)rest.sm.smCount;
     }
   }
-  if (world > 1) {
+  const char* tr = getenv("MM_TRANSPORT");
+  if (world > 1 && !(tr && std::strcmp(tr, "nccl") == 0)) {
+    // IPC transport (default): shared-memory rendezvous + CUDA IPC pulls/flags
+    if (!nccl_id) MM_FAIL(MM_EINVAL, "multi-process ctx needs a 128-byte rendezvous id");
+    const int32_t me = first_owned(ctx);
+    CU_OK(cudaSetDevice(ctx->dev[me].phys));
+    ctx->ipc = new (std::nothrow) IpcChannel();
+    if (!ctx->ipc) MM_FAIL(MM_ENOMEM, "ipc channel");
+    mm_status st = ipc_open(ctx->ipc, nccl_id, my_rank, world);
+    if (st) return st;
+  } else if (world > 1) {
     if (!nccl_id) MM_FAIL(MM_EINVAL, "multi-process ctx needs an NCCL unique id");
     if (!nccl().ok) MM_FAIL(MM_ENCCL, "libnccl.so.2 could not be loaded");
     ncclUniqueId id;
@@ -1203,6 +1379,14 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
 
 void mm_ctx_destroy(mm_ctx* ctx) {
   if (!ctx) return;
+  if (ctx->ipc && ctx->ipc->shm) {   // collective: no rank unmaps while a peer may still pull from it
+    const int32_t me = first_owned(ctx);
+    if (me >= 0) {
+      set_dev(ctx, me);
+      cudaDeviceSynchronize();
+    }
+    ipc_barrier(ctx->ipc);
+  }
   for (auto& r : ctx->dev) {
     if (!r.mine) continue;
     cudaSetDevice(r.phys);
@@ -1216,6 +1400,10 @@ void mm_ctx_destroy(mm_ctx* ctx) {
     if (d < ctx->ext_ev.size() && ctx->ext_ev[d]) cudaEventDestroy(ctx->ext_ev[d]);
     if (d < ctx->lib_ev.size() && ctx->lib_ev[d]) cudaEventDestroy(ctx->lib_ev[d]);
     if (r.gctx) drv().GreenCtxDestroy(r.gctx);
+  }
+  if (ctx->ipc) {
+    ipc_close(ctx->ipc);
+    delete ctx->ipc;
   }
   if (ctx->comm) nccl().CommDestroy(ctx->comm);
   if (ctx->bar_buf) cudaFree(ctx->bar_buf);
@@ -1359,7 +1547,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   mm_run_stats* S = st ? st : &local;
   *S = mm_run_stats{};
   const bool timing = o && o->time_kernels;
-  const bool graph = o && o->use_graph && !timing && ctx->world == 1;
+  const bool graph = o && o->use_graph && !timing && (ctx->world == 1 || ctx->ipc);
   mm_status r = ensure_rt(ctx, plan, timing);
   if (r) return r;
   if ((r = join_external(ctx, true))) return r;
@@ -1390,6 +1578,11 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     return MM_OK;
   }
   rt->last_adaptive = false;
+  if (ctx->ipc) {   // every rank's buffers, mapped into this process (host barrier)
+    std::vector<void*> mine(plan.app.buffers.size(), nullptr);
+    for (size_t b = 0; b < mine.size(); ++b) mine[b] = buffers[b * (size_t)ctx->G + root];
+    if ((r = ipc_exchange_buffers(ctx->ipc, mine, ctx->ipc_bufs))) return r;
+  }
   if (graph) {
     // Everything the captured graph bakes in is part of its key: the app
     // buffers, each device's library scratch (operand splits, split-K
@@ -1412,6 +1605,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     for (size_t b = 0; b < plan.app.buffers.size(); ++b)
       key.push_back(o && o->host ? o->host[b] : nullptr);
     for (void* p : ctx->flush_scratch) key.push_back(p);
+    for (char* p : ctx->ipc_bufs) key.push_back(p);
     if (!rt->gexec || key != rt->graph_bufs) {
       if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
       if (rt->graph) cudaGraphDestroy(rt->graph);
@@ -1421,7 +1615,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       CU_OK(cudaStreamBeginCapture(rs, cudaStreamCaptureModeThreadLocal));
       mm_run_stats cap{};
       const int64_t l0 = g_kernel_launches.load();
-      r = issue_local(ctx, plan, buffers, o, false, &cap);
+      r = ctx->ipc ? issue_ipc(ctx, plan, buffers, o, false, &cap) : issue_local(ctx, plan, buffers, o, false, &cap);
       const int64_t captured = g_kernel_launches.load() - l0;
       g_kernel_launches.fetch_sub(captured, std::memory_order_relaxed);   // counted per replay
       cudaGraph_t g = nullptr;
@@ -1454,6 +1648,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     CU_OK(cudaEventRecord(rt->t_start, rs));
     const int64_t l0 = g_kernel_launches.load();
     if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
+    else if (ctx->ipc) r = issue_ipc(ctx, plan, buffers, o, timing, S);
     else r = issue_dist(ctx, plan, buffers, o, timing, S);
     S->n_launches = g_kernel_launches.load() - l0;
     if (r) return r;
@@ -1522,7 +1717,21 @@ mm_status mm_tune_chunks(mm_ctx* ctx, const mm_app* app, const mm_profile* prof,
     std::sort(v.begin(), v.end());
     t[c] = v[v.size() / 2];
   }
-  if (ctx->world > 1) {   // every rank must pick the same candidate: max over ranks
+  if (ctx->ipc) {   // every rank must pick the same candidate: max over ranks
+    std::vector<uint64_t> row(n), all;
+    for (int32_t c = 0; c < n; ++c) std::memcpy(&row[c], &t[c], 8);
+    for (int32_t c0 = 0; c0 < n; c0 += 64) {
+      const int32_t m = std::min<int32_t>(64, n - c0);
+      mm_status st = ipc_allgather_u64(ctx->ipc, row.data() + c0, m, all);
+      if (st) return st;
+      for (int32_t q = 0; q < ctx->world; ++q)
+        for (int32_t c = 0; c < m; ++c) {
+          double v;
+          std::memcpy(&v, &all[(size_t)q * m + c], 8);
+          t[c0 + c] = std::max(t[c0 + c], v);
+        }
+    }
+  } else if (ctx->world > 1) {   // every rank must pick the same candidate: max over ranks
     const int32_t me = first_owned(ctx);
     CU_OK(cudaSetDevice(ctx->dev[me].phys));
     double* dbuf = nullptr;
@@ -1742,7 +1951,27 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
   } catch (const std::bad_alloc&) {
     MM_FAIL(MM_ENOMEM, "profile: host memory");
   }
-  if (ctx->world > 1) {
+  if (ctx->ipc) {
+    // exchange the per-device rows so every rank holds the same profile
+    const int32_t me = first_owned(ctx);
+    const int32_t rowlen = 2 * MM_MAX_K + 1;
+    for (int32_t k = 0; k < MM_MAX_K; ++k) {
+      row[k] = out->fs_item[me][k];
+      row[MM_MAX_K + k] = out->chunk_est_ns[me][k];
+    }
+    row[2 * MM_MAX_K] = out->link_Bps[me];
+    std::vector<uint64_t> all;
+    mm_status st = ipc_allgather_u64(ctx->ipc, row.data(), rowlen, all);
+    if (st) return st;
+    for (int32_t d = 0; d < G; ++d) {
+      const uint64_t* rr = all.data() + (size_t)ctx->dev[d].rank * rowlen;
+      for (int32_t k = 0; k < MM_MAX_K; ++k) {
+        out->fs_item[d][k] = rr[k];
+        out->chunk_est_ns[d][k] = rr[MM_MAX_K + k];
+      }
+      out->link_Bps[d] = rr[2 * MM_MAX_K];
+    }
+  } else if (ctx->world > 1) {
     // exchange the per-device rows so every rank holds the same profile
     const int32_t me = first_owned(ctx);
     const size_t rowlen = 2 * MM_MAX_K + 1;

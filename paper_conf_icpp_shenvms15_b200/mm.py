@@ -177,6 +177,7 @@ _SIGS = {
     "mm_plan_owners": [_P, C.c_int32, C.POINTER(mm_range), C.POINTER(C.c_int32), C.c_int64,
                        C.POINTER(C.c_int64)],
     "mm_nccl_unique_id": [C.c_void_p],
+    "mm_rendezvous_id": [C.c_void_p],
     "mm_ctx_create": [C.POINTER(mm_device_spec), C.c_int32, C.c_int32, C.c_int32, C.c_void_p, C.POINTER(_P)],
     "mm_ctx_stream": [_P, C.c_int32, C.POINTER(_P)],
     "mm_ctx_sm_count": [_P, C.c_int32, C.POINTER(C.c_int32)],
@@ -456,6 +457,13 @@ def mm_plan_owners(plan: int, slot: int) -> List[Tuple[int, int, int]]:
     oo = (C.c_int32 * max(1, n.value))()
     _call("mm_plan_owners", plan, slot, rr, oo, n.value, C.byref(n))
     return [(rr[i].begin, rr[i].end, oo[i]) for i in range(n.value)]
+
+
+def mm_rendezvous_id() -> bytes:
+    """128 random bytes naming a multi-process context (IPC transport)."""
+    buf = C.create_string_buffer(128)
+    _call("mm_rendezvous_id", buf)
+    return buf.raw
 
 
 def mm_nccl_unique_id() -> bytes:

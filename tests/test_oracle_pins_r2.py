@@ -208,3 +208,79 @@ def test_pipelined_staged_program_moves_each_element_once(P, passes):
             d, lo, hi = o[1], o[3], o[4]
             later = [k for (k, b, e) in last_kernel[d] if k > i and b < hi and lo < e]
             assert not later
+
+
+# ------------------------------------------------------------ DP-Dep (R30) --
+# Hand-traced chains of the 3 x 3-tile Cholesky DAG.  Creation order (P119
+# breadth-first; loop nest k, then TRSM i, SYRK i, GEMM j<i):
+#   t0 POTRF(0)  t1 TRSM(1,0)  t2 TRSM(2,0)  t3 SYRK(1,0)  t4 SYRK(2,0)
+#   t5 GEMM(2,1,0)  t6 POTRF(1)  t7 TRSM(2,1)  t8 SYRK(2,1)  t9 POTRF(2)
+# t0 new chain; t1 continues t0 (RAW on tile 00); t2: t0 closed -> new chain;
+# t3 continues t1 (RAW 10); t4 continues t2 (RAW 20); t5: t1, t2 closed ->
+# new chain; t6 continues t3 (WAW 11); t7 continues t5 (WAW 21); t8 continues
+# t4 (WAW 22); t9 continues t8 (WAW 22).
+DP_DEP_CHOL3 = {2: [0, 0, 1, 0, 1, 0, 0, 0, 1, 1],
+                3: [0, 0, 1, 0, 1, 2, 0, 2, 1, 1]}
+
+
+@pytest.mark.parametrize("G", [2, 3])
+def test_dp_dep_cholesky_chains_by_hand(G):
+    _, dev = oc.dp_dep(oa.cholesky_tasks(3, 1), G)
+    assert dev == DP_DEP_CHOL3[G]
+
+
+def test_dp_dep_cholesky_shards_and_keeps_tiles():
+    # T = 8 over 4 devices: every device gets work, and every tile stays on
+    # the device of its first writer (WAW chains never break)
+    app = oa.cholesky_tasks(8, 1)
+    tasks, dev = oc.dp_dep(app, 4)
+    assert sorted(set(dev)) == [0, 1, 2, 3]
+    owner = {}
+    for t, d in zip(tasks, dev):
+        owner.setdefault(t.ij, d)
+        assert owner[t.ij] == d
+
+
+def test_dp_dep_cpp_matches_hand_chains():
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    for G in (2, 3):
+        app = mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [3 * 32, 32])
+        prof = mm.make_profile(G, [[1000] * 4] * G, [[1000] * 4] * G, [10 ** 9] * G)
+        plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_DP_DEP))
+        assert [c.device for c in mm.mm_plan_chunks(plan)] == DP_DEP_CHOL3[G]
+        mm.mm_plan_destroy(plan)
+        mm.mm_app_destroy(app)
+
+
+# ------------------------------------------------- DP-Perf busy lanes (R31) --
+# 3 x 3 tiles, one device, per-task estimates POTRF 100, TRSM 10, SYRK 1,
+# GEMM 1 ns; POTRF/TRSM on lane 1, SYRK/GEMM on lane 0, each lane its own
+# busy time (same task order t0..t9 as above).  By hand:
+#   t0 POTRF(0)  lane1: 0 + 100                          = 100
+#   t1 TRSM(1,0) lane1: max(100, ready 100) + 10         = 110
+#   t2 TRSM(2,0) lane1: max(110, 100) + 10               = 120
+#   t3 SYRK(1,0) lane0: max(0, ready t1 110) + 1         = 111
+#   t4 SYRK(2,0) lane0: max(111, ready t2 120) + 1       = 121
+#   t5 GEMM(2,1) lane0: max(121, ready 120) + 1          = 122
+#   t6 POTRF(1)  lane1: max(120, ready t3 111) + 100     = 220
+#   t7 TRSM(2,1) lane1: max(220, ready t6 220, t5 122) + 10 = 230
+#   t8 SYRK(2,1) lane0: max(122, ready t7 230, t4 121) + 1  = 231
+#   t9 POTRF(2)  lane1: max(230, ready t8 231) + 100     = 331
+DP_PERF_LANES_FIN = [100, 110, 120, 111, 121, 122, 220, 230, 231, 331]
+
+
+def test_dp_perf_lanes_by_hand():
+    app = oa.cholesky_tasks(3, 1)
+    prof = oc.Profile(G=1, fs_item=[[1] * 4], chunk_est_ns=[[100, 10, 1, 1]], link_Bps=[10 ** 9])
+    _, dev, fin = oc.dp_perf(app, prof)
+    assert dev == [0] * 10 and fin == DP_PERF_LANES_FIN
+
+
+def test_dp_perf_lanes_cpp_matches_hand():
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    app = mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [3 * 32, 32])
+    prof = mm.make_profile(1, [[1] * 4], [[100, 10, 1, 1]], [10 ** 9])
+    plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_DP_PERF))
+    assert [c.finish_ns for c in mm.mm_plan_chunks(plan)] == DP_PERF_LANES_FIN
+    mm.mm_plan_destroy(plan)
+    mm.mm_app_destroy(app)
