@@ -130,7 +130,9 @@ def cholesky_exact_factor(n: int, band: int = 4, seed: int = SEED):
     for d in range(1, band + 1):
         off = integers(n - d, AID_CHOL_L + 100 + d, -1, 1, seed)
         L[i[d:], i[:-d]] = off
-    A = L @ L.T  # integer input construction (not the method)
+    Lf = L.astype(np.float64)
+    A = (Lf @ Lf.T).astype(np.int64)  # integer input construction (not the method); every
+    # product and partial sum is an integer far below 2**53, so FP64 BLAS is exact
     assert np.abs(A).max() < 2 ** 24
     return A.astype(np.float32), L.astype(np.float32)
 

