@@ -28,6 +28,7 @@
 #include <vector>
 
 #include "kernels.h"
+#include "tc_ptx.h"
 
 namespace mm {
 
@@ -35,6 +36,8 @@ cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner,
                                uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
 
 namespace {
+
+using namespace tcx;
 
 // BN = 256 (the default tile), or 64 for plain SGEMMs too small to give
 // every SM a 128 x 256 tile (BASELINE configs[0], 1024^2: 32 -> 128 tiles).
@@ -63,52 +66,6 @@ struct GemmJob {
   int32_t ti[kCholBatch], tj[kCholBatch];
 };
 
-__device__ __forceinline__ uint32_t saddr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t c) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(saddr(b)), "r"(c));
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(saddr(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(saddr(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n"
-      "W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}\n" ::"r"(saddr(b)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int32_t x, int32_t y, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          saddr(dst)),
-      "l"((uint64_t)map), "r"(x), "r"(y), "r"(saddr(bar))
-      : "memory");
-}
-// UMMA shared-memory descriptor: K-major, SWIZZLE_64B (rows of 64 B, 8-row
-// core-matrix groups 512 B apart).
-__device__ __forceinline__ uint64_t sdesc(const void* p) {
-  const uint64_t a = saddr(p);
-  uint64_t d = (a >> 4) & 0x3FFFull;         // start address
-  d |= 1ull << 16;                           // leading byte offset (unused for swizzled K-major)
-  d |= (uint64_t)(512 >> 4) << 32;           // stride byte offset
-  d |= 1ull << 46;                           // descriptor version (sm_100)
-  d |= 4ull << 61;                           // SWIZZLE_64B
-  return d;
-}
-__device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
-      " tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-      "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-__device__ __forceinline__ void mma_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(saddr(bar))
-               : "memory");
-}
 
 // Operand coordinates and output of tile `tile` (task-major, n fastest).
 struct TileGeo {
@@ -147,36 +104,6 @@ __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int ti
   return g;
 }
 
-__device__ __forceinline__ uint32_t peer_addr(const void* p, uint32_t rank) {   // shared::cluster address in CTA `rank`
-  uint32_t a;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(a) : "r"(saddr(p)), "r"(rank));
-  return a;
-}
-// Pair-mode TMA: data into this CTA's smem, completion bytes on the leader's barrier.
-__device__ __forceinline__ void tma_load_2d_pair(void* dst, const CUtensorMap* map, int32_t x, int32_t y,
-                                                 uint32_t bar_cluster) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3}], [%4];" ::"r"(saddr(dst)),
-      "l"((uint64_t)map), "r"(x), "r"(y), "r"(bar_cluster)
-      : "memory");
-}
-__device__ __forceinline__ void mma_tf32_pair(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
-      " tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-      "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-__device__ __forceinline__ void mma_commit_pair(uint64_t* bar) {   // arrive on `bar` in both CTAs
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
-          saddr(bar)),
-      "h"((uint16_t)0x3)
-      : "memory");
-}
-__device__ __forceinline__ void cluster_sync_all() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n barrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
 
 template <int BN, bool PAIR> constexpr int gemm_stages() { return PAIR ? 6 : kStages; }
 template <int BN, bool PAIR> constexpr int gemm_stage_bytes() {
@@ -427,16 +354,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreadsGemm, 1)
   gemm_body<BN, true>(tAhi, tAlo, tBhi, tBlo, C, N, row0, mrows, nkb, npairs, job);
 }
 
-__device__ __forceinline__ float tf32_rn(float x) {
-  uint32_t r;
-  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
-  return __uint_as_float(r);
-}
-
-__device__ __forceinline__ void split2(float x, float& h, float& l) {
-  h = tf32_rn(x);
-  l = tf32_rn(x - h);
-}
 
 // One launch for both SGEMM operands: blocks [0, nblk_a) split A rows
 // [r0, r0+mrows) into hi/lo (row stride Kp, zero padding K..Kp; float4 when
@@ -769,11 +686,22 @@ size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
   return (size_t)(2 * mrows * Kp + 2 * N * Kp + (S > 1 ? S * mrows * N : 0)) * sizeof(float);
 }
 
+int sgemm_fused_splits(const float* A, const float* B, float* C, int64_t mrows, int64_t N, int64_t K, int64_t r0);
+cudaError_t sgemm_fused_rows(const float* A, const float* B, float* C, int64_t N, int64_t K, int64_t r0,
+                             int64_t mrows, int S, cudaStream_t s);
+
 cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
                               int64_t r0, int64_t r1, cudaStream_t s, int sms, Scratch* scr, bool b_readonly) {
   (void)M;
   const int64_t mrows = r1 - r0;
   if (mrows <= 0 || N <= 0) return cudaSuccess;
+  if ((sms <= 0 || sms >= 148) && use_mc_env()) {
+    // too few tile pairs for the GPU: ONE launch that splits the raw operands
+    // in shared memory and reduces its K splits inside the cluster
+    // (kernels_sgemm_fused.cu) instead of split -> GEMM -> reduce below
+    const int S = sgemm_fused_splits(A, B, C, mrows, N, K, r0);
+    if (S > 1) return sgemm_fused_rows(A, B, C, N, K, r0, mrows, S, s);
+  }
   if (!scr || !scr->ptr || scr->bytes < sgemm_tf32x3_scratch(N, K, mrows)) return cudaErrorNotSupported;
   const int64_t Kp = (K + KPAD - 1) / KPAD * KPAD;
   // scratch layout: [B_hi^T | B_lo^T] (N x Kp each) then [A_hi | A_lo] (mrows x Kp each)

@@ -1,0 +1,427 @@
+// Small-SGEMM path of MatrixMul (BASELINE configs[0], 1024^2; P311 C = A x B,
+// row-wise split) in ONE launch: no operand-split pass, no reduction pass.
+//
+// A cluster of 2 S CTAs computes one 256 x 256 output tile pair over S K
+// splits (S in 2..4, chosen so that every cluster is resident at once): CTA
+// rank r = 2 z + h is half h (128 rows) of the 2-SM pair (tcgen05
+// cta_group::2) of K split z (k-blocks [z nkb / S, (z+1) nkb / S)).
+//  warp 0      TMA producer: RAW fp32 tiles straight from A (row-major,
+//              K-major: box 16 x 128 rows, SWIZZLE_64B) and B (row-major:
+//              four boxes of 32 columns x 16 k-rows, SWIZZLE_128B) into a
+//              4-stage raw ring.
+//  warps 2-5   converters: x -> hi = tf32_rn(x), lo = tf32_rn(x - hi) (the
+//              split of the two-pass path) into a 4-stage split ring — A in
+//              place of its swizzled layout, B transposed on the way into
+//              the K-major SWIZZLE_64B layout of the two-pass path's B^T (an
+//              MN-major B descriptor read zeros on this B200); proxy fence;
+//              one arrival per warp on the leader CTA's stage barrier.
+//  warp 1      (leader CTA) tcgen05.mma.cta_group::2.kind::tf32, 3 MMAs per
+//              k-step (lo.hi + hi.lo + hi.hi) into a 256-column TMEM
+//              accumulator; commits free the split stages of both CTAs.
+//  epilogue    warps 2-5: TMEM -> registers -> this CTA's smem (padded
+//              rows); cluster barrier; CTA z sums float4 columns
+//              [z 64 / S, (z+1) 64 / S) of its 128 rows over the S partials in
+//              split order ((p0 + p1) + p2) + p3 by distributed-shared-memory
+//              loads from its cluster peers and stores C; cluster barrier
+//              before exit.
+// Measured (1024^2, S = 3: 16 clusters of 6 CTAs; 8-CTA clusters fit only 15
+// at a time): ~0.7 us set-up, ~14 us main loop (shared-memory traffic of the
+// in-place split + transposition on top of the MMA operand reads), ~1 us
+// TMEM -> smem, ~4.5 us reduction (DSMEM moves ~20 B/clk per SM; a push of
+// the partial slices by cp.async.bulk and a reduction through L2 were both
+// slower).
+#include <cuda.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdlib>
+
+#include "kernels.h"
+#include "tc_ptx.h"
+
+namespace mm {
+
+cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                               uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
+
+namespace {
+
+using namespace tcx;
+
+constexpr int FBM = 128, FBK = 16, FHALF = 128;                // rows per CTA, k per stage, B columns per CTA
+constexpr int kRawStages = 4, kSplitStages = 4, kFThreads = 192;
+constexpr int RAW_A = FBM * FBK * 4, RAW_B = FHALF * FBK * 4;  // 8 KB + 8 KB
+constexpr int RAW_BYTES = RAW_A + RAW_B;
+constexpr int SPLIT_BYTES = 2 * RAW_BYTES;                     // A_hi, A_lo, B_hi, B_lo
+constexpr int kRingBytes = kRawStages * RAW_BYTES + kSplitStages * SPLIT_BYTES;   // 192 KB
+constexpr int RED_LD = 256 + 4;        // padded fp32 row of the partial (reuses the drained rings)
+constexpr int kFusedSmem = kRingBytes + 1024 + 256;
+static_assert(FBM * RED_LD * 4 <= kRingBytes, "partial buffer");
+
+// arrive on the barrier of cluster peer `rank` (default .release.cta
+// semantics, as CUTLASS's ClusterBarrier::arrive(cta_id): a .cluster-scope
+// release compiles to a GPU-wide MEMBAR per arrival)
+__device__ __forceinline__ void arrive_remote(uint64_t* bar, uint32_t rank) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(peer_addr(bar, rank)) : "memory");
+}
+
+__device__ __forceinline__ void cluster_arrive_relaxed_wait() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;\n barrier.cluster.wait.aligned;" ::: "memory");
+}
+
+// tcgen05.commit of the pair's MMAs: arrive on `bar` in both CTAs of the pair
+// (cluster ranks pair0, pair0 + 1)
+__device__ __forceinline__ void commit_pair_at(uint64_t* bar, uint32_t pair0) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          saddr(bar)),
+      "h"((uint16_t)(0x3u << pair0))
+      : "memory");
+}
+
+// mbarrier wait that fails (trap -> launch error) instead of hanging if a
+// phase never completes (a lost arrival would otherwise wedge the GPU)
+template <bool CLUSTER = false>
+__device__ __forceinline__ uint32_t try_wait(uint64_t* b, uint32_t parity) {
+  uint32_t done;
+  if (CLUSTER)
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n"
+        " selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(saddr(b)), "r"(parity)
+        : "memory");
+  else
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(saddr(b)), "r"(parity)
+        : "memory");
+  return done;
+}
+
+template <bool CLUSTER = false>
+__device__ __forceinline__ void fwait(uint64_t* b, uint32_t parity) {
+  if (try_wait<CLUSTER>(b, parity)) return;
+  uint64_t t0;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    if (try_wait<CLUSTER>(b, parity)) return;
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 4000000000ull) __trap();
+  }
+}
+
+__device__ __forceinline__ float4 ld_dsmem_f4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(addr)
+               : "memory");
+  return v;
+}
+
+// One 256 x 256 tile pair, K split z of S (k-blocks [z nkb / S, (z+1) nkb / S));
+// cluster = 2 S CTAs.
+__global__ void __launch_bounds__(kFThreads, 1)
+    sgemm_fused(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB, float* __restrict__ C,
+                int64_t N, int64_t row0, int64_t mrows, int nblk, int S, int nkb_all) {
+  uint32_t rank;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const uint32_t h = rank & 1u, z = rank >> 1;
+  const bool leader = h == 0;
+  const int cl = (int)(blockIdx.x / (2 * S));
+  const int mp = cl / nblk, nb = cl % nblk;
+  const int m_blk = 2 * mp + (int)h;
+  const int kb0 = (int)z * nkb_all / S, nkb = ((int)z + 1) * nkb_all / S - kb0;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* raw = base;
+  uint8_t* spl = base + kRawStages * RAW_BYTES;
+  uint64_t* raw_full = reinterpret_cast<uint64_t*>(base + kRingBytes);
+  uint64_t* raw_empty = raw_full + kRawStages;
+  uint64_t* split_full = raw_empty + kRawStages;   // leader: the 4 converter warps of both CTAs
+  uint64_t* split_empty = split_full + kSplitStages;
+  uint64_t* tfull = split_empty + kSplitStages;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < kRawStages; ++s) {
+      mbar_init(&raw_full[s], 1);
+      mbar_init(&raw_empty[s], 4);          // the 4 converter warps of this CTA
+    }
+    for (int s = 0; s < kSplitStages; ++s) {
+      mbar_init(&split_full[s], 8);
+      mbar_init(&split_empty[s], 1);        // the leader's commit, multicast
+    }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tB) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(saddr(tslot)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  cluster_arrive_relaxed_wait();   // peers' barriers initialised (fence.mbarrier_init above)
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tslot;
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+
+  if (warp == 0) {
+    if (lane == 0) {   // ===== producer: raw tiles of this CTA (own barrier)
+      const int32_t ya = m_blk * FBM;
+      const int32_t xb = nb * 256 + (int32_t)h * FHALF;
+      for (int i = 0; i < nkb; ++i) {
+        const int s = i % kRawStages;
+        if (i >= kRawStages) fwait(&raw_empty[s], (uint32_t)(((i / kRawStages) - 1) & 1));
+        uint8_t* st = raw + s * RAW_BYTES;
+        const int32_t kx = (kb0 + i) * FBK;
+        mbar_expect_tx(&raw_full[s], RAW_BYTES);
+        tma_load_2d(st, &tA, kx, ya, &raw_full[s]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) tma_load_2d(st + RAW_A + j * 2048, &tB, xb + 32 * j, kx, &raw_full[s]);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0 && leader) {   // ===== MMA issuer
+      const uint32_t idesc = (1u << 4)                 // D: fp32
+                             | (2u << 7) | (2u << 10)  // A, B: tf32
+                             | ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+      for (int i = 0; i < nkb; ++i) {
+        const int s = i % kSplitStages;
+        fwait(&split_full[s], (uint32_t)((i / kSplitStages) & 1));
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        uint8_t* st = spl + s * SPLIT_BYTES;
+        const uint64_t ahi = sdesc(st), alo = sdesc(st + RAW_A);
+        const uint64_t bhi = sdesc(st + 2 * RAW_A), blo = sdesc(st + 2 * RAW_A + RAW_B);
+#pragma unroll
+        for (int kk = 0; kk < FBK / 8; ++kk) {
+          const uint64_t adv = (uint64_t)(kk * 32) >> 4;     // 8 fp32 along K inside the 64-B row
+          mma_tf32_pair(tmem, alo + adv, bhi + adv, idesc, (i | kk) != 0);
+          mma_tf32_pair(tmem, ahi + adv, blo + adv, idesc, 1u);
+          mma_tf32_pair(tmem, ahi + adv, bhi + adv, idesc, 1u);
+        }
+        commit_pair_at(&split_empty[s], rank);
+      }
+      commit_pair_at(tfull, rank);
+    }
+    __syncwarp();
+  } else {   // ===== converters, then the epilogue (warps 2..5)
+    const int ct = threadIdx.x - 64;   // 0..127
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % kRawStages, q = i % kSplitStages;
+      fwait(&raw_full[s], (uint32_t)((i / kRawStages) & 1));
+      if (i >= kSplitStages) fwait(&split_empty[q], (uint32_t)(((i / kSplitStages) - 1) & 1));
+      const uint8_t* rs = raw + s * RAW_BYTES;
+      uint8_t* dst = spl + q * SPLIT_BYTES;
+      // A: 512 float4 of the K-major SWIZZLE_64B tile, split in place
+      float4 v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) v[j] = reinterpret_cast<const float4*>(rs)[ct + 128 * j];
+      // B: the raw tile is MN-major (4 boxes of 16 k-rows x 32 columns,
+      // SWIZZLE_128B: 16-B chunk c of row k stored at chunk c ^ (k & 7)); it is
+      // transposed into the K-major SWIZZLE_64B layout the MMA reads (row n =
+      // 64 B of 16 k, chunk c stored at c ^ ((n >> 1) & 3)).  Output float4 o:
+      // n = o & 127, k = 4 (o >> 7) .. +3; a warp reads 32 consecutive columns
+      // of one raw row per load (conflict-free).
+      float4 w[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int o = ct + 128 * j, n = o & 127, k0 = 4 * (o >> 7);
+        const uint8_t* box = rs + RAW_A + (n >> 5) * 2048 + (n & 3) * 4;
+        const int c16 = (n & 31) >> 2;
+        float t[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int k = k0 + u;
+          t[u] = *reinterpret_cast<const float*>(box + k * 128 + ((c16 ^ (k & 7)) << 4));
+        }
+        w[j] = make_float4(t[0], t[1], t[2], t[3]);
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float4 hi, lo;
+        split2(v[j].x, hi.x, lo.x);
+        split2(v[j].y, hi.y, lo.y);
+        split2(v[j].z, hi.z, lo.z);
+        split2(v[j].w, hi.w, lo.w);
+        reinterpret_cast<float4*>(dst)[ct + 128 * j] = hi;
+        reinterpret_cast<float4*>(dst + RAW_A)[ct + 128 * j] = lo;
+        const int o = ct + 128 * j, n = o & 127, kc4 = o >> 7;
+        const int boff = n * 64 + ((kc4 ^ ((n >> 1) & 3)) << 4);
+        split2(w[j].x, hi.x, lo.x);
+        split2(w[j].y, hi.y, lo.y);
+        split2(w[j].z, hi.z, lo.z);
+        split2(w[j].w, hi.w, lo.w);
+        *reinterpret_cast<float4*>(dst + 2 * RAW_A + boff) = hi;
+        *reinterpret_cast<float4*>(dst + 2 * RAW_A + RAW_B + boff) = lo;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> tensor-core reads
+      __syncwarp();
+      if (lane == 0) {
+        mbar_arrive(&raw_empty[s]);
+        if (leader) mbar_arrive(&split_full[q]);
+        else arrive_remote(&split_full[q], rank ^ 1u);
+      }
+    }
+    // ---- epilogue: accumulator (TMEM lanes 32 grp .. +32 = this warp's rows)
+    const int grp = warp & 3;
+    fwait(tfull, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int r = grp * 32 + lane;                       // row within the CTA's 128
+    const int64_t grow = (int64_t)m_blk * FBM + r;       // row within [row0, row0 + mrows)
+    float* red = reinterpret_cast<float*>(base);         // all rings drained: reuse for the partial
+    for (int c = 0; c < 256; c += 16) {
+      uint32_t v[16];
+      const uint32_t ta = tmem + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+          : "r"(ta));
+      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      if (S > 1) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          *reinterpret_cast<float4*>(red + r * RED_LD + c + 4 * q) =
+              make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]), __uint_as_float(v[4 * q + 2]),
+                          __uint_as_float(v[4 * q + 3]));
+      } else if (grow < mrows) {
+        const int64_t n0 = (int64_t)nb * 256 + c;
+        float* crow = C + (row0 + grow) * N;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (n0 + 4 * q < N)
+            *reinterpret_cast<float4*>(crow + n0 + 4 * q) =
+                make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]),
+                            __uint_as_float(v[4 * q + 2]), __uint_as_float(v[4 * q + 3]));
+      }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  }
+  __syncthreads();
+  if (S > 1) {
+    cluster_sync_all();   // every partial of the cluster is in shared memory
+    // CTA z reduces float4 columns [z 64 / S, (z+1) 64 / S) of its 128 rows:
+    // the S partial loads of an element issued before the adds, summed in
+    // split order ((p0 + p1) + p2) + p3; all 192 threads take part
+    const int c4a = (int)z * 64 / S, c4n = ((int)z + 1) * 64 / S - c4a;
+    const float* red = reinterpret_cast<const float*>(base);
+    uint32_t peer[4];
+#pragma unroll
+    for (int zz = 0; zz < 4; ++zz) peer[zz] = peer_addr(red, (uint32_t)(2 * (zz < S ? zz : 0)) + h);
+    for (int e = threadIdx.x; e < FBM * c4n; e += kFThreads) {
+      const int rr = e / c4n, cc = 4 * (c4a + e % c4n);
+      const uint32_t off = (uint32_t)((rr * RED_LD + cc) * 4);
+      float4 p[4];
+#pragma unroll
+      for (int zz = 0; zz < 4; ++zz)
+        if (zz < S) p[zz] = ld_dsmem_f4(peer[zz] + off);
+      float4 a = p[0];
+#pragma unroll
+      for (int zz = 1; zz < 4; ++zz)
+        if (zz < S) {
+          a.x += p[zz].x; a.y += p[zz].y; a.z += p[zz].z; a.w += p[zz].w;
+        }
+      const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * 256 + cc;
+      if (grow < mrows && n0 < N) *reinterpret_cast<float4*>(C + (row0 + grow) * N + n0) = a;
+    }
+    cluster_arrive_relaxed_wait();   // every bulk copy out of this CTA's smem has landed
+  } else {
+    cluster_sync_all();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 256;" ::"r"(tmem));
+  }
+}
+
+}  // namespace
+
+int max_active_clusters(int csize);
+
+// K splits of the fused path for a row range: the largest S <= 4 with at
+// least 8 k-blocks per split whose clusters of 2 S CTAs all fit on the GPU at
+// once (one wave: cudaOccupancyMaxActiveClusters), 0 = use the two-pass path
+// (the tile pairs alone fill the GPU, or the operands are not 16-B aligned).
+int sgemm_fused_splits(const float* A, const float* B, float* C, int64_t mrows, int64_t N, int64_t K, int64_t r0) {
+  static const int env = getenv("MM_SGEMM_FUSED") ? atoi(getenv("MM_SGEMM_FUSED")) : 1;
+  if (!env || (K & 3) || (N & 3)) return 0;
+  if ((reinterpret_cast<uintptr_t>(A + r0 * K) | reinterpret_cast<uintptr_t>(B) | reinterpret_cast<uintptr_t>(C)) & 15)
+    return 0;
+  const int64_t pairs = ((mrows + FBM - 1) / FBM + 1) / 2 * ((N + 255) / 256);
+  const int64_t nkb = (K + FBK - 1) / FBK;
+  if (pairs * 2 > 148 / 2) return 0;   // at least half the GPU in tile pairs already: no K split
+  for (int S = 4; S >= 2; --S)
+    if (nkb / S >= 8 && max_active_clusters(2 * S) >= pairs) return S;
+  return 0;
+}
+
+int max_active_clusters(int csize) {
+  static int cache[9] = {-1, -1, -1, -1, -1, -1, -1, -1, -1};
+  if (csize < 1 || csize > 8) return 0;
+  if (cache[csize] >= 0) return cache[csize];
+  if (cudaFuncSetAttribute(sgemm_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, kFusedSmem) != cudaSuccess ||
+      cudaFuncSetAttribute(sgemm_fused, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+    return 0;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(csize * 16));
+  cfg.blockDim = dim3(kFThreads);
+  cfg.dynamicSmemBytes = kFusedSmem;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)csize;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, (void*)sgemm_fused, &cfg) != cudaSuccess) n = 0;
+  cache[csize] = n;
+  return n;
+}
+
+cudaError_t sgemm_fused_rows(const float* A, const float* B, float* C, int64_t N, int64_t K, int64_t r0,
+                             int64_t mrows, int S, cudaStream_t s) {
+  CUtensorMap tA, tB;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(&tA, A + r0 * K, K, mrows, K * 4, FBK, FBM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tB, B, N, K, N * 4, 32, FBK)) != cudaSuccess) return e;
+  static std::atomic<uint64_t> attr{0};
+  e = once_per_device(attr, [] {
+    cudaError_t r = cudaFuncSetAttribute(sgemm_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, kFusedSmem);
+    if (r != cudaSuccess) return r;
+    return cudaFuncSetAttribute(sgemm_fused, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  });
+  if (e != cudaSuccess) return e;
+  const int mblk = (int)((mrows + FBM - 1) / FBM);
+  const int mpairs = (mblk + 1) / 2;
+  const int nblk = (int)((N + 255) / 256);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(mpairs * nblk * 2 * S));
+  cfg.blockDim = dim3(kFThreads);
+  cfg.dynamicSmemBytes = kFusedSmem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)(2 * S);
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  // programmatic dependent launch: barrier/TMEM set-up overlaps the previous
+  // kernel's tail; the first global access follows griddepcontrol.wait
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  note_launch();
+  return cudaLaunchKernelEx(&cfg, sgemm_fused, tA, tB, C, N, r0, mrows, nblk, S, (int)((K + FBK - 1) / FBK));
+}
+
+}  // namespace mm

@@ -70,6 +70,24 @@ def verdict(order, times):
     return ok, pairs
 
 
+MEM_BOUND = (mm.MM_APP_STREAM, mm.MM_APP_BLACKSCHOLES, mm.MM_APP_HOTSPOT, mm.MM_APP_STENCIL_REDUCTION)
+
+
+def emulation_note(budgets, cls, app_id):
+    """Where a platform of logical devices on ONE B200 distorts an ordering."""
+    notes = []
+    if len(budgets) > 1 and all(b == 0 for b in budgets):
+        notes.append("HOMO: every logical device claims the whole GPU, so concurrent devices contend for the "
+                     "same SMs and HBM; sharding adds transfers without adding hardware (single-GPU artefact)")
+        if cls == mm.MM_MK_DAG:
+            notes.append("MK-DAG: a strategy that keeps the DAG on one device wins by construction here; "
+                         "on separate GPUs it would leave the others idle")
+    elif app_id in MEM_BOUND:
+        notes.append("HET: SMs are partitioned (green contexts) but HBM bandwidth is shared, so memory-bound "
+                     "kernels of the small devices steal bandwidth from the big one (single-GPU artefact)")
+    return "; ".join(notes) or None
+
+
 def run_config(name, app_id, ip, budgets, staged, reps):
     G = len(budgets)
     s = runner.session(app_id, ip, G=G, sm_budgets=budgets)
@@ -77,9 +95,10 @@ def run_config(name, app_id, ip, budgets, staged, reps):
         cls = s.classify()
         ns = mm.mm_needs_sync(s.app)
         order = expected_order(cls, ns)
-        prof = s.profile(reps=3)
-        if staged:
-            prof.staged = 1
+        # Glinda's transfer metric (P49) measured on the link the data crosses:
+        # the pinned host link for staged runs (sets prof.staged), the
+        # device-to-device exchange link for resident ones
+        prof = s.profile(reps=3, link="host" if staged else "peer")
         s.fill()
         host = None
         if staged:
@@ -147,6 +166,8 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 "ranking_holds": ok, "top_choice_holds": top_ok, "pairs": pairs,
                 "dp_perf_adaptive_ms": None if adaptive_ms is None else round(adaptive_ms, 4),
                 "dp_perf_adaptive_task_share": ad_share,
+                "profile_link_Bps": [int(prof.link_Bps[d]) for d in range(G)],
+                "emulation_note": emulation_note(budgets, cls, app_id),
                 "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(G)],
                 "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(G)]}
     finally:
@@ -155,7 +176,7 @@ def run_config(name, app_id, ip, budgets, staged, reps):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r1_ranking.json"))
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r2_ranking.json"))
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quick", action="store_true")
     ap.add_argument("--platforms", default="HET-2,HOMO-2",
