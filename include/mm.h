@@ -229,6 +229,9 @@ typedef struct {
   uint64_t fs_item[MM_MAX_DEV][MM_MAX_K];    /* femtoseconds per item (R_GC)  */
   uint64_t chunk_est_ns[MM_MAX_DEV][MM_MAX_K]; /* DP-Perf estimate per nominal chunk */
   uint64_t link_Bps[MM_MAX_DEV];             /* bytes/s into device d (R_GD)  */
+  uint64_t link_lat_ns[MM_MAX_DEV];          /* fixed cost of one transfer into d (ns):
+                                                DP-Perf prices a pull of B bytes as
+                                                link_lat_ns + ceil(B 1e9 / link_Bps) (R32) */
 } mm_profile;
 
 /* Static split (SP-Single / SP-Unified / SP-Varied): out[k*G + d]. */

@@ -1126,7 +1126,7 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
         uint64_t rr = fin[p.first];
         if (ap.task_dev[p.first] != d) {
           const uint64_t link = std::max<uint64_t>(1, ap.prof.link_Bps[d]);
-          rr += (uint64_t)(((unsigned __int128)p.second * 1000000000ull + link - 1) / link);
+          rr += ap.prof.link_lat_ns[d] + (uint64_t)(((unsigned __int128)p.second * 1000000000ull + link - 1) / link);
         }
         ready = std::max(ready, rr);
       }
@@ -1798,7 +1798,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
   out->G = G;
   out->K = K;
   out->staged = po && po->measure_link == 2 ? 1 : 0;
-  std::vector<uint64_t> row(2 * MM_MAX_K + 1, 0);
+  std::vector<uint64_t> row(2 * MM_MAX_K + 2, 0);
   try {
     for (int32_t d = 0; d < G; ++d) {
       if (!ctx->dev[d].mine) continue;
@@ -1923,27 +1923,36 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
           CU_OK(cudaDeviceSynchronize());
           CU_OK(set_dev(ctx, d));
         }
-        float best = 0.f;
-        for (int32_t i = 0; i < 1 + std::max<int32_t>(reps, 2); ++i) {   // first = warm-up
-          CU_OK(cudaEventRecord(a, s));
-          if (host) {
-            CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyHostToDevice, s));
-            CU_OK(cudaMemcpyAsync(x, y, bytes, cudaMemcpyDeviceToHost, s));
-          } else if (src_phys != ctx->dev[d].phys) {
-            CU_OK(cudaMemcpyPeerAsync(y, ctx->dev[d].phys, x, src_phys, bytes, s));
-          } else {
-            CU_OK(cudaMemcpyAsync(y, x, bytes, cudaMemcpyDeviceToDevice, s));
+        // time `nb` bytes of the link's copy (best of the timed repetitions)
+        auto time_copy = [&](size_t nb, float* best) -> mm_status {
+          *best = 0.f;
+          for (int32_t i = 0; i < 1 + std::max<int32_t>(reps, 2); ++i) {   // first = warm-up
+            CU_OK(cudaEventRecord(a, s));
+            if (host) {
+              CU_OK(cudaMemcpyAsync(y, x, nb, cudaMemcpyHostToDevice, s));
+              CU_OK(cudaMemcpyAsync(x, y, nb, cudaMemcpyDeviceToHost, s));
+            } else if (src_phys != ctx->dev[d].phys) {
+              CU_OK(cudaMemcpyPeerAsync(y, ctx->dev[d].phys, x, src_phys, nb, s));
+            } else {
+              CU_OK(cudaMemcpyAsync(y, x, nb, cudaMemcpyDeviceToDevice, s));
+            }
+            CU_OK(cudaEventRecord(b, s));
+            CU_OK(cudaEventSynchronize(b));
+            float ms = 0.f;
+            CU_OK(cudaEventElapsedTime(&ms, a, b));
+            if (i > 0 && (*best == 0.f || ms < *best)) *best = ms;
           }
-          CU_OK(cudaEventRecord(b, s));
-          CU_OK(cudaEventSynchronize(b));
-          float ms = 0.f;
-          CU_OK(cudaEventElapsedTime(&ms, a, b));
-          if (i > 0 && (best == 0.f || ms < best)) best = ms;
-        }
+          return MM_OK;
+        };
+        float best = 0.f, small = 0.f;
+        if (mm_status r = time_copy(bytes, &best)) return r;
+        // R32: the fixed cost of one transfer = a 4 KiB copy of the same kind
+        if (mm_status r = time_copy(4096, &small)) return r;
         if (host) cudaFreeHost(x);
         else cudaFree(x);
         cudaFree(y);
         out->link_Bps[d] = (uint64_t)((double)(host ? 2 * bytes : bytes) / ((double)best * 1e-3));
+        out->link_lat_ns[d] = (uint64_t)((double)small * 1e6 / (host ? 2.0 : 1.0));
       }
       cudaEventDestroy(a);
       cudaEventDestroy(b);
@@ -1954,12 +1963,13 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
   if (ctx->ipc) {
     // exchange the per-device rows so every rank holds the same profile
     const int32_t me = first_owned(ctx);
-    const int32_t rowlen = 2 * MM_MAX_K + 1;
+    const int32_t rowlen = 2 * MM_MAX_K + 2;
     for (int32_t k = 0; k < MM_MAX_K; ++k) {
       row[k] = out->fs_item[me][k];
       row[MM_MAX_K + k] = out->chunk_est_ns[me][k];
     }
     row[2 * MM_MAX_K] = out->link_Bps[me];
+    row[2 * MM_MAX_K + 1] = out->link_lat_ns[me];
     std::vector<uint64_t> all;
     mm_status st = ipc_allgather_u64(ctx->ipc, row.data(), rowlen, all);
     if (st) return st;
@@ -1970,16 +1980,18 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
         out->chunk_est_ns[d][k] = rr[MM_MAX_K + k];
       }
       out->link_Bps[d] = rr[2 * MM_MAX_K];
+      out->link_lat_ns[d] = rr[2 * MM_MAX_K + 1];
     }
   } else if (ctx->world > 1) {
     // exchange the per-device rows so every rank holds the same profile
     const int32_t me = first_owned(ctx);
-    const size_t rowlen = 2 * MM_MAX_K + 1;
+    const size_t rowlen = 2 * MM_MAX_K + 2;
     for (int32_t k = 0; k < MM_MAX_K; ++k) {
       row[k] = out->fs_item[me][k];
       row[MM_MAX_K + k] = out->chunk_est_ns[me][k];
     }
     row[2 * MM_MAX_K] = out->link_Bps[me];
+    row[2 * MM_MAX_K + 1] = out->link_lat_ns[me];
     uint64_t *dsend = nullptr, *drecv = nullptr;
     CU_OK(set_dev(ctx, me));
     CU_OK(cudaMalloc(&dsend, rowlen * 8));
@@ -1998,6 +2010,7 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
         out->chunk_est_ns[d][k] = rr[MM_MAX_K + k];
       }
       out->link_Bps[d] = rr[2 * MM_MAX_K];
+      out->link_lat_ns[d] = rr[2 * MM_MAX_K + 1];
     }
   }
   return MM_OK;

@@ -81,7 +81,7 @@ class mm_profile(C.Structure):
     _fields_ = [("G", C.c_int32), ("K", C.c_int32), ("staged", C.c_int32), ("_pad", C.c_int32),
                 ("fs_item", (C.c_uint64 * MM_MAX_K) * MM_MAX_DEV),
                 ("chunk_est_ns", (C.c_uint64 * MM_MAX_K) * MM_MAX_DEV),
-                ("link_Bps", C.c_uint64 * MM_MAX_DEV)]
+                ("link_Bps", C.c_uint64 * MM_MAX_DEV), ("link_lat_ns", C.c_uint64 * MM_MAX_DEV)]
 
 
 class mm_plan_opts(C.Structure):
@@ -356,8 +356,10 @@ def mm_rank(cls: int, needs_sync: bool) -> List[int]:
     return list(out[:n.value])
 
 
-def make_profile(G: int, fs_item, chunk_est_ns=None, link_Bps=None, staged: bool = False) -> mm_profile:
-    """Marshal a profile from nested lists fs_item[d][k] (fs), chunk_est_ns[d][k], link_Bps[d]."""
+def make_profile(G: int, fs_item, chunk_est_ns=None, link_Bps=None, staged: bool = False,
+                 link_lat_ns=None) -> mm_profile:
+    """Marshal a profile from nested lists fs_item[d][k] (fs), chunk_est_ns[d][k], link_Bps[d],
+    link_lat_ns[d]."""
     p = mm_profile()
     p.G = G
     p.K = MM_MAX_K
@@ -370,6 +372,8 @@ def make_profile(G: int, fs_item, chunk_est_ns=None, link_Bps=None, staged: bool
                 p.chunk_est_ns[d][k] = int(v)
         if link_Bps is not None:
             p.link_Bps[d] = int(link_Bps[d])
+        if link_lat_ns is not None:
+            p.link_lat_ns[d] = int(link_lat_ns[d])
     return p
 
 

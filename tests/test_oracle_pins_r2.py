@@ -284,3 +284,76 @@ def test_dp_perf_lanes_cpp_matches_hand():
     assert [c.finish_ns for c in mm.mm_plan_chunks(plan)] == DP_PERF_LANES_FIN
     mm.mm_plan_destroy(plan)
     mm.mm_app_destroy(app)
+
+
+# ---------------------------------------- DP-Perf transfer latency (R32) ----
+def _two_kernel_app():
+    """kernel 0 writes X (chunks of 32 items), kernel 1 reads X and writes Y."""
+    k0 = oc.Kernel("produce", 64, 32, 1, [oc.Access(0, oc.WRITE)])
+    k1 = oc.Kernel("consume", 64, 32, 1, [oc.Access(0, oc.READ), oc.Access(1, oc.WRITE)])
+    return oc.App(buffers=[(4, 64), (4, 64)], kernels=[k0, k1])
+
+
+# G = 2, one chunk per device per kernel (2 chunks of 32 items), estimates
+# kernel 0: 10 / 30 ns, kernel 1: 10 / 10 ns, link 1e15 B/s (128 B -> 1 ns).
+#   t0 produce c0: dev0 10 vs dev1 30                    -> dev0, 10
+#   t1 produce c1: dev0 20 vs dev1 30                    -> dev0, 20
+#   t2 consume c0 (X from t0 on dev0, fin 10):
+#      dev0 max(20, 10) + 10 = 30;  dev1 max(0, 10 + L + 1) + 10 = 21 + L
+#      L = 0  -> dev1, 21;   L = 20 -> dev0, 30 (the pull's fixed cost wins)
+#   t3 consume c1 (X from t1, fin 20):
+#      L = 0:  dev0 max(20, 20) + 10 = 30; dev1 max(21, 21) + 10 = 31 -> dev0, 30
+#      L = 20: dev0 max(30, 20) + 10 = 40; dev1 20 + 21 + 10 = 51    -> dev0, 40
+@pytest.mark.parametrize("L,dev,fin", [(0, [0, 0, 1, 0], [10, 20, 21, 30]),
+                                       (20, [0, 0, 0, 0], [10, 20, 30, 40])])
+def test_dp_perf_transfer_latency_by_hand(L, dev, fin):
+    prof = oc.Profile(G=2, fs_item=[[1, 1]] * 2, chunk_est_ns=[[10, 10], [30, 10]],
+                      link_Bps=[10 ** 15] * 2, link_lat_ns=[L, L])
+    _, d, f = oc.dp_perf(_two_kernel_app(), prof, 1)
+    assert d == dev and f == fin
+
+
+@pytest.mark.parametrize("L,dev,fin", [(0, [0, 0, 1, 0], [10, 20, 21, 30]),
+                                       (20, [0, 0, 0, 0], [10, 20, 30, 40])])
+def test_dp_perf_transfer_latency_cpp(L, dev, fin):
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    app = mm.mm_app_create()
+    mm.mm_app_add_buffer(app, 4, 64)
+    mm.mm_app_add_buffer(app, 4, 64)
+    cb = mm.mm_launch_fn(lambda user, d, r, ops, stream: 0)   # planning only: never launched
+    for name, acc in (("produce", [(0, mm.MM_WRITE, 1, 0)]),
+                      ("consume", [(0, mm.MM_READ, 1, 0), (1, mm.MM_WRITE, 1, 0)])):
+        desc = mm.kernel_desc(name, mm.MM_OP_CUSTOM, 64, acc)
+        desc.launch = cb
+        mm.mm_app_add_kernel(app, desc)
+    prof = mm.make_profile(2, [[1, 1]] * 2, [[10, 10], [30, 10]], [10 ** 15] * 2, link_lat_ns=[L, L])
+    plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_DP_PERF, chunks_per_dev=1))
+    ch = mm.mm_plan_chunks(plan)
+    assert [c.device for c in ch] == dev and [c.finish_ns for c in ch] == fin
+    mm.mm_plan_destroy(plan)
+    mm.mm_app_destroy(app)
+
+
+def test_dp_perf_random_latency_parity():
+    """C++ DP-Perf = oracle DP-Perf bit for bit with random per-device
+    transfer latencies (STREAM w sync, HotSpot halos, Cholesky DAG)."""
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    import random
+    rnd = random.Random(7)
+    cases = [(mm.mm_app_builtin(mm.MM_APP_STREAM, [777, 2, 1, 32, 1]), oa.stream(777, 2, 1, 32, 1), 4),
+             (mm.mm_app_builtin(mm.MM_APP_HOTSPOT, [90, 8, 5, 1, 1]), oa.hotspot(90, 8, 5, 1, 1), 1),
+             (mm.mm_app_builtin(mm.MM_APP_CHOLESKY, [5 * 32, 32]), oa.cholesky_tasks(5, 32), 4)]
+    for capp, oapp, K in cases:
+        for G in (2, 3):
+            ps = [[rnd.randint(100, 5000) for _ in range(K)] for _ in range(G)]
+            est = [[rnd.randint(1000, 10 ** 5) for _ in range(K)] for _ in range(G)]
+            link = [rnd.randint(10 ** 8, 10 ** 12) for _ in range(G)]
+            lat = [rnd.randint(0, 10 ** 5) for _ in range(G)]
+            po = oc.Profile(G=G, fs_item=ps, chunk_est_ns=est, link_Bps=link, link_lat_ns=lat)
+            pc = mm.make_profile(G, ps, est, link, link_lat_ns=lat)
+            _, dev, fin = oc.dp_perf(oapp, po, 2)
+            plan = mm.mm_plan_build(capp, pc, mm.plan_opts(mm.MM_DP_PERF, chunks_per_dev=2))
+            ch = mm.mm_plan_chunks(plan)
+            assert [c.device for c in ch] == dev and [c.finish_ns for c in ch] == fin
+            mm.mm_plan_destroy(plan)
+        mm.mm_app_destroy(capp)

@@ -167,6 +167,7 @@ def run_config(name, app_id, ip, budgets, staged, reps):
                 "dp_perf_adaptive_ms": None if adaptive_ms is None else round(adaptive_ms, 4),
                 "dp_perf_adaptive_task_share": ad_share,
                 "profile_link_Bps": [int(prof.link_Bps[d]) for d in range(G)],
+                "profile_link_lat_ns": [int(prof.link_lat_ns[d]) for d in range(G)],
                 "emulation_note": emulation_note(budgets, cls, app_id),
                 "profile_fs_item": [[int(prof.fs_item[d][k]) for k in range(s.K)] for d in range(G)],
                 "profile_chunk_est_ns": [[int(prof.chunk_est_ns[d][k]) for k in range(s.K)] for d in range(G)]}
