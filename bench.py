@@ -37,7 +37,7 @@ APPS = {
                "MK-Seq STREAM-Seq copy/scale/add/triad, 2^28 FP32 (BASELINE configs[1])"),
     "stream-loop": ("MM_APP_STREAM", [1 << 28, 10, 0], lambda p: 40 * p[0] * p[1],
                     "MK-Loop STREAM-Loop x10, 2^28 FP32"),
-    "hotspot": ("MM_APP_HOTSPOT", [8192, 8192, 1000], lambda p: 12 * p[0] * p[1] * p[2],
+    "hotspot": ("MM_APP_HOTSPOT", [8192, 8192, 1000], lambda p: p[0] * p[1] * p[2],
                 "SK-Loop HotSpot 8192^2 x 1000 iterations (BASELINE configs[2])"),
     "stencil": ("MM_APP_STENCIL_REDUCTION", [16384, 16384, 100, 1], lambda p: 20 * p[0] * p[1] * p[2],
                 "MK-Loop stencil + FP64 residual 16384^2 x 100 steps, w-sync (BASELINE configs[3])"),
@@ -53,6 +53,9 @@ APPS = {
               "SK-Loop Nbody 1,048,576 bodies, 1 step (P319; 20 flop/interaction)"),
 }
 FLOP_APPS = ("sgemm", "matmul1k", "cholesky", "nbody")
+# HotSpot with temporal blocking moves 12 B per cell per h iterations, so a
+# "bytes per iteration" rate is not a bandwidth: report cell updates per second
+CELL_APPS = ("hotspot",)
 # HotSpot temporal block: iterations per launch in the bench
 # step (1000 % HOTSPOT_TB == 0); the result is bit-identical for every value
 HOTSPOT_TB = 8
@@ -145,6 +148,14 @@ def dist_env():
     return world, rank, local
 
 
+def unit_of(app: str):
+    if app in FLOP_APPS:
+        return "TFLOP/s", 1e12
+    if app in CELL_APPS:
+        return "Gcell-updates/s", 1e9
+    return "GB/s", 1e9
+
+
 def cpu_baseline(app: str, seconds: float = 10.0):
     """The oracle, as it stands, single-threaded on a bounded sample."""
     import numpy as np
@@ -173,6 +184,9 @@ def cpu_baseline(app: str, seconds: float = 10.0):
             t, out = out, t
             it += 1
         dt = time.perf_counter() - t0
+        if app == "hotspot":
+            return {"value": rows * cols * it / dt / 1e9, "unit": "Gcell-updates/s", "cores": 1, "kind": "oracle",
+                    "sample": f"{it} HotSpot iterations over 1024 of the 8192 rows"}
         return {"value": 12 * rows * cols * it / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
                 "sample": f"{it} HotSpot iterations over 1024 of the 8192 rows"}
     if app == "blackscholes":
@@ -224,7 +238,7 @@ def run_reference(args):
     world, rank, local = dist_env()
     if rank != 0:
         return
-    unit = "TFLOP/s" if args.app in FLOP_APPS else "GB/s"
+    unit = unit_of(args.app)[0]
     # each step = a bounded sample of the workload on the oracle (host cores)
     vals = []
     for i in range(args.warmup + args.steps):
@@ -254,6 +268,8 @@ def main():
     ap.add_argument("--chol-n", type=int, default=None, help="Cholesky order n (default 32768)")
     ap.add_argument("--pipeline", type=int, default=32,
                     help="e2e staged pipeline sub-chunks per device (R24; 8: 171.5, 16: 174.1, 32: 176.4, 64: 175.4 GB/s STREAM)")
+    ap.add_argument("--no-graph", action="store_true",
+                    help="timed steps issue the op program eagerly instead of replaying a CUDA graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-strategies", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the staged (host-buffer) e2e pass")
@@ -357,9 +373,18 @@ def main():
         if pristine:
             torch.cuda.synchronize()
 
-    for _ in range(args.warmup):
+    # timed steps: the op program replayed as one CUDA graph, enqueued without
+    # a host round trip per step (mm_run no_wait; steps are ordered on the
+    # library's streams); the last ceil(K/5) steps run eagerly with CUDA events
+    # around every kernel for the roofline (--kernel-timing)
+    graph_ok = world == 1 or os.environ.get("MM_TRANSPORT") != "nccl"
+    fast = dict(use_graph=graph_ok and not args.no_graph, no_wait=True)
+    for w in range(args.warmup):
         restore()
-        step(plan, time_kernels=True)
+        if w == 0:
+            step(plan, time_kernels=True)
+        else:
+            step(plan, **fast)
     barrier()
     l0 = mm.mm_kernel_launch_count()
     stream = sess.stream(rank if world > 1 else 0)
@@ -375,7 +400,7 @@ def main():
                 ev0 = torch.cuda.Event(enable_timing=True)
                 ev0.record(stream)
             kt = args.kernel_timing == "all" or (args.kernel_timing == "last" and i >= args.steps - n_last)
-            st = step(plan, time_kernels=kt)
+            st = step(plan, time_kernels=True) if kt else step(plan, **fast)
             for d in range(G):
                 for k in range(K):
                     kms[d][k] += st.kernel_ms[d][k]
@@ -395,11 +420,8 @@ def main():
         dist.all_reduce(lt)
         gpu_launches = int(lt.item())
     ms_step = ms_total / args.steps
-    value = algo_bytes / (ms_step * 1e-3) / 1e9
-    unit = "GB/s"
-    if args.app in FLOP_APPS:
-        value = algo_bytes / (ms_step * 1e-3) / 1e12
-        unit = "TFLOP/s"
+    unit, scale = unit_of(args.app)
+    value = algo_bytes / (ms_step * 1e-3) / scale
 
     # --- roofline of the dominant kernel (event-timed inside the timed region)
     dom, bpi = DOMINANT[args.app]
@@ -533,7 +555,7 @@ def main():
             t = torch.tensor([ms_e2e], dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms_e2e = float(t.item())
-        ev = algo_bytes / (ms_e2e * 1e-3) / (1e12 if unit == "TFLOP/s" else 1e9)
+        ev = algo_bytes / (ms_e2e * 1e-3) / scale
         e2e = {"value": ev, "unit": unit, "h2d_bytes_per_step": int(hb), "d2h_bytes_per_step": int(db),
                "ms_per_step": ms_e2e, "mode": f"staged (pinned host inputs; H2D / kernels / D2H pipelined over {args.pipeline} sub-chunks per device)"}
         del host
@@ -592,6 +614,8 @@ def main():
                        "kernel_timing": {"all": "per-kernel CUDA events in every timed step",
                                          "last": f"per-kernel CUDA events in the last {n_last} of {args.steps} timed steps",
                                          "none": "no per-kernel events"}[args.kernel_timing],
+                       "issue": ("other timed steps: the op program replayed as a CUDA graph, enqueued back to back"
+                                 if fast["use_graph"] else "other timed steps: eager issue, enqueued back to back"),
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
                        **({"temporal_block": tb} if args.app == "hotspot" else {})},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,

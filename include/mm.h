@@ -412,6 +412,12 @@ typedef struct {
   int32_t max_inflight;      /* adaptive: chunks in flight per device before the scheduler
                                 waits for completions (default 4) */
   void* const* host;         /* staged / flush: host (pinned) pointer per slot, or NULL */
+  int32_t no_wait;           /* 1: return once the run is enqueued (not with time_kernels or
+                                adaptive): its streams are joined into the first owned device's
+                                stream (mm_ctx_stream), so later runs and a caller stream set by
+                                mm_ctx_set_stream are ordered after it; device_ms = -1; host
+                                buffers must not be touched before that stream completes */
+  int32_t _pad;
 } mm_run_opts;
 
 /* One adaptive DP-Perf decision: the snapshot it was taken on.  All times in
@@ -438,8 +444,8 @@ typedef struct {
   int64_t h2d_bytes, d2h_bytes;
 } mm_run_stats;
 
-/* Execute the plan's op program (blocking: returns when this process's
- * devices are done).  buffers as in mm_profile_run, or NULL for the buffers
+/* Execute the plan's op program (blocking unless opts->no_wait: returns when
+ * this process's devices are done).  buffers as in mm_profile_run, or NULL for the buffers
  * registered with mm_buffer_register; runs are ordered with the streams set
  * by mm_ctx_set_stream. */
 mm_status mm_run(mm_ctx* ctx, mm_plan* plan, void* const* buffers, const mm_run_opts* opts,

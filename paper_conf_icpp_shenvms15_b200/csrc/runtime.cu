@@ -1655,6 +1655,18 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_stop, rs));
   }
+  if (o && o->no_wait && !timing) {
+    // enqueue only: every library stream of this run is joined into the root
+    // stream, so the next run (or a caller stream set with mm_ctx_set_stream,
+    // or a synchronisation of mm_ctx_stream(root)) is ordered after it
+    if ((r = join_external(ctx, false))) return r;
+    S->wall_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    S->device_ms = -1.0;
+    for (size_t i = 0; i < plan.ops.size(); ++i)
+      if (plan.ops[i].kind == MM_OPK_KERNEL && ctx->dev[plan.ops[i].device].mine)
+        S->kernel_launches[plan.ops[i].device][plan.ops[i].kernel]++;
+    return MM_OK;
+  }
   CU_OK(cudaEventSynchronize(rt->t_stop));
   auto t1 = std::chrono::steady_clock::now();
   if ((r = join_external(ctx, false))) return r;
