@@ -1121,17 +1121,16 @@ mm_status run_adaptive(mm_ctx* ctx, Plan& plan, PlanRt* rt, void* const* buffers
     const int64_t items = app.is_dag ? 1 : std::max<int64_t>(1, task.e - task.b);
     int32_t best = -1;
     for (int32_t d = 0; d < G; ++d) {
-      uint64_t ready = 0;
+      uint64_t ready = 0, xfer = 0;   // R21/R32 as in the frozen schedule; the pulls go into cost_ns
       for (auto& p : preds) {
-        uint64_t rr = fin[p.first];
+        ready = std::max(ready, fin[p.first]);
         if (ap.task_dev[p.first] != d) {
           const uint64_t link = std::max<uint64_t>(1, ap.prof.link_Bps[d]);
-          rr += ap.prof.link_lat_ns[d] + (uint64_t)(((unsigned __int128)p.second * 1000000000ull + link - 1) / link);
+          xfer += ap.prof.link_lat_ns[d] + (uint64_t)(((unsigned __int128)p.second * 1000000000ull + link - 1) / link);
         }
-        ready = std::max(ready, rr);
       }
       const uint64_t busy = std::max(dec.now_ns, pred_fin[d]);
-      const uint64_t cost = (uint64_t)(est[d][task.kernel] * (double)items / (double)nominal[task.kernel]);
+      const uint64_t cost = xfer + (uint64_t)(est[d][task.kernel] * (double)items / (double)nominal[task.kernel]);
       dec.busy_ns[d] = busy;
       dec.ready_ns[d] = ready;
       dec.cost_ns[d] = cost;

@@ -295,26 +295,31 @@ def _two_kernel_app():
 
 
 # G = 2, one chunk per device per kernel (2 chunks of 32 items), estimates
-# kernel 0: 10 / 30 ns, kernel 1: 10 / 10 ns, link 1e15 B/s (128 B -> 1 ns).
-#   t0 produce c0: dev0 10 vs dev1 30                    -> dev0, 10
-#   t1 produce c1: dev0 20 vs dev1 30                    -> dev0, 20
-#   t2 consume c0 (X from t0 on dev0, fin 10):
-#      dev0 max(20, 10) + 10 = 30;  dev1 max(0, 10 + L + 1) + 10 = 21 + L
-#      L = 0  -> dev1, 21;   L = 20 -> dev0, 30 (the pull's fixed cost wins)
-#   t3 consume c1 (X from t1, fin 20):
-#      L = 0:  dev0 max(20, 20) + 10 = 30; dev1 max(21, 21) + 10 = 31 -> dev0, 30
-#      L = 20: dev0 max(30, 20) + 10 = 40; dev1 20 + 21 + 10 = 51    -> dev0, 40
-@pytest.mark.parametrize("L,dev,fin", [(0, [0, 0, 1, 0], [10, 20, 21, 30]),
-                                       (20, [0, 0, 0, 0], [10, 20, 30, 40])])
+# kernel 0: 5 / 30 ns, kernel 1: 10 / 5 ns, link 1e15 B/s (128 B -> 1 ns).  A
+# task's inputs held by another device are pulled by the consuming device
+# before the task: eft = max(busy, ready) + pulls + cost (R21/R32).
+#   t0 produce c0: dev0 5 vs dev1 30                     -> dev0, 5
+#   t1 produce c1: dev0 10 vs dev1 30                    -> dev0, 10
+#   t2 consume c0 (X from t0 on dev0, fin 5):
+#      dev0 max(10, 5) + 10 = 20;  dev1 max(0, 5) + (L + 1) + 5 = 11 + L
+#      L = 0 -> dev1, 11;  L = 20 -> dev0, 20
+#   t3 consume c1 (X from t1, fin 10):
+#      L = 0:  dev0 max(20, 10) + 10 = 30; dev1 max(11, 10) + 1 + 5 = 17 -> dev1, 17
+#              (pricing the pull in the ready time instead would give 16)
+#      L = 20: dev0 max(20, 10) + 10 = 30; dev1 max(0, 10) + 21 + 5 = 36 -> dev0, 30
+LAT_CASES = [(0, [0, 0, 1, 1], [5, 10, 11, 17]), (20, [0, 0, 0, 0], [5, 10, 20, 30])]
+LAT_EST = [[5, 10], [30, 5]]
+
+
+@pytest.mark.parametrize("L,dev,fin", LAT_CASES)
 def test_dp_perf_transfer_latency_by_hand(L, dev, fin):
-    prof = oc.Profile(G=2, fs_item=[[1, 1]] * 2, chunk_est_ns=[[10, 10], [30, 10]],
+    prof = oc.Profile(G=2, fs_item=[[1, 1]] * 2, chunk_est_ns=LAT_EST,
                       link_Bps=[10 ** 15] * 2, link_lat_ns=[L, L])
     _, d, f = oc.dp_perf(_two_kernel_app(), prof, 1)
     assert d == dev and f == fin
 
 
-@pytest.mark.parametrize("L,dev,fin", [(0, [0, 0, 1, 0], [10, 20, 21, 30]),
-                                       (20, [0, 0, 0, 0], [10, 20, 30, 40])])
+@pytest.mark.parametrize("L,dev,fin", LAT_CASES)
 def test_dp_perf_transfer_latency_cpp(L, dev, fin):
     mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
     app = mm.mm_app_create()
@@ -326,7 +331,7 @@ def test_dp_perf_transfer_latency_cpp(L, dev, fin):
         desc = mm.kernel_desc(name, mm.MM_OP_CUSTOM, 64, acc)
         desc.launch = cb
         mm.mm_app_add_kernel(app, desc)
-    prof = mm.make_profile(2, [[1, 1]] * 2, [[10, 10], [30, 10]], [10 ** 15] * 2, link_lat_ns=[L, L])
+    prof = mm.make_profile(2, [[1, 1]] * 2, LAT_EST, [10 ** 15] * 2, link_lat_ns=[L, L])
     plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_DP_PERF, chunks_per_dev=1))
     ch = mm.mm_plan_chunks(plan)
     assert [c.device for c in ch] == dev and [c.finish_ns for c in ch] == fin

@@ -180,6 +180,7 @@ def main():
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "r2_ranking.json"))
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--only", default="", help="run only the apps whose name contains this string")
     ap.add_argument("--platforms", default="HET-2,HOMO-2",
                     help="comma list of " + ",".join(PLATFORMS))
     args = ap.parse_args()
@@ -189,6 +190,8 @@ def main():
     t0 = time.time()
     for pname, budgets in plats:
         for name, app_id, ip in APPS:
+            if args.only and args.only not in name:
+                continue
             modes = [False]
             if app_id == mm.MM_APP_STREAM and not args.quick:
                 modes.append(True)
