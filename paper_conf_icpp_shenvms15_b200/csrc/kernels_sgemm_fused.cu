@@ -1,35 +1,37 @@
 // Small-SGEMM path of MatrixMul (BASELINE configs[0], 1024^2; P311 C = A x B,
 // row-wise split) in ONE launch: no operand-split pass, no reduction pass.
 //
-// A cluster of 2 S CTAs computes one 256 x 256 output tile pair over S K
-// splits (S in 2..4, chosen so that every cluster is resident at once): CTA
-// rank r = 2 z + h is half h (128 rows) of the 2-SM pair (tcgen05
+// A cluster of 2 S CTAs computes one 256 x 128 output tile pair over S K
+// splits (S in 2..4, the largest whose clusters are all resident at once):
+// CTA rank r = 2 z + h is half h (128 rows) of the 2-SM pair (tcgen05
 // cta_group::2) of K split z (k-blocks [z nkb / S, (z+1) nkb / S)).
 //  warp 0      TMA producer: RAW fp32 tiles straight from A (row-major,
-//              K-major: box 16 x 128 rows, SWIZZLE_64B) and B (row-major:
-//              four boxes of 32 columns x 16 k-rows, SWIZZLE_128B) into a
-//              4-stage raw ring.
-//  warps 2-5   converters: x -> hi = tf32_rn(x), lo = tf32_rn(x - hi) (the
-//              split of the two-pass path) into a 4-stage split ring — A in
-//              place of its swizzled layout, B transposed on the way into
-//              the K-major SWIZZLE_64B layout of the two-pass path's B^T (an
-//              MN-major B descriptor read zeros on this B200); proxy fence;
-//              one arrival per warp on the leader CTA's stage barrier.
-//  warp 1      (leader CTA) tcgen05.mma.cta_group::2.kind::tf32, 3 MMAs per
-//              k-step (lo.hi + hi.lo + hi.hi) into a 256-column TMEM
-//              accumulator; commits free the split stages of both CTAs.
-//  epilogue    warps 2-5: TMEM -> registers -> this CTA's smem (padded
-//              rows); cluster barrier; CTA z sums float4 columns
-//              [z 64 / S, (z+1) 64 / S) of its 128 rows over the S partials in
-//              split order ((p0 + p1) + p2) + p3 by distributed-shared-memory
-//              loads from its cluster peers and stores C; cluster barrier
-//              before exit.
-// Measured (1024^2, S = 3: 16 clusters of 6 CTAs; 8-CTA clusters fit only 15
-// at a time): ~0.7 us set-up, ~14 us main loop (shared-memory traffic of the
-// in-place split + transposition on top of the MMA operand reads), ~1 us
-// TMEM -> smem, ~4.5 us reduction (DSMEM moves ~20 B/clk per SM; a push of
-// the partial slices by cp.async.bulk and a reduction through L2 were both
-// slower).
+//              K-major: box 16 x 128 rows, SWIZZLE_64B) and B (row-major: two
+//              boxes of 32 columns x 16 k-rows, SWIZZLE_128B) into a 12-stage
+//              raw ring (L2/HBM latency).
+//  warps 2-9   two groups of four converter warps, alternating k-steps:
+//              x -> hi = tf32_rn(x), lo = tf32_rn(x - hi) (the split of the
+//              two-pass path); A rows (thread = TMEM lane) straight into 32
+//              TMEM columns per stage (tcgen05.st), B transposed into the
+//              K-major SWIZZLE_64B layout of the two-pass path's B^T in a
+//              4-stage smem ring (an MN-major B descriptor read zeros on this
+//              B200); one arrival per warp on the leader CTA's barrier.
+//  warp 1      (leader CTA) tcgen05.mma.cta_group::2.kind::tf32 with A from
+//              TMEM, B from smem: 3 MMAs per k-step (lo.hi + hi.lo + hi.hi)
+//              into a 128-column TMEM accumulator; commits free the stages.
+//  epilogue    the converter warps: TMEM -> registers -> this CTA's smem
+//              (padded rows); cluster barrier; CTA z sums float4 columns
+//              [z 32 / S, (z+1) 32 / S) of its 128 rows over the S partials
+//              in split order ((p0 + p1) + p2) + p3 by distributed-shared-
+//              memory loads from its cluster peers and stores C; cluster
+//              barrier before exit.
+// 1024^2 (S = 2, 128 CTAs in clusters of 4): 23.5 us (ncu, cold) against 33 us
+// for the split -> GEMM -> reduce chain.  globaltimer stamps: set-up 0.8 us,
+// first MMA at 1.9 us, ~490 ns per k-step (MMA-issue-bound: the converters
+// run up to 3 steps ahead), reduction ~4 us (DSMEM moves ~20 B/clk per SM).
+// Tried and dropped: 256-wide pairs with S = 3 (24.9 us, both operands in
+// smem: 26 us), a cp.async.bulk push of the partial slices and a reduction
+// through L2 (both slower than the DSMEM pull).
 #include <cuda.h>
 
 #include <algorithm>
@@ -48,13 +50,23 @@ namespace {
 
 using namespace tcx;
 
-constexpr int FBM = 128, FBK = 16, FHALF = 128;                // rows per CTA, k per stage, B columns per CTA
-constexpr int kRawStages = 4, kSplitStages = 4, kFThreads = 192;
-constexpr int RAW_A = FBM * FBK * 4, RAW_B = FHALF * FBK * 4;  // 8 KB + 8 KB
+constexpr int FBM = 128, FBK = 16, FHALF = 64;                 // rows per CTA, k per stage, B columns per CTA
+constexpr int FBN = 2 * FHALF;                                 // output columns of a tile pair (MMA N)
+// warps: 0 producer, 1 MMA issuer, 2.. kConvGroups groups of 4 converter warps
+// (group g converts the stages i with i % kConvGroups == g: a converter's
+// per-stage chain — smem loads, split, TMEM stores + wait, arrive — is
+// latency-bound, so two groups alternate)
+constexpr int kConvGroups = 2;
+// The raw ring is deep: its TMA loads come from L2/HBM (~1 us), and a 4-stage
+// ring bounded a k-step to latency / 4 (measured 470 ns per k-step).
+constexpr int kRawStages = 12, kSplitStages = 4, kFThreads = 64 + 128 * kConvGroups;
+constexpr int RAW_A = FBM * FBK * 4, RAW_B = FHALF * FBK * 4;  // 8 KB + 4 KB
 constexpr int RAW_BYTES = RAW_A + RAW_B;
-constexpr int SPLIT_BYTES = 2 * RAW_BYTES;                     // A_hi, A_lo, B_hi, B_lo
+constexpr int SPLIT_BYTES = 2 * RAW_B;                         // B_hi, B_lo (A_hi, A_lo go to TMEM)
 constexpr int kRingBytes = kRawStages * RAW_BYTES + kSplitStages * SPLIT_BYTES;   // 192 KB
-constexpr int RED_LD = 256 + 4;        // padded fp32 row of the partial (reuses the drained rings)
+constexpr int RED_LD = FBN + 4;        // padded fp32 row of the partial (reuses the drained rings)
+constexpr int kTmemCols = 256;         // FBN accumulator columns + kSplitStages x 32 A columns
+static_assert(FBN + kSplitStages * 32 <= kTmemCols, "TMEM columns");
 constexpr int kFusedSmem = kRingBytes + 1024 + 256;
 static_assert(FBM * RED_LD * 4 <= kRingBytes, "partial buffer");
 
@@ -113,6 +125,25 @@ __device__ __forceinline__ void fwait(uint64_t* b, uint32_t parity) {
   }
 }
 
+// 3xTF32 pair MMA with A read from tensor memory (TS form), B from smem
+__device__ __forceinline__ void mma_tf32_pair_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t b, uint32_t idesc,
+                                                 uint32_t acc) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(b), "r"(idesc), "r"(acc));
+}
+
+// 16 consecutive 32-bit TMEM columns of this thread's lane
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const float (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]), "f"(v[8]), "f"(v[9]),
+      "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15])
+      : "memory");
+}
+
 __device__ __forceinline__ float4 ld_dsmem_f4(uint32_t addr) {
   float4 v;
   asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
@@ -162,7 +193,8 @@ __global__ void __launch_bounds__(kFThreads, 1)
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tB) : "memory");
   }
   if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(saddr(tslot)));
+    // FBN accumulator columns + per split stage 32 columns of A (hi 16, lo 16)
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)), "n"(kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -175,7 +207,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
   if (warp == 0) {
     if (lane == 0) {   // ===== producer: raw tiles of this CTA (own barrier)
       const int32_t ya = m_blk * FBM;
-      const int32_t xb = nb * 256 + (int32_t)h * FHALF;
+      const int32_t xb = nb * FBN + (int32_t)h * FHALF;
       for (int i = 0; i < nkb; ++i) {
         const int s = i % kRawStages;
         if (i >= kRawStages) fwait(&raw_empty[s], (uint32_t)(((i / kRawStages) - 1) & 1));
@@ -184,7 +216,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
         mbar_expect_tx(&raw_full[s], RAW_BYTES);
         tma_load_2d(st, &tA, kx, ya, &raw_full[s]);
 #pragma unroll
-        for (int j = 0; j < 4; ++j) tma_load_2d(st + RAW_A + j * 2048, &tB, xb + 32 * j, kx, &raw_full[s]);
+        for (int j = 0; j < FHALF / 32; ++j) tma_load_2d(st + RAW_A + j * 2048, &tB, xb + 32 * j, kx, &raw_full[s]);
       }
     }
     __syncwarp();
@@ -192,20 +224,20 @@ __global__ void __launch_bounds__(kFThreads, 1)
     if (lane == 0 && leader) {   // ===== MMA issuer
       const uint32_t idesc = (1u << 4)                 // D: fp32
                              | (2u << 7) | (2u << 10)  // A, B: tf32
-                             | ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+                             | ((uint32_t)(FBN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
       for (int i = 0; i < nkb; ++i) {
         const int s = i % kSplitStages;
         fwait(&split_full[s], (uint32_t)((i / kSplitStages) & 1));
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         uint8_t* st = spl + s * SPLIT_BYTES;
-        const uint64_t ahi = sdesc(st), alo = sdesc(st + RAW_A);
-        const uint64_t bhi = sdesc(st + 2 * RAW_A), blo = sdesc(st + 2 * RAW_A + RAW_B);
+        const uint64_t bhi = sdesc(st), blo = sdesc(st + RAW_B);
+        const uint32_t ahi = tmem + (uint32_t)FBN + (uint32_t)(s * 32), alo = ahi + 16u;   // A in TMEM columns
 #pragma unroll
         for (int kk = 0; kk < FBK / 8; ++kk) {
-          const uint64_t adv = (uint64_t)(kk * 32) >> 4;     // 8 fp32 along K inside the 64-B row
-          mma_tf32_pair(tmem, alo + adv, bhi + adv, idesc, (i | kk) != 0);
-          mma_tf32_pair(tmem, ahi + adv, blo + adv, idesc, 1u);
-          mma_tf32_pair(tmem, ahi + adv, bhi + adv, idesc, 1u);
+          const uint64_t adv = (uint64_t)(kk * 32) >> 4;     // 8 fp32 along K inside B's 64-B row
+          mma_tf32_pair_ts(tmem, alo + 8u * kk, bhi + adv, idesc, (i | kk) != 0);
+          mma_tf32_pair_ts(tmem, ahi + 8u * kk, blo + adv, idesc, 1u);
+          mma_tf32_pair_ts(tmem, ahi + 8u * kk, bhi + adv, idesc, 1u);
         }
         commit_pair_at(&split_empty[s], rank);
       }
@@ -213,27 +245,33 @@ __global__ void __launch_bounds__(kFThreads, 1)
     }
     __syncwarp();
   } else {   // ===== converters, then the epilogue (warps 2..5)
-    const int ct = threadIdx.x - 64;   // 0..127
-    for (int i = 0; i < nkb; ++i) {
+    const int cg = (warp - 2) / 4;                // converter group
+    const int ct = (threadIdx.x - 64) & 127;      // 0..127 within the group
+    for (int i = cg; i < nkb; i += kConvGroups) {
       const int s = i % kRawStages, q = i % kSplitStages;
       fwait(&raw_full[s], (uint32_t)((i / kRawStages) & 1));
       if (i >= kSplitStages) fwait(&split_empty[q], (uint32_t)(((i / kSplitStages) - 1) & 1));
       const uint8_t* rs = raw + s * RAW_BYTES;
       uint8_t* dst = spl + q * SPLIT_BYTES;
-      // A: 512 float4 of the K-major SWIZZLE_64B tile, split in place
+      // A: row r = this thread's TMEM lane (warp w owns lanes 32 (w % 4) ..):
+      // its 16 k of the raw K-major SWIZZLE_64B tile (chunk c of row r at
+      // chunk c ^ ((r >> 1) & 3)), split, written to TMEM columns of slot q
+      const int ar = (warp & 3) * 32 + lane;
       float4 v[4];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) v[j] = reinterpret_cast<const float4*>(rs)[ct + 128 * j];
+      for (int c = 0; c < 4; ++c)
+        v[c] = *reinterpret_cast<const float4*>(rs + ar * 64 + ((c ^ ((ar >> 1) & 3)) << 4));
       // B: the raw tile is MN-major (4 boxes of 16 k-rows x 32 columns,
       // SWIZZLE_128B: 16-B chunk c of row k stored at chunk c ^ (k & 7)); it is
       // transposed into the K-major SWIZZLE_64B layout the MMA reads (row n =
       // 64 B of 16 k, chunk c stored at c ^ ((n >> 1) & 3)).  Output float4 o:
       // n = o & 127, k = 4 (o >> 7) .. +3; a warp reads 32 consecutive columns
       // of one raw row per load (conflict-free).
-      float4 w[4];
+      constexpr int NB4 = FHALF * 4 / 128;   // B output float4 per converter thread
+      float4 w[NB4];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int o = ct + 128 * j, n = o & 127, k0 = 4 * (o >> 7);
+      for (int j = 0; j < NB4; ++j) {
+        const int o = ct + 128 * j, n = o % FHALF, k0 = 4 * (o / FHALF);
         const uint8_t* box = rs + RAW_A + (n >> 5) * 2048 + (n & 3) * 4;
         const int c16 = (n & 31) >> 2;
         float t[4];
@@ -244,25 +282,34 @@ __global__ void __launch_bounds__(kFThreads, 1)
         }
         w[j] = make_float4(t[0], t[1], t[2], t[3]);
       }
+      {
+        float ah[16], al[16];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+        for (int c = 0; c < 4; ++c) {
+          split2(v[c].x, ah[4 * c], al[4 * c]);
+          split2(v[c].y, ah[4 * c + 1], al[4 * c + 1]);
+          split2(v[c].z, ah[4 * c + 2], al[4 * c + 2]);
+          split2(v[c].w, ah[4 * c + 3], al[4 * c + 3]);
+        }
+        const uint32_t ta = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)FBN + (uint32_t)(q * 32);
+        tmem_st16(ta, ah);
+        tmem_st16(ta + 16u, al);
+      }
+#pragma unroll
+      for (int j = 0; j < NB4; ++j) {
         float4 hi, lo;
-        split2(v[j].x, hi.x, lo.x);
-        split2(v[j].y, hi.y, lo.y);
-        split2(v[j].z, hi.z, lo.z);
-        split2(v[j].w, hi.w, lo.w);
-        reinterpret_cast<float4*>(dst)[ct + 128 * j] = hi;
-        reinterpret_cast<float4*>(dst + RAW_A)[ct + 128 * j] = lo;
-        const int o = ct + 128 * j, n = o & 127, kc4 = o >> 7;
+        const int o = ct + 128 * j, n = o % FHALF, kc4 = o / FHALF;
         const int boff = n * 64 + ((kc4 ^ ((n >> 1) & 3)) << 4);
         split2(w[j].x, hi.x, lo.x);
         split2(w[j].y, hi.y, lo.y);
         split2(w[j].z, hi.z, lo.z);
         split2(w[j].w, hi.w, lo.w);
-        *reinterpret_cast<float4*>(dst + 2 * RAW_A + boff) = hi;
-        *reinterpret_cast<float4*>(dst + 2 * RAW_A + RAW_B + boff) = lo;
+        *reinterpret_cast<float4*>(dst + boff) = hi;
+        *reinterpret_cast<float4*>(dst + RAW_B + boff) = lo;
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> tensor-core reads
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");   // A in TMEM
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B: generic writes -> tensor-core reads
       __syncwarp();
       if (lane == 0) {
         mbar_arrive(&raw_empty[s]);
@@ -277,7 +324,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
     const int r = grp * 32 + lane;                       // row within the CTA's 128
     const int64_t grow = (int64_t)m_blk * FBM + r;       // row within [row0, row0 + mrows)
     float* red = reinterpret_cast<float*>(base);         // all rings drained: reuse for the partial
-    for (int c = 0; c < 256; c += 16) {
+    for (int c = cg * (FBN / kConvGroups); c < (cg + 1) * (FBN / kConvGroups); c += 16) {
       uint32_t v[16];
       const uint32_t ta = tmem + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
       asm volatile(
@@ -293,7 +340,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
               make_float4(__uint_as_float(v[4 * q]), __uint_as_float(v[4 * q + 1]), __uint_as_float(v[4 * q + 2]),
                           __uint_as_float(v[4 * q + 3]));
       } else if (grow < mrows) {
-        const int64_t n0 = (int64_t)nb * 256 + c;
+        const int64_t n0 = (int64_t)nb * FBN + c;
         float* crow = C + (row0 + grow) * N;
 #pragma unroll
         for (int q = 0; q < 4; ++q)
@@ -309,10 +356,10 @@ __global__ void __launch_bounds__(kFThreads, 1)
   __syncthreads();
   if (S > 1) {
     cluster_sync_all();   // every partial of the cluster is in shared memory
-    // CTA z reduces float4 columns [z 64 / S, (z+1) 64 / S) of its 128 rows:
+    // CTA z reduces float4 columns [z FBN/4 / S, (z+1) FBN/4 / S) of its 128 rows:
     // the S partial loads of an element issued before the adds, summed in
     // split order ((p0 + p1) + p2) + p3; all 192 threads take part
-    const int c4a = (int)z * 64 / S, c4n = ((int)z + 1) * 64 / S - c4a;
+    const int c4a = (int)z * (FBN / 4) / S, c4n = ((int)z + 1) * (FBN / 4) / S - c4a;
     const float* red = reinterpret_cast<const float*>(base);
     uint32_t peer[4];
 #pragma unroll
@@ -330,7 +377,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
         if (zz < S) {
           a.x += p[zz].x; a.y += p[zz].y; a.z += p[zz].z; a.w += p[zz].w;
         }
-      const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * 256 + cc;
+      const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * FBN + cc;
       if (grow < mrows && n0 < N) *reinterpret_cast<float4*>(C + (row0 + grow) * N + n0) = a;
     }
     cluster_arrive_relaxed_wait();   // every bulk copy out of this CTA's smem has landed
@@ -339,7 +386,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
   }
   if (warp == 1) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 256;" ::"r"(tmem));
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmemCols));
   }
 }
 
@@ -356,7 +403,7 @@ int sgemm_fused_splits(const float* A, const float* B, float* C, int64_t mrows, 
   if (!env || (K & 3) || (N & 3)) return 0;
   if ((reinterpret_cast<uintptr_t>(A + r0 * K) | reinterpret_cast<uintptr_t>(B) | reinterpret_cast<uintptr_t>(C)) & 15)
     return 0;
-  const int64_t pairs = ((mrows + FBM - 1) / FBM + 1) / 2 * ((N + 255) / 256);
+  const int64_t pairs = ((mrows + FBM - 1) / FBM + 1) / 2 * ((N + FBN - 1) / FBN);
   const int64_t nkb = (K + FBK - 1) / FBK;
   if (pairs * 2 > 148 / 2) return 0;   // at least half the GPU in tile pairs already: no K split
   for (int S = 4; S >= 2; --S)
@@ -403,7 +450,7 @@ cudaError_t sgemm_fused_rows(const float* A, const float* B, float* C, int64_t N
   if (e != cudaSuccess) return e;
   const int mblk = (int)((mrows + FBM - 1) / FBM);
   const int mpairs = (mblk + 1) / 2;
-  const int nblk = (int)((N + 255) / 256);
+  const int nblk = (int)((N + FBN - 1) / FBN);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(mpairs * nblk * 2 * S));
   cfg.blockDim = dim3(kFThreads);
