@@ -380,7 +380,7 @@ __global__ void __launch_bounds__(kFThreads, 1)
       const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * FBN + cc;
       if (grow < mrows && n0 < N) *reinterpret_cast<float4*>(C + (row0 + grow) * N + n0) = a;
     }
-    cluster_arrive_relaxed_wait();   // every bulk copy out of this CTA's smem has landed
+    cluster_arrive_relaxed_wait();   // no CTA exits while a peer still reads its shared memory
   } else {
     cluster_sync_all();
   }
