@@ -320,6 +320,11 @@ __global__ void __launch_bounds__(kFThreads, 1)
     // ---- epilogue: accumulator (TMEM lanes 32 grp .. +32 = this warp's rows)
     const int grp = warp & 3;
     fwait(tfull, 0);
+    // the partial reuses the rings: every converter's raw-ring reads happened
+    // before its stage arrival and so before the last MMA's commit (tfull);
+    // the named barrier states it in a form compute-sanitizer's racecheck
+    // follows (it does not model the tcgen05.commit arrival)
+    asm volatile("bar.sync 1, %0;" ::"n"(128 * kConvGroups) : "memory");
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const int r = grp * 32 + lane;                       // row within the CTA's 128
     const int64_t grow = (int64_t)m_blk * FBM + r;       // row within [row0, row0 + mrows)
