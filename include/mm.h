@@ -253,6 +253,12 @@ typedef struct {
                                 the host as soon as it is final, so H2D, kernels and D2H of
                                 different sub-chunks overlap on separate streams (0/1 = off) */
   const mm_range* split;     /* optional SP split override [K*G] */
+  int32_t halo_split;        /* SP plans, kernels with halo reads, G > 1 (R33, not in the paper):
+                                each device range is run as its interior rows first, then the
+                                rows within the halo depth of a neighbouring device's range, so
+                                the interior kernel needs no pulled halo and overlaps the pulls
+                                (device-to-device pulls run on the copy-in stream) */
+  int32_t _pad2;
 } mm_plan_opts;
 
 /* One scheduled task. */

@@ -87,7 +87,7 @@ class mm_profile(C.Structure):
 class mm_plan_opts(C.Structure):
     _fields_ = [("strategy", C.c_int32), ("chunks_per_dev", C.c_int32), ("staged", C.c_int32),
                 ("grid_rows", C.c_int32), ("one_shot", C.c_int32), ("pipeline", C.c_int32),
-                ("split", C.POINTER(mm_range))]
+                ("split", C.POINTER(mm_range)), ("halo_split", C.c_int32), ("_pad2", C.c_int32)]
 
 
 class mm_chunk(C.Structure):
@@ -388,9 +388,10 @@ def mm_split(app: int, prof: mm_profile, strategy: int) -> Tuple[List[List[Tuple
 
 
 def plan_opts(strategy: int, chunks_per_dev: int = 8, staged: bool = False, grid_rows: int = 0,
-              split=None, one_shot: bool = False, pipeline: int = 0) -> mm_plan_opts:
+              split=None, one_shot: bool = False, pipeline: int = 0, halo_split: bool = False) -> mm_plan_opts:
     o = mm_plan_opts()
     o.pipeline = pipeline
+    o.halo_split = int(halo_split)
     o.strategy = strategy
     o.chunks_per_dev = chunks_per_dev
     o.staged = int(staged)

@@ -26,6 +26,7 @@ CASES = {
     "hotspot": (mm.MM_APP_HOTSPOT, [257, 256, 7, 1, 1], mm.MM_SP_SINGLE, (1,), 2),
     "hotspot_tb4": (mm.MM_APP_HOTSPOT, [300, 64, 24, 1, 1, 4], mm.MM_SP_SINGLE, (0,), 2),
     "hotspot_dp_dep": (mm.MM_APP_HOTSPOT, [200, 128, 6, 1, 1], mm.MM_DP_DEP, (0,), 2),
+    "hotspot_split": (mm.MM_APP_HOTSPOT, [300, 64, 24, 1, 1, 4], mm.MM_SP_SINGLE, (0,), 2),
     "stencil": (mm.MM_APP_STENCIL_REDUCTION, [200, 96, 5, 1, 1, 1], mm.MM_SP_VARIED, (1, 3), 2),
     "chol": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_DP_DEP, (0,), 1),
     "chol_cyclic": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_SP_CYCLIC, (0,), 1),
@@ -54,7 +55,7 @@ def main():
             s.load(0, A.reshape(T, b, T, b).transpose(0, 2, 1, 3).copy())
         else:
             s.fill()
-        plan = s.plan(strategy, prof, chunks_per_dev=kpd)
+        plan = s.plan(strategy, prof, chunks_per_dev=kpd, halo_split=case.endswith("_split"))
         for _ in range(runs):
             if app_id == mm.MM_APP_CHOLESKY and runs > 1:
                 s.load(0, A.reshape(T, b, T, b).transpose(0, 2, 1, 3).copy())

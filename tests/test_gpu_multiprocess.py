@@ -71,12 +71,13 @@ def test_stream_multiprocess(tmp_path, case, world, graph):
         assert sum(int(r["xfer"][0]) for r in res) > 0   # the re-sync pulled across processes
 
 
-@pytest.mark.parametrize("case,world", [("hotspot", 2), ("hotspot", 3), ("hotspot_tb4", 2), ("hotspot_dp_dep", 2)])
+@pytest.mark.parametrize("case,world", [("hotspot", 2), ("hotspot", 3), ("hotspot_tb4", 2), ("hotspot_dp_dep", 2),
+                                        ("hotspot_split", 3)])
 @pytest.mark.parametrize("graph", [False, True])
 def test_hotspot_multiprocess(tmp_path, case, world, graph):
     rows, cols, iters, tb = {"hotspot": (257, 256, 7, 1), "hotspot_tb4": (300, 64, 24, 4),
-                             "hotspot_dp_dep": (200, 128, 6, 1)}[case]
-    slot = {"hotspot": 1, "hotspot_tb4": 0, "hotspot_dp_dep": 0}[case]
+                             "hotspot_dp_dep": (200, 128, 6, 1), "hotspot_split": (300, 64, 24, 4)}[case]
+    slot = {"hotspot": 1, "hotspot_tb4": 0, "hotspot_dp_dep": 0, "hotspot_split": 0}[case]
     t0, p = synthgen.hotspot(rows, cols)
     res = run_ranks(case, world, tmp_path, graph=graph, runs=1)
     got = assemble(res, slot, rows * cols, np.float32).reshape(rows, cols)

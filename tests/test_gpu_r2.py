@@ -284,3 +284,40 @@ def test_collect_rejects_bad_destination(R):
         s.run(plan)
         with pytest.raises(mm.MMError):
             mm.mm_collect(s.ctx, plan, s.ptrs(), 0, s.bufs[(0, 0)].data_ptr(), 2)
+
+
+# ------------------------------------------------ halo overlap split (R33) --
+@pytest.mark.parametrize("tb,G", [(1, 3), (8, 3), (4, 2)])
+def test_hotspot_halo_split_bit_exact(R, tb, G):
+    """SP-Single HotSpot with each device range run interior-first (R33):
+    bit-identical to the oracle (same cells, same per-cell arithmetic)."""
+    mm, runner = R
+    rows, cols, iters = 300, 256, 32   # an even number of launches per run: the result is in slot 0
+    t0, p = synthgen.hotspot(rows, cols)
+    ref = on.hotspot_run(t0, p, iters)
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1, tb], G=G) as s:
+        s.fill()
+        plan = s.plan(mm.MM_SP_SINGLE, _prof(mm, G, 1), halo_split=True)
+        n_split = len(mm.mm_plan_chunks(plan))
+        assert n_split > (iters // tb) * G   # the ranges were cut
+        s.run(plan)
+        s.run(plan, use_graph=True)           # steady-state program, second pass from the first's output
+        got = s.collect(plan, 0).reshape(rows, cols)
+    ref2 = on.hotspot_run(ref, p, iters)
+    assert np.array_equal(got, ref2)
+
+
+def test_stencil_reduction_halo_split(R):
+    mm, runner = R
+    rows, cols, steps = 200, 96, 5
+    t0, p = synthgen.hotspot(rows, cols)
+    T, rs = on.stencil_reduction_run(t0, p, steps)
+    with runner.session(mm.MM_APP_STENCIL_REDUCTION, [rows, cols, steps, 1, 1, 1], G=3) as s:
+        s.fill()
+        plan = s.plan(mm.MM_SP_VARIED, _prof(mm, 3, 2), halo_split=True)
+        s.run(plan)
+        got = s.collect(plan, 1).reshape(rows, cols)
+        rowsum = s.collect(plan, 3)
+    assert np.array_equal(got, T)
+    import math
+    assert abs(math.fsum(rowsum) - rs[-1]) <= 1e-12 * abs(rs[-1])

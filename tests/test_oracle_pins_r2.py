@@ -362,3 +362,80 @@ def test_dp_perf_random_latency_parity():
             assert [c.device for c in ch] == dev and [c.finish_ns for c in ch] == fin
             mm.mm_plan_destroy(plan)
         mm.mm_app_destroy(capp)
+
+
+# ------------------------------------------------ halo overlap split (R33) --
+def _elems_pulled(ops):
+    """{(dst, src, buffer, element)} of the device-to-device pulls."""
+    out = set()
+    for o in ops:
+        if o[0] == oc.OP_XFER and o[2] >= 0:
+            out |= {(o[1], o[2], o[3], x) for x in range(o[4], o[5])}
+    return out
+
+
+@pytest.mark.parametrize("G,tb", [(2, 1), (3, 1), (3, 4), (4, 2)])
+def test_halo_split_same_work_and_pulls(G, tb):
+    """R33 only cuts each device's SP task (P249: one task of size n_d per
+    invocation) into interior + boundary pieces: per invocation and device the
+    pieces cover exactly the unsplit task's items, the interior piece comes
+    first, needs no halo pulled from another device, and the program pulls
+    exactly the same elements as the unsplit one."""
+    rows, cols, iters = 97, 8, 12
+    app = oa.hotspot(rows, cols, iters, tb=tb)
+    prof = oc.Profile(G=G, fs_item=[[1000 + 150 * d] for d in range(G)], chunk_est_ns=[[1]] * G,
+                      link_Bps=[10 ** 9] * G)
+    ranges = oc.sp_split(app, prof, oc.SP_SINGLE)
+    t0, d0 = oc.sp_tasks(app, ranges)
+    t1, d1 = oc.sp_tasks_halo_split(app, ranges)
+    cover0, cover1 = {}, {}
+    for t, d in zip(t0, d0):
+        cover0.setdefault((t.inv, d), set()).update(range(t.begin, t.end))
+    for t, d in zip(t1, d1):
+        s = cover1.setdefault((t.inv, d), set())
+        assert not (s & set(range(t.begin, t.end)))
+        s.update(range(t.begin, t.end))
+    assert cover0 == cover1
+    ops0 = oc.op_program(app, G, t0, d0, oc.SP_SINGLE)
+    ops1 = oc.op_program(app, G, t1, d1, oc.SP_SINGLE)
+    assert _elems_pulled(ops0) == _elems_pulled(ops1)
+    # interior pieces (the first of a split (invocation, device)) need no
+    # pull: op_program emits a task's pulls right before its KERNEL op
+    pieces = {}
+    for t, d in zip(t1, d1):
+        pieces[(t.inv, d)] = pieces.get((t.inv, d), 0) + 1
+    seen, n_interior = set(), 0
+    pending = []            # pulls since the previous KERNEL op
+    for o in ops1:
+        if o[0] == oc.OP_XFER and o[2] >= 0:
+            pending.append(o)
+        elif o[0] == oc.OP_KERNEL:
+            inv = next(i for i, (k, it) in enumerate(oc.invocations(app)) if it == o[3])
+            key = (inv, o[1])
+            if key not in seen and pieces[key] > 1:
+                assert not [x for x in pending if x[1] == o[1]], (key, pending)
+                n_interior += 1
+            seen.add(key)
+            pending = []
+    assert n_interior > 0
+
+
+@pytest.mark.parametrize("G,tb", [(2, 1), (3, 4), (3, 8)])
+def test_halo_split_cpp_matches_oracle(G, tb):
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    rows, cols, iters = 150, 8, 16
+    capp = mm.mm_app_builtin(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1, tb])
+    oapp = oa.hotspot(rows, cols, iters, 1, 1, tb)
+    fs = [[1000 + 150 * d] for d in range(G)]
+    pc = mm.make_profile(G, fs, [[1]] * G, [10 ** 9] * G)
+    po = oc.Profile(G=G, fs_item=fs, chunk_est_ns=[[1]] * G, link_Bps=[10 ** 9] * G)
+    plan = mm.mm_plan_build(capp, pc, mm.plan_opts(mm.MM_SP_SINGLE, one_shot=True, halo_split=True))
+    ranges = oc.sp_split(oapp, po, oc.SP_SINGLE)
+    tasks, dev = oc.sp_tasks_halo_split(oapp, ranges)
+    ch = mm.mm_plan_chunks(plan)
+    assert [c.device for c in ch] == dev
+    assert [(c.items.begin, c.items.end) for c in ch] == [(t.begin, t.end) for t in tasks]
+    from test_control_parity import ops_as_tuples
+    assert ops_as_tuples(plan) == oc.op_program(oapp, G, tasks, dev, oc.SP_SINGLE)
+    mm.mm_plan_destroy(plan)
+    mm.mm_app_destroy(capp)
