@@ -268,6 +268,9 @@ def main():
     ap.add_argument("--chol-n", type=int, default=None, help="Cholesky order n (default 32768)")
     ap.add_argument("--pipeline", type=int, default=32,
                     help="e2e staged pipeline sub-chunks per device (R24; 8: 171.5, 16: 174.1, 32: 176.4, 64: 175.4 GB/s STREAM)")
+    ap.add_argument("--halo-split", default="auto", choices=["auto", "on", "off"],
+                    help="R33: SP ranges of halo-reading kernels run interior-first so the interior overlaps "
+                         "the halo pulls (auto = on when the job spans more than one device)")
     ap.add_argument("--no-graph", action="store_true",
                     help="timed steps issue the op program eagerly instead of replaying a CUDA graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -347,7 +350,8 @@ def main():
     cls = mm.mm_classify(sess.app)
     ranked = mm.mm_rank(cls, mm.mm_needs_sync(sess.app))
     best = ranked[0]
-    plan = sess.plan(best, prof)
+    halo_split = args.halo_split == "on" or (args.halo_split == "auto" and G > 1)
+    plan = sess.plan(best, prof, halo_split=halo_split)
     info = mm.mm_plan_info(plan)
     K = sess.K
 
@@ -617,6 +621,7 @@ def main():
                        "issue": ("other timed steps: the op program replayed as a CUDA graph, enqueued back to back"
                                  if fast["use_graph"] else "other timed steps: eager issue, enqueued back to back"),
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
+                       "halo_split": halo_split,
                        **({"temporal_block": tb} if args.app == "hotspot" else {})},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": gpu_launches,
             "clocks": clk.summary(), "strategies_ms": strategies, "strategies_graph_ms": strategies_graph,
