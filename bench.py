@@ -405,9 +405,10 @@ def main():
                 ev0.record(stream)
             kt = args.kernel_timing == "all" or (args.kernel_timing == "last" and i >= args.steps - n_last)
             st = step(plan, time_kernels=True) if kt else step(plan, **fast)
-            for d in range(G):
-                for k in range(K):
-                    kms[d][k] += st.kernel_ms[d][k]
+            if kt:
+                for d in range(G):
+                    for k in range(K):
+                        kms[d][k] += st.kernel_ms[d][k]
             launches += st.n_launches
             if pristine or i == args.steps - 1:
                 ev1 = torch.cuda.Event(enable_timing=True)

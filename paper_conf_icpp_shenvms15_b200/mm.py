@@ -222,8 +222,16 @@ def _check(st: int, fn: str):
         raise MMError(st, fn, (lib.mm_last_error() or b"").decode())
 
 
+_FN = {}
+
+
 def _call(fn: str, *args):
-    _check(getattr(lib, fn)(*args), fn)
+    f = _FN.get(fn)
+    if f is None:
+        f = _FN[fn] = getattr(lib, fn)
+    st = f(*args)
+    if st:
+        _check(st, fn)
 
 
 # --------------------------------------------------------- same-name calls --

@@ -65,6 +65,12 @@ class Session:
                 if self.mine[d]:
                     self.bufs[(s, d)] = torch.empty(max(n, 1), dtype=_DT[eb],
                                                     device=f"cuda:{cuda_devices[d]}")
+        # register the buffers once (mm_buffer_register): runs then pass no
+        # pointer array (mm_run with buffers == NULL)
+        ptrs = self.ptrs()
+        for slot in range(self.nbuf):
+            eb, n = mm.mm_app_buffer_info(app, slot)
+            mm.mm_buffer_register(self.ctx, eb, n, ptrs[slot * G:(slot + 1) * G])
         self.plans: List[int] = []
         self.tile = 0   # Cholesky tile size (set by session())
 
@@ -145,7 +151,7 @@ class Session:
         return p
 
     def run(self, plan: int, **kw) -> mm.mm_run_stats:
-        return mm.mm_run(self.ctx, plan, self.ptrs(), **kw)
+        return mm.mm_run(self.ctx, plan, None, **kw)   # the registered buffers
 
     def tune_chunks(self, strategy: int, prof: mm.mm_profile, candidates=(1, 2, 4, 8, 16, 32), reps: int = 3,
                     **opts):
