@@ -279,7 +279,7 @@ def main():
     ap.add_argument("--no-profile", action="store_true",
                     help="use an equal synthetic profile instead of measuring one (ncu runs)")
     ap.add_argument("--kernel-timing", default="last", choices=["all", "last", "none"],
-                    help="per-kernel CUDA events in the timed steps: every step, the last ceil(K/5) steps, or none")
+                    help="per-kernel CUDA events in the timed steps: every step, the last step, or none")
     ap.add_argument("--share-gpu", action="store_true",
                     help="ranks share GPUs (rank r on cuda:r %% count): exercises the multi-process "
                          "IPC path on a box with fewer GPUs than ranks; not a scaling measurement")
@@ -379,8 +379,8 @@ def main():
 
     # timed steps: the op program replayed as one CUDA graph, enqueued without
     # a host round trip per step (mm_run no_wait; steps are ordered on the
-    # library's streams); the last ceil(K/5) steps run eagerly with CUDA events
-    # around every kernel for the roofline (--kernel-timing)
+    # library's streams); the last step runs eagerly with CUDA events around
+    # every kernel for the roofline (--kernel-timing)
     graph_ok = world == 1 or os.environ.get("MM_TRANSPORT") != "nccl"
     fast = dict(use_graph=graph_ok and not args.no_graph, no_wait=True)
     for w in range(args.warmup):
@@ -395,7 +395,11 @@ def main():
     kms = [[0.0] * K for _ in range(G)]
     launches = 0
     spans = []
-    n_last = max(1, (args.steps + 4) // 5)   # --kernel-timing last: the last ceil(K/5) timed steps
+    # --kernel-timing last: the final timed step carries CUDA events around every
+    # kernel; it runs eagerly and blocks once (the other steps are graph replays
+    # enqueued back to back), so timing more steps would add host round trips
+    # to the measured region
+    n_last = 1
     with ClockSampler(local) as clk:
         for i in range(args.steps):
             if pristine or i == 0:
