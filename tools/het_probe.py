@@ -1,5 +1,5 @@
 import numpy as np, torch, sys, time
-sys.path.insert(0, '/root/repo')
+sys.path.insert(0, __import__('os').path.dirname(__import__('os').path.dirname(__import__('os').path.abspath(__file__))))
 import synthgen
 from oracle import numeric as on
 from paper_conf_icpp_shenvms15_b200 import mm, runner

@@ -1,10 +1,14 @@
 """Host-side cost of one bench step (MatrixMul 1024^2, SP-Single) broken
 down per call: wall time per call averaged over many steps (GPU box)."""
+import os
+import sys
 import time
 
-import torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
-from paper_conf_icpp_shenvms15_b200 import mm, runner
+import torch  # noqa: E402
+
+from paper_conf_icpp_shenvms15_b200 import mm, runner  # noqa: E402
 
 
 def main(n=300):
@@ -34,6 +38,10 @@ def main(n=300):
     for _ in range(n):
         tm("mm_run(untimed)", lambda: mm.mm_run(s.ctx, plan, p))
         tm("mm_run(graph)", lambda: mm.mm_run(s.ctx, plan, p, use_graph=True))
+    torch.cuda.synchronize()
+    for _ in range(n):   # the bench's timed steps: registered buffers, graph, enqueue only
+        tm("mm_run(graph,no_wait)", lambda: mm.mm_run(s.ctx, plan, None, use_graph=True, no_wait=True))
+    torch.cuda.synchronize()
     for k, v in T.items():
         print(f"{k:18s} {v / n / 1000:8.2f} us")
     print("device ms (last timed run)", st.device_ms, "kernel ms", st.kernel_ms[0][0])
