@@ -392,7 +392,9 @@ typedef struct {
   int32_t measure_link;      /* link_Bps[d], Glinda's transfer metric (P49):
                                 0/1 (MM_LINK_PEER): 64 MiB copy into d from another
                                 logical device (peer GPU, else a device-to-device copy
-                                on the shared GPU); the resident exchange link.
+                                on the shared GPU; multi-process: a pull out of the
+                                next rank's memory through its IPC mapping); the
+                                resident exchange link.
                                 2 (MM_LINK_HOST): pinned host->device + device->host of
                                 64 MiB each, serialised (P119's staged transfers); sets
                                 mm_profile.staged = 1 so mm_split adds the transfer term */

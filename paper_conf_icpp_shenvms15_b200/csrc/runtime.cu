@@ -1924,9 +1924,20 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
             break;
           }
         CU_OK(cudaMalloc(&y, bytes));
+        void* peer_src = nullptr;   // multi-process: the next rank's buffer, mapped (IPC)
         if (host) {
           CU_OK(cudaMallocHost(&x, bytes));
           std::memset(x, 0, bytes);
+        } else if (ctx->ipc) {
+          // the exchange link of a rank = a pull out of the next rank's memory
+          // through its IPC mapping (NVLink between GPUs), as the XFERs do
+          CU_OK(cudaMalloc(&x, bytes));
+          CU_OK(cudaMemset(x, 0, bytes));
+          CU_OK(cudaDeviceSynchronize());
+          std::vector<char*> mapped;
+          mm_status st = ipc_exchange_buffers(ctx->ipc, std::vector<void*>{x}, mapped);
+          if (st) return st;
+          peer_src = mapped[(size_t)((ctx->my_rank + 1) % ctx->world)];
         } else {
           if (src_phys != ctx->dev[d].phys) CU_OK(cudaSetDevice(src_phys));
           CU_OK(cudaMalloc(&x, bytes));
@@ -1942,6 +1953,8 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
             if (host) {
               CU_OK(cudaMemcpyAsync(y, x, nb, cudaMemcpyHostToDevice, s));
               CU_OK(cudaMemcpyAsync(x, y, nb, cudaMemcpyDeviceToHost, s));
+            } else if (peer_src) {
+              CU_OK(cudaMemcpyAsync(y, peer_src, nb, cudaMemcpyDefault, s));
             } else if (src_phys != ctx->dev[d].phys) {
               CU_OK(cudaMemcpyPeerAsync(y, ctx->dev[d].phys, x, src_phys, nb, s));
             } else {
@@ -1959,6 +1972,10 @@ mm_status mm_profile_run(mm_ctx* ctx, const mm_app* app_h, void* const* buffers,
         if (mm_status r = time_copy(bytes, &best)) return r;
         // R32: the fixed cost of one transfer = a 4 KiB copy of the same kind
         if (mm_status r = time_copy(4096, &small)) return r;
+        if (peer_src) {   // no rank frees its buffer while a peer may still be pulling from it
+          CU_OK(cudaDeviceSynchronize());
+          if (mm_status st = ipc_barrier(ctx->ipc)) return st;
+        }
         if (host) cudaFreeHost(x);
         else cudaFree(x);
         cudaFree(y);

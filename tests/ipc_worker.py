@@ -30,6 +30,7 @@ CASES = {
     "stencil": (mm.MM_APP_STENCIL_REDUCTION, [200, 96, 5, 1, 1, 1], mm.MM_SP_VARIED, (1, 3), 2),
     "chol": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_DP_DEP, (0,), 1),
     "chol_cyclic": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_SP_CYCLIC, (0,), 1),
+    "profile": (mm.MM_APP_STREAM, [1 << 20, 1, 0, 32, 1], mm.MM_DP_PERF, (0,), 2),
 }
 
 
@@ -55,6 +56,13 @@ def main():
             s.load(0, A.reshape(T, b, T, b).transpose(0, 2, 1, 3).copy())
         else:
             s.fill()
+        if case == "profile":   # collective mm_profile_run: every rank returns the same profile
+            p = s.profile(reps=2)
+            np.savez(out, fs=np.array([[p.fs_item[d][k] for k in range(4)] for d in range(G)]),
+                     link=np.array([p.link_Bps[d] for d in range(G)]),
+                     lat=np.array([p.link_lat_ns[d] for d in range(G)]))
+            print(f"rank {rank} ok", flush=True)
+            return
         plan = s.plan(strategy, prof, chunks_per_dev=kpd, halo_split=case.endswith("_split"))
         for _ in range(runs):
             if app_id == mm.MM_APP_CHOLESKY and runs > 1:

@@ -111,3 +111,14 @@ def test_cholesky_multiprocess(tmp_path, case, graph):
     T = n // b
     L = got.reshape(T, T, b, b).transpose(0, 2, 1, 3).reshape(n, n)
     assert np.array_equal(np.tril(L), L0)
+
+
+def test_profile_multiprocess(tmp_path):
+    """mm_profile_run across 3 ranks: per-rank probes, the exchange link as a
+    pull out of the next rank's memory through its IPC mapping, rows
+    exchanged so every rank returns the same profile (P49)."""
+    res = run_ranks("profile", 3, tmp_path)
+    for r in res[1:]:
+        for key in ("fs", "link", "lat"):
+            assert np.array_equal(r[key], res[0][key]), key
+    assert (res[0]["fs"] > 0).all() and (res[0]["link"] > 10 ** 10).all() and (res[0]["lat"] > 0).all()
