@@ -1263,9 +1263,11 @@ mm_status mm_ctx_create(const mm_device_spec* devs, int32_t G, int32_t my_rank, 
       CU_OK(cudaStreamCreateWithFlags(&r.h2d, cudaStreamNonBlocking));
       CU_OK(cudaStreamCreateWithFlags(&r.d2h, cudaStreamNonBlocking));
       {  // lane 1 carries the critical path: highest stream priority
+         // (MM_LANE1_PRIO=0: default priority, development knob)
         int lo = 0, hi = 0;
         CU_OK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        CU_OK(cudaStreamCreateWithPriority(&r.lane1, cudaStreamNonBlocking, hi));
+        static const int p1 = getenv("MM_LANE1_PRIO") ? atoi(getenv("MM_LANE1_PRIO")) : 1;
+        CU_OK(cudaStreamCreateWithPriority(&r.lane1, cudaStreamNonBlocking, p1 ? hi : lo));
       }
       continue;
     }
