@@ -31,6 +31,8 @@ CASES = {
     "chol": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_DP_DEP, (0,), 1),
     "chol_cyclic": (mm.MM_APP_CHOLESKY, [1024, 256], mm.MM_SP_CYCLIC, (0,), 1),
     "profile": (mm.MM_APP_STREAM, [1 << 20, 1, 0, 32, 1], mm.MM_DP_PERF, (0,), 2),
+    "stream_staged": (mm.MM_APP_STREAM, [100003, 1, 0, 32, 1], mm.MM_SP_UNIFIED, (0, 1, 2), 2),
+    "stream_staged_dp": (mm.MM_APP_STREAM, [100003, 1, 1, 32, 1], mm.MM_DP_PERF, (0, 1, 2), 2),
 }
 
 
@@ -61,6 +63,24 @@ def main():
             np.savez(out, fs=np.array([[p.fs_item[d][k] for k in range(4)] for d in range(G)]),
                      link=np.array([p.link_Bps[d] for d in range(G)]),
                      lat=np.array([p.link_lat_ns[d] for d in range(G)]))
+            print(f"rank {rank} ok", flush=True)
+            return
+        if case.startswith("stream_staged"):
+            # staged (P119): inputs in this rank's pinned host memory, the run
+            # copies them in and flushes the outputs this rank produced back
+            import synthgen
+            n = ip[0]
+            host = [torch.from_numpy(x.copy()).pin_memory() for x in synthgen.stream_random(n)]
+            plan = s.plan(strategy, prof, chunks_per_dev=kpd, staged=True)
+            st = s.run(plan, host=[h.data_ptr() for h in host], use_graph=graph)
+            torch.cuda.synchronize()
+            res = {"xfer": np.array([st.xfer_bytes]), "h2d": np.array([st.h2d_bytes])}
+            for slot in slots:
+                segs = [(b0, e0) for (b0, e0, o) in mm.mm_plan_owners(plan, slot) if o == rank]
+                hv = host[slot].numpy()
+                res[f"r{slot}"] = np.array(segs, dtype=np.int64).reshape(-1, 2)
+                res[f"v{slot}"] = np.concatenate([hv[b0:e0] for b0, e0 in segs]) if segs else hv[:0]
+            np.savez(out, **res)
             print(f"rank {rank} ok", flush=True)
             return
         plan = s.plan(strategy, prof, chunks_per_dev=kpd, halo_split=case.endswith("_split"))

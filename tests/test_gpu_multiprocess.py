@@ -122,3 +122,19 @@ def test_profile_multiprocess(tmp_path):
         for key in ("fs", "link", "lat"):
             assert np.array_equal(r[key], res[0][key]), key
     assert (res[0]["fs"] > 0).all() and (res[0]["link"] > 10 ** 10).all() and (res[0]["lat"] > 0).all()
+
+
+@pytest.mark.parametrize("case", ["stream_staged", "stream_staged_dp"])
+@pytest.mark.parametrize("graph", [False, True])
+def test_stream_staged_multiprocess(tmp_path, case, graph):
+    """Staged mode across 2 ranks (P119's host-resident regime): each rank's
+    inputs start in its pinned host memory, and the outputs each rank
+    produced end there (FLUSH); DP-Perf with barriers also pulls chunk inputs
+    across processes."""
+    n = 100003
+    a0, b0, c0 = synthgen.stream_random(n)
+    ref = on.stream_run(a0, b0, c0, 1)
+    res = run_ranks(case, 2, tmp_path, graph=graph)
+    for slot in range(3):
+        assert np.array_equal(assemble(res, slot, n, np.float32), ref[slot]), (case, slot)
+    assert all(int(r["h2d"][0]) > 0 for r in res)
