@@ -122,6 +122,13 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
 cudaError_t chol_trsm_prepare(float* A, int64_t T, int64_t b, int32_t k, cudaStream_t s, Scratch* scr,
                               float** hi, float** lo, int32_t* slot0);
 void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, int32_t n);
+// TRSM of a batch of step-k tiles in one launch (kernels_chol_trsm.cu; b % 128
+// == 0, 256 <= b <= 4096, else cudaErrorNotSupported); MM_TRSM_COL=0 selects
+// the leaf path.  Its transposed L_kk leaves live after the POTRF flags.
+bool chol_trsm_col_enabled();
+size_t chol_trsm_lt_bytes(int64_t b);
+cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n, cudaStream_t s,
+                          Scratch* scr);
 cudaError_t chol_trsm_update_tc(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n,
                                 int32_t kx0, int32_t K, int32_t n0, cudaStream_t s, Scratch* scr,
                                 bool pdl = false);   // pdl: launched as a programmatic dependent of a leaf

@@ -1,0 +1,502 @@
+// Cholesky TRSM of one step's column in ONE launch (round 2): X_i <- A_ik
+// L_kk^{-T} for a batch of tiles i (substitution, no inverse;
+// reading R28), replacing the 8 leaf + 7 block-update launches per step of the
+// leaf path in kernels_chol.cu.
+//
+// A CTA owns 128 rows of one tile (grid = (b/128, tasks)); its rows are
+// independent of every other CTA's, so there is no cross-CTA traffic.  Left
+// looking over the 128-column leaves q = 0 .. b/128-1:
+//
+//   acc_q  = sum_{j<q} X_j L_qj^T           3xTF32 tcgen05.mma, M = N = 128,
+//                                            FP32 accumulator in TMEM
+//   leaf q: X_q = (B_q - acc_q) L_qq^{-T}    substitution, thread = row, four
+//                                            32-column sub-blocks in registers
+//
+// Warp roles (192 threads, one CTA per SM):
+//   warp 0   TMA producer: operand stages of the j <= q-2 terms (X_j hi/lo
+//            from the step's panel slot, written back by this CTA's earlier
+//            leaves; L_qj hi/lo from the L_kk slot) and the B half of the
+//            j = q-1 term
+//   warp 1   TMEM allocator (512 columns: acc A, acc B, X hi, X lo) and the
+//            single-thread MMA issuer; the j = q-1 term reads X_{q-1} straight
+//            from TMEM (TS form), so the critical hand-off leaf q-1 -> acc_q
+//            never goes through global memory
+//   warps 2-5 the substitution (TMEM lane = row).  A sub-block: x = B -
+//            acc (tcgen05.ld), minus the earlier sub-blocks of the leaf
+//            (accumulated first, ascending, as in the leaf kernels), then the
+//            32-column forward substitution with div_rcp quotients; the
+//            solved x goes to TMEM (fp32 into the consumed acc columns for
+//            the later sub-blocks, hi/lo for the MMA) and through a SWIZZLE_128B
+//            staging buffer to global memory by TMA stores (X into the tile,
+//            hi/lo into the panel slot the step's SYRK/GEMM and this CTA's
+//            later leaves read).
+// acc_{q+1}'s j <= q-1 terms run on the tensor pipe while leaf q substitutes.
+// The leaf's L_qq block arrives transposed with its reciprocal diagonal
+// (lkk_prep, one launch per step) by one bulk copy into shared memory.
+//
+// Exact-factor inputs stay exact (every product and partial sum an integer
+// below 2^24, every quotient exact), so the factor is L0 bit for bit; the
+// result of a tile does not depend on the batch it runs in.
+#include <cuda.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <vector>
+
+#include "kernels.h"
+#include "tc_ptx.h"
+
+namespace mm {
+
+cudaError_t encode_tmap_2d_f32(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer,
+                               uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer);
+size_t chol_potrf_flag_bytes(int64_t b);
+
+namespace {
+
+using namespace tcx;
+
+constexpr int kTcRows = 128, kTcLeaf = 128, kTcBK = 16, kTcStages = 3, kTcThreads = 192;
+constexpr int kTcOpBytes = kTcRows * kTcBK * 4;            // 8 KB: one operand box (16 fp32 x 128 rows)
+constexpr int kTcStageBytes = 4 * kTcOpBytes;               // A hi, A lo, B hi, B lo
+constexpr int kLtLd = kTcLeaf + 4;                          // LsT row stride (floats)
+constexpr int kLtFloats = kTcLeaf * kLtLd + kTcLeaf;        // LsT + reciprocal diagonal
+constexpr int kLtBytes = kLtFloats * 4;                     // 68096
+constexpr int kStgBytes = kTcRows * 32 * 4;                 // 16 KB: 128 rows x 32 fp32 (SWIZZLE_128B)
+constexpr int kMaxLeaves = 32;                              // b <= 4096
+constexpr int kSmRing = 0, kSmStg = kTcStages * kTcStageBytes, kSmLt = kSmStg + 3 * kStgBytes;
+constexpr int kSmBar = kSmLt + kLtBytes;
+constexpr int kTcSmem = kSmBar + 8 * (2 * kTcStages + 4 * kMaxLeaves) + 16 + 1024;
+
+struct ColJob {
+  int32_t n, k, slot0, nleaf;
+  int64_t T, b;
+  int32_t ti[kCholBatch];
+};
+
+__device__ __forceinline__ bool tw(uint64_t* b, uint32_t parity) {
+  uint32_t done;
+  asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+               : "=r"(done)
+               : "r"(saddr(b)), "r"(parity)
+               : "memory");
+  return done;
+}
+// mbarrier wait that traps after ~4 s instead of hanging the GPU
+__device__ __forceinline__ void twait(uint64_t* b, uint32_t parity) {
+  if (tw(b, parity)) return;
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    if (tw(b, parity)) return;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 4000000000ull) __trap();
+  }
+}
+
+__device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc), "r"(acc));
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t ta, float (&v)[32]) {
+  uint32_t* u = reinterpret_cast<uint32_t*>(v);
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(u[0]), "=r"(u[1]), "=r"(u[2]), "=r"(u[3]), "=r"(u[4]), "=r"(u[5]), "=r"(u[6]), "=r"(u[7]),
+        "=r"(u[8]), "=r"(u[9]), "=r"(u[10]), "=r"(u[11]), "=r"(u[12]), "=r"(u[13]), "=r"(u[14]), "=r"(u[15]),
+        "=r"(u[16]), "=r"(u[17]), "=r"(u[18]), "=r"(u[19]), "=r"(u[20]), "=r"(u[21]), "=r"(u[22]), "=r"(u[23]),
+        "=r"(u[24]), "=r"(u[25]), "=r"(u[26]), "=r"(u[27]), "=r"(u[28]), "=r"(u[29]), "=r"(u[30]), "=r"(u[31])
+      : "r"(ta));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_ld16(uint32_t ta, float (&v)[16]) {
+  uint32_t* u = reinterpret_cast<uint32_t*>(v);
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(u[0]), "=r"(u[1]), "=r"(u[2]), "=r"(u[3]), "=r"(u[4]), "=r"(u[5]), "=r"(u[6]), "=r"(u[7]),
+        "=r"(u[8]), "=r"(u[9]), "=r"(u[10]), "=r"(u[11]), "=r"(u[12]), "=r"(u[13]), "=r"(u[14]), "=r"(u[15])
+      : "r"(ta));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_st16(uint32_t ta, const float (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          ta),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]), "f"(v[8]), "f"(v[9]),
+      "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st32(uint32_t ta, const float (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(ta),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]), "f"(v[8]),
+      "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15]), "f"(v[16]),
+      "f"(v[17]), "f"(v[18]), "f"(v[19]), "f"(v[20]), "f"(v[21]), "f"(v[22]), "f"(v[23]), "f"(v[24]),
+      "f"(v[25]), "f"(v[26]), "f"(v[27]), "f"(v[28]), "f"(v[29]), "f"(v[30]), "f"(v[31])
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, int32_t x, int32_t y, const void* src) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"((uint64_t)map),
+               "r"(x), "r"(y), "r"(saddr(src))
+               : "memory");
+}
+
+__device__ __forceinline__ float div_q(float a, float b, float y) {   // = kernels_chol.cu div_rcp
+  const float q0 = __fmul_rn(a, y);
+  const float r = __fmaf_rn(-b, q0, a);
+  return __fmaf_rn(r, y, q0);
+}
+
+__global__ void __launch_bounds__(kTcThreads, 1)
+    trsm_col(float* __restrict__ A, const float* __restrict__ lt, const __grid_constant__ CUtensorMap tLhi,
+             const __grid_constant__ CUtensorMap tLlo, const __grid_constant__ CUtensorMap tSx,
+             const __grid_constant__ CUtensorMap tShi, const __grid_constant__ CUtensorMap tSlo,
+             const __grid_constant__ ColJob job) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* ring = base + kSmRing;
+  float* stg = reinterpret_cast<float*>(base + kSmStg);       // [3][128 rows][32] swizzled: x, hi, lo
+  float* LsT = reinterpret_cast<float*>(base + kSmLt);        // LsT[m][c] = L[c0+c][c0+m], then rd[128]
+  uint64_t* full = reinterpret_cast<uint64_t*>(base + kSmBar);
+  uint64_t* empty = full + kTcStages;
+  uint64_t* tfull = empty + kTcStages;      // [leaf] acc_q complete (MMA commit)
+  uint64_t* xtm = tfull + kMaxLeaves;       // [leaf] X_q in TMEM, acc buffer of leaf q free (128 arrivals)
+  uint64_t* xgl = xtm + kMaxLeaves;         // [leaf] X_q hi/lo in global (TMA stores complete)
+  uint64_t* lsb = xgl + kMaxLeaves;         // [leaf] LsT of leaf q in smem
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(lsb + kMaxLeaves);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nleaf = job.nleaf;
+  const int64_t b = job.b;
+  const int32_t ti = job.ti[blockIdx.y];
+  const int32_t r0 = (int32_t)blockIdx.x * kTcRows;                        // rows of the tile
+  const int32_t ya = (job.slot0 + ti) * (int32_t)b + r0;                   // panel slot rows (X_i)
+  const int32_t yl = (job.slot0 + job.k) * (int32_t)b;                     // L_kk slot rows
+  const int32_t yx = (int32_t)(((int64_t)ti * job.T + job.k) * b) + r0;    // rows of A (tile (ti, k))
+  const bool issuer = threadIdx.x == 64;                                   // warp 2 lane 0
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kTcStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int q = 0; q < kMaxLeaves; ++q) {
+      mbar_init(&tfull[q], 1);
+      mbar_init(&xtm[q], 128);
+      mbar_init(&xgl[q], 1);
+      mbar_init(&lsb[q], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tLhi) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tLlo) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(saddr(tslot)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {   // ===== TMA producer
+      int it = 0;
+      for (int q = 1; q < nleaf; ++q) {
+        const int32_t yb = yl + q * kTcLeaf;
+        for (int j = 0; j <= q - 1; ++j) {
+          const bool ts = j == q - 1;                 // X_{q-1} comes from TMEM
+          if (!ts && j == q - 2) twait(&xgl[j], 0);   // X_j of this CTA's leaf j is in global memory
+          for (int kb = 0; kb < kTcLeaf / kTcBK; ++kb, ++it) {
+            const int s = it % kTcStages;
+            if (it >= kTcStages) twait(&empty[s], (uint32_t)(((it / kTcStages) - 1) & 1));
+            uint8_t* st = ring + s * kTcStageBytes;
+            const int32_t kx = j * kTcLeaf + kb * kTcBK;
+            mbar_expect_tx(&full[s], ts ? 2 * kTcOpBytes : kTcStageBytes);
+            if (!ts) {
+              tma_load_2d(st, &tLhi, kx, ya, &full[s]);
+              tma_load_2d(st + kTcOpBytes, &tLlo, kx, ya, &full[s]);
+            }
+            tma_load_2d(st + 2 * kTcOpBytes, &tLhi, kx, yb, &full[s]);
+            tma_load_2d(st + 3 * kTcOpBytes, &tLlo, kx, yb, &full[s]);
+          }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0) {   // ===== MMA issuer
+      const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(kTcLeaf >> 3) << 17) |
+                             ((uint32_t)(kTcRows >> 4) << 24);
+      int it = 0;
+      for (int q = 1; q < nleaf; ++q) {
+        const uint32_t acc = tmem + (uint32_t)((q & 1) * 128);
+        if (q >= 2) twait(&xtm[q - 2], 0);   // leaf q-2 no longer reads this accumulator
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        bool first = true;
+        for (int j = 0; j <= q - 1; ++j) {
+          const bool ts = j == q - 1;
+          if (ts) {
+            twait(&xtm[q - 1], 0);           // X_{q-1} hi/lo stored in TMEM
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          }
+          for (int kb = 0; kb < kTcLeaf / kTcBK; ++kb, ++it) {
+            const int s = it % kTcStages;
+            twait(&full[s], (uint32_t)((it / kTcStages) & 1));
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            uint8_t* st = ring + s * kTcStageBytes;
+            const uint64_t bhi = sdesc(st + 2 * kTcOpBytes), blo = sdesc(st + 3 * kTcOpBytes);
+#pragma unroll
+            for (int kk = 0; kk < kTcBK / 8; ++kk) {
+              const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+              if (ts) {
+                const uint32_t ahi = tmem + 256u + (uint32_t)(kb * kTcBK + kk * 8), alo = ahi + 128u;
+                mma_ts(acc, alo, bhi + adv, idesc, first ? 0u : 1u);
+                mma_ts(acc, ahi, blo + adv, idesc, 1u);
+                mma_ts(acc, ahi, bhi + adv, idesc, 1u);
+              } else {
+                const uint64_t ahi = sdesc(st), alo = sdesc(st + kTcOpBytes);
+                mma_tf32(acc, alo + adv, bhi + adv, idesc, first ? 0u : 1u);
+                mma_tf32(acc, ahi + adv, blo + adv, idesc, 1u);
+                mma_tf32(acc, ahi + adv, bhi + adv, idesc, 1u);
+              }
+              first = false;
+            }
+            mma_commit(&empty[s]);
+          }
+        }
+        mma_commit(&tfull[q]);
+      }
+    }
+    __syncwarp();
+  } else {   // ===== substitution: warps 2..5, row = TMEM lane
+    const int grp = warp & 3, rr = grp * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(grp * 32) << 16;
+    const float* brow = A + ((int64_t)yx + rr) * b;   // this row of tile (ti, k): B, then X
+    const float* rd = LsT + kTcLeaf * kLtLd;
+    if (issuer) {   // LsT of leaf 0
+      mbar_expect_tx(&lsb[0], kLtBytes);
+      asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                       saddr(LsT)),
+                   "l"(lt), "r"(kLtBytes), "r"(saddr(&lsb[0]))
+                   : "memory");
+    }
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(brow) : "memory");
+#pragma unroll 1
+    for (int q = 0; q < nleaf; ++q) {
+      const int c0 = q * kTcLeaf;
+      const uint32_t accq = tmem + (uint32_t)((q & 1) * 128) + lane_off;
+      twait(&lsb[q], 0);
+      if (q >= 1) {
+        twait(&tfull[q], 0);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      }
+#pragma unroll 1
+      for (int s = 0; s < 4; ++s) {
+        float x[32];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {   // B (its line was prefetched into L1 one sub-block ahead)
+          const float4 v = *reinterpret_cast<const float4*>(brow + c0 + 32 * s + 4 * u);
+          x[4 * u] = v.x; x[4 * u + 1] = v.y; x[4 * u + 2] = v.z; x[4 * u + 3] = v.w;
+        }
+        if (c0 + 32 * s + 32 < b)
+          asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + c0 + 32 * s + 32) : "memory");
+        if (q >= 1) {
+          float a[32];
+          tmem_ld32(accq + (uint32_t)(32 * s), a);
+#pragma unroll
+          for (int c = 0; c < 32; ++c) x[c] -= a[c];
+        }
+        if (s > 0) {   // earlier sub-blocks of this leaf: accumulate ascending, subtract once
+          float acc[32];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) acc[c] = 0.f;
+#pragma unroll 1
+          for (int m0 = 0; m0 < 32 * s; m0 += 16) {
+            float xm[16];
+            tmem_ld16(accq + (uint32_t)m0, xm);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              const float4* l4 = reinterpret_cast<const float4*>(LsT + (m0 + i) * kLtLd + 32 * s);
+#pragma unroll
+              for (int u = 0; u < 8; ++u) {
+                const float4 l = l4[u];
+                acc[4 * u + 0] = fmaf(xm[i], l.x, acc[4 * u + 0]);
+                acc[4 * u + 1] = fmaf(xm[i], l.y, acc[4 * u + 1]);
+                acc[4 * u + 2] = fmaf(xm[i], l.z, acc[4 * u + 2]);
+                acc[4 * u + 3] = fmaf(xm[i], l.w, acc[4 * u + 3]);
+              }
+            }
+          }
+#pragma unroll
+          for (int c = 0; c < 32; ++c) x[c] -= acc[c];
+        }
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+          const float* lc = LsT + (32 * s + c) * kLtLd + 32 * s;   // lc[c2] = L[c0+32s+c2][c0+32s+c]
+          x[c] = div_q(x[c], lc[c], rd[32 * s + c]);
+#pragma unroll
+          for (int c2 = c + 1; c2 < 32; ++c2) x[c2] -= x[c] * lc[c2];
+        }
+        // fp32 x into the consumed accumulator columns, hi/lo for the MMA
+        tmem_st32(accq + (uint32_t)(32 * s), x);
+        // staging (SWIZZLE_128B: 16-B chunk u of row r at chunk u ^ (r & 7)) -> TMA stores
+        if (issuer) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {
+          float h[16], l[16];
+#pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            h[c] = tf32_rn(x[16 * hh + c]);
+            l[c] = tf32_rn(x[16 * hh + c] - h[c]);
+          }
+          tmem_st16(tmem + 256u + lane_off + (uint32_t)(32 * s + 16 * hh), h);
+          tmem_st16(tmem + 384u + lane_off + (uint32_t)(32 * s + 16 * hh), l);
+#pragma unroll
+          for (int v = 0; v < 4; ++v) {
+            const int u = 4 * hh + v, off = rr * 32 + ((u ^ (rr & 7)) * 4);
+            *reinterpret_cast<float4*>(stg + off) = make_float4(x[4 * u], x[4 * u + 1], x[4 * u + 2], x[4 * u + 3]);
+            *reinterpret_cast<float4*>(stg + 4096 + off) = make_float4(h[4 * v], h[4 * v + 1], h[4 * v + 2], h[4 * v + 3]);
+            *reinterpret_cast<float4*>(stg + 8192 + off) = make_float4(l[4 * v], l[4 * v + 1], l[4 * v + 2], l[4 * v + 3]);
+          }
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (issuer) {
+          const int32_t xc = c0 + 32 * s;
+          tma_store_2d(&tSx, xc, yx, stg);
+          tma_store_2d(&tShi, xc, ya, stg + 4096);
+          tma_store_2d(&tSlo, xc, ya, stg + 8192);
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+      // leaf q done: X_q in TMEM (and this accumulator free), LsT free
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      mbar_arrive(&xtm[q]);
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (issuer) {
+        if (q + 1 < nleaf) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          mbar_expect_tx(&lsb[q + 1], kLtBytes);
+          asm volatile(
+              "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                  saddr(LsT)),
+              "l"(lt + (int64_t)(q + 1) * kLtFloats), "r"(kLtBytes), "r"(saddr(&lsb[q + 1]))
+              : "memory");
+        }
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // X_q in global: the producer may load it
+        asm volatile("fence.proxy.async.global;" ::: "memory");
+        mbar_arrive(&xgl[q]);
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+  }
+}
+
+// Per step: L_kk split into its panel slot (hi/lo, = split_tiles) and, per
+// leaf q, LsT_q[m][c] = L[c0+c][c0+m] (c0 = 128 q) followed by RN(1/L[c0+m][c0+m]).
+__global__ void __launch_bounds__(256) lkk_prep(const float* __restrict__ L, float* __restrict__ hi,
+                                                float* __restrict__ lo, float* __restrict__ lt, int b, int nsplit) {
+  __shared__ float t[32][33];
+  if ((int)blockIdx.x < nsplit) {
+    const int64_t n4 = (int64_t)b * b / 4;
+    for (int64_t e = (int64_t)blockIdx.x * 256 + threadIdx.x; e < n4; e += (int64_t)nsplit * 256) {
+      const float4 x = reinterpret_cast<const float4*>(L)[e];
+      float4 h, l;
+      split2(x.x, h.x, l.x);
+      split2(x.y, h.y, l.y);
+      split2(x.z, h.z, l.z);
+      split2(x.w, h.w, l.w);
+      reinterpret_cast<float4*>(hi)[e] = h;
+      reinterpret_cast<float4*>(lo)[e] = l;
+    }
+    return;
+  }
+  const int idx = (int)blockIdx.x - nsplit, q = idx / 16, mi = (idx % 16) / 4, ci = idx % 4;
+  const int c0 = q * kTcLeaf, tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  float* dst = lt + (int64_t)q * kLtFloats;
+#pragma unroll
+  for (int j = ty; j < 32; j += 8)   // t[c][m] = L[c0 + 32ci + c][c0 + 32mi + m]
+    t[j][tx] = L[(int64_t)(c0 + 32 * ci + j) * b + c0 + 32 * mi + tx];
+  __syncthreads();
+#pragma unroll
+  for (int j = ty; j < 32; j += 8)   // LsT[32mi + j][32ci + tx] = t[tx][j]
+    dst[(32 * mi + j) * kLtLd + 32 * ci + tx] = t[tx][j];
+  if (mi == ci && threadIdx.x < 32)
+    dst[kTcLeaf * kLtLd + 32 * mi + tx] = __frcp_rn(t[tx][tx]);
+}
+
+}  // namespace
+
+size_t chol_trsm_lt_bytes(int64_t b) { return (size_t)(b / kTcLeaf) * kLtBytes; }
+
+bool chol_trsm_col_enabled() {
+  static const int env = getenv("MM_TRSM_COL") ? atoi(getenv("MM_TRSM_COL")) : 1;
+  return env != 0;
+}
+
+// One launch per batch; the step's L_kk preparation once per step and device
+// (split tag of slot k, as chol_trsm_prepare).
+cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n, cudaStream_t s,
+                          Scratch* scr) {
+  if (n <= 0) return cudaSuccess;
+  if (b % kTcLeaf != 0 || b / kTcLeaf > kMaxLeaves || b < 2 * kTcLeaf) return cudaErrorNotSupported;
+  if (!scr || !scr->ptr || scr->bytes < chol_scratch_bytes(T, b)) return cudaErrorNotSupported;
+  float* hi = static_cast<float*>(scr->ptr);
+  float* lo = hi + 2 * T * b * b;
+  float* lt = reinterpret_cast<float*>(static_cast<char*>(scr->ptr) + chol_tc_scratch(T, b) +
+                                       chol_potrf_flag_bytes(b));
+  const int32_t slot0 = (k & 1) * (int32_t)T;
+  static std::atomic<uint64_t> attr{0};
+  cudaError_t e = once_per_device(attr, [] {
+    return cudaFuncSetAttribute(trsm_col, cudaFuncAttributeMaxDynamicSharedMemorySize, kTcSmem);
+  });
+  if (e != cudaSuccess) return e;
+  if (scr->panel.size() != (size_t)(2 * T)) scr->panel.assign(2 * T, 0);
+  const uint64_t tag = (scr->epoch << 20) | (uint64_t)(k + 1);   // = kernels_gemm_tc.cu split_tag
+  if (scr->panel[slot0 + k] != tag) {
+    scr->panel[slot0 + k] = tag;
+    const int nsplit = 64;
+    note_launch();
+    lkk_prep<<<(unsigned)(nsplit + (b / kTcLeaf) * 16), 256, 0, s>>>(A + ((int64_t)k * T + k) * b * b,
+                                                                     hi + (slot0 + k) * b * b,
+                                                                     lo + (slot0 + k) * b * b, lt, (int)b, nsplit);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  CUtensorMap mLhi, mLlo, mSx, mShi, mSlo;
+  if ((e = encode_tmap_2d_f32(&mLhi, hi, b, 2 * T * b, b * 4, kTcBK, kTcRows)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&mLlo, lo, b, 2 * T * b, b * 4, kTcBK, kTcRows)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&mSx, A, b, T * T * b, b * 4, 32, kTcRows)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&mShi, hi, b, 2 * T * b, b * 4, 32, kTcRows)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&mSlo, lo, b, 2 * T * b, b * 4, 32, kTcRows)) != cudaSuccess) return e;
+  ColJob job;
+  job.k = k;
+  job.slot0 = slot0;
+  job.nleaf = (int32_t)(b / kTcLeaf);
+  job.T = T;
+  job.b = b;
+  for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
+    job.n = std::min<int32_t>(kCholBatch, n - q0);
+    for (int32_t q = 0; q < job.n; ++q) job.ti[q] = ti[q0 + q];
+    note_launch();
+    trsm_col<<<dim3((unsigned)(b / kTcRows), (unsigned)job.n), kTcThreads, kTcSmem, s>>>(A, lt, mLhi, mLlo, mSx, mShi,
+                                                                                       mSlo, job);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  for (int32_t q = 0; q < n; ++q) scr->panel[slot0 + ti[q]] = tag;
+  return cudaSuccess;
+}
+
+}  // namespace mm

@@ -449,26 +449,44 @@ def test_cholesky_random_spd_schedule_invariant(R, nb):
         assert np.array_equal(got, ref), (strategy, G)
 
 
-def test_cholesky_trsm_leaf_variants_identical(gpu, tmp_path):
-    """The wide (one 256-row CTA per SM, large batches) and narrow (64-row
-    CTAs, small batches) TRSM leaves do the same arithmetic: forcing the wide
-    leaf for every batch (MM_LEAF_WIDE_MIN=1, a fresh process) gives the
-    default run's factor bit for bit."""
+def _chol_subprocess(tmp_path, tag, env_set, n=2048, b=512):
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    outs = []
-    for env_min in (None, "1"):
-        out = str(tmp_path / f"chol_{env_min}.npy")
-        env = dict(os.environ)
-        env.pop("MM_LEAF_WIDE_MIN", None)
-        if env_min:
-            env["MM_LEAF_WIDE_MIN"] = env_min
-        code = _CHOL_SCRIPT.format(root=root, n=2048, b=512, out=out)
-        subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=root, timeout=600)
-        outs.append(np.load(out))
-    assert np.array_equal(outs[0], outs[1])
+    out = str(tmp_path / f"chol_{tag}.npy")
+    env = dict(os.environ)
+    for key in ("MM_LEAF_WIDE_MIN", "MM_TRSM_COL"):
+        env.pop(key, None)
+    env.update(env_set)
+    code = _CHOL_SCRIPT.format(root=root, n=n, b=b, out=out)
+    subprocess.run([sys.executable, "-c", code], check=True, env=env, cwd=root, timeout=600)
+    return np.load(out)
+
+
+def test_cholesky_trsm_leaf_variants_identical(gpu, tmp_path):
+    """Leaf path (MM_TRSM_COL=0): the wide (one 256-row CTA per SM, large
+    batches) and narrow (64-row CTAs, small batches) TRSM leaves do the same
+    arithmetic: forcing the wide leaf for every batch (MM_LEAF_WIDE_MIN=1, a
+    fresh process) gives the leaf path's default factor bit for bit."""
+    a = _chol_subprocess(tmp_path, "leaf", {"MM_TRSM_COL": "0"})
+    w = _chol_subprocess(tmp_path, "wide", {"MM_TRSM_COL": "0", "MM_LEAF_WIDE_MIN": "1"})
+    assert np.array_equal(a, w)
+
+
+def test_cholesky_trsm_column_vs_leaf_path(gpu, tmp_path):
+    """The one-launch column TRSM (default, kernels_chol_trsm.cu: left-looking
+    over the 128-column leaves, one FP32 accumulation of the earlier leaves'
+    3xTF32 products) and the leaf path (right-looking: one subtraction per
+    earlier leaf) round differently on random SPD data but agree within the
+    3xTF32 tolerance, and both match the FP64 oracle (R28)."""
+    n, b = 2048, 512
+    col = _chol_subprocess(tmp_path, "col", {})
+    leaf = _chol_subprocess(tmp_path, "leaf", {"MM_TRSM_COL": "0"})
+    ref = on.cholesky(synthgen.spd_random(n).astype(np.float64))
+    for got in (col, leaf):
+        L = np.tril(_from_tiles(got, n, b)).astype(np.float64)
+        assert np.max(np.abs(L - ref)) / np.max(np.abs(ref)) <= 1e-4
 
 
 def test_cholesky_device_spd_generator(R):
