@@ -40,6 +40,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <vector>
 
@@ -59,14 +60,21 @@ using namespace tcx;
 constexpr int kTcRows = 128, kTcLeaf = 128, kTcBK = 16, kTcStages = 3, kTcThreads = 192;
 constexpr int kTcOpBytes = kTcRows * kTcBK * 4;            // 8 KB: one operand box (16 fp32 x 128 rows)
 constexpr int kTcStageBytes = 4 * kTcOpBytes;               // A hi, A lo, B hi, B lo
-constexpr int kLtLd = kTcLeaf + 4;                          // LsT row stride (floats)
-constexpr int kLtFloats = kTcLeaf * kLtLd + kTcLeaf;        // LsT + reciprocal diagonal
-constexpr int kLtBytes = kLtFloats * 4;                     // 68096
+// The leaf's L block, packed as the 32 x 32 blocks the substitution reads
+// (all threads read the same address: broadcasts):
+//   U[s(s-1)/2 + mb][i][c] = L[c0+32s+c][c0+32mb+i]   s = 1..3, mb < s
+//   D[s][c][c2]            = L[c0+32s+c2][c0+32s+c]   s = 0..3
+//   rd[m]                  = RN(1 / L[c0+m][c0+m])
+constexpr int kLtU = 0, kLtD = 6 * 1024, kLtRd = 10 * 1024;
+constexpr int kLtFloats = kLtRd + kTcLeaf;
+constexpr int kLtBytes = kLtFloats * 4;                     // 41472
 constexpr int kStgBytes = kTcRows * 32 * 4;                 // 16 KB: 128 rows x 32 fp32 (SWIZZLE_128B)
 constexpr int kMaxLeaves = 32;                              // b <= 4096
-constexpr int kSmRing = 0, kSmStg = kTcStages * kTcStageBytes, kSmLt = kSmStg + 3 * kStgBytes;
-constexpr int kSmBar = kSmLt + kLtBytes;
-constexpr int kTcSmem = kSmBar + 8 * (2 * kTcStages + 4 * kMaxLeaves) + 16 + 1024;
+constexpr int kSmRing = 0, kSmStg = kTcStages * kTcStageBytes, kSmBpre = kSmStg + 3 * kStgBytes;
+constexpr int kSmLt = kSmBpre + 2 * kStgBytes, kSmBar = kSmLt + kLtBytes;
+constexpr int kNBar = 2 * kTcStages + 2 + 7 * kMaxLeaves;  // see trsm_col
+constexpr int kTcSmem = kSmBar + 8 * kNBar + 16 + 1024;
+constexpr int kStampsPerCta = 64;   // MM_TRSM_STAMPS: globaltimer per CTA (see trsm_col)
 
 struct ColJob {
   int32_t n, k, slot0, nleaf;
@@ -157,19 +165,23 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     trsm_col(float* __restrict__ A, const float* __restrict__ lt, const __grid_constant__ CUtensorMap tLhi,
              const __grid_constant__ CUtensorMap tLlo, const __grid_constant__ CUtensorMap tSx,
              const __grid_constant__ CUtensorMap tShi, const __grid_constant__ CUtensorMap tSlo,
-             const __grid_constant__ ColJob job) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* base = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+             const __grid_constant__ ColJob job, uint64_t* __restrict__ stamps) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  // 1024-B aligned (SWIZZLE_64B / 128B atoms), pointer arithmetic on the
+  // shared array so the accesses stay LDS/STS
+  uint8_t* base = smem_raw + ((1024u - (saddr(smem_raw) & 1023u)) & 1023u);
   uint8_t* ring = base + kSmRing;
   float* stg = reinterpret_cast<float*>(base + kSmStg);       // [3][128 rows][32] swizzled: x, hi, lo
-  float* LsT = reinterpret_cast<float*>(base + kSmLt);        // LsT[m][c] = L[c0+c][c0+m], then rd[128]
+  float* LsT = reinterpret_cast<float*>(base + kSmLt);        // packed leaf block (kLtU / kLtD / kLtRd)
   uint64_t* full = reinterpret_cast<uint64_t*>(base + kSmBar);
   uint64_t* empty = full + kTcStages;
-  uint64_t* tfull = empty + kTcStages;      // [leaf] acc_q complete (MMA commit)
-  uint64_t* xtm = tfull + kMaxLeaves;       // [leaf] X_q in TMEM, acc buffer of leaf q free (128 arrivals)
-  uint64_t* xgl = xtm + kMaxLeaves;         // [leaf] X_q hi/lo in global (TMA stores complete)
-  uint64_t* lsb = xgl + kMaxLeaves;         // [leaf] LsT of leaf q in smem
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(lsb + kMaxLeaves);
+  uint64_t* tfull = empty + kTcStages;        // [q] acc_q complete (MMA commit)
+  uint64_t* xsub = tfull + kMaxLeaves;        // [4q+s] hi/lo of X_q sub-block s in TMEM (128 arrivals)
+  uint64_t* xgl = xsub + 4 * kMaxLeaves;      // [q] X_q hi/lo in global (TMA stores complete)
+  uint64_t* lsb = xgl + kMaxLeaves;           // [q] L block of leaf q in smem
+  uint64_t* bful = lsb + kMaxLeaves;          // [2] B sub-block prefetch buffer loaded (tx)
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bful + 2);
+  float* bpre = reinterpret_cast<float*>(base + kSmBpre);    // [2][128 rows][32] swizzled: B sub-blocks
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nleaf = job.nleaf;
   const int64_t b = job.b;
@@ -187,10 +199,12 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     }
     for (int q = 0; q < kMaxLeaves; ++q) {
       mbar_init(&tfull[q], 1);
-      mbar_init(&xtm[q], 128);
       mbar_init(&xgl[q], 1);
       mbar_init(&lsb[q], 1);
+      for (int u = 0; u < 4; ++u) mbar_init(&xsub[4 * q + u], 128);
     }
+    mbar_init(&bful[0], 1);
+    mbar_init(&bful[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tLhi) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tLlo) : "memory");
@@ -203,6 +217,15 @@ __global__ void __launch_bounds__(kTcThreads, 1)
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tslot;
+  uint64_t* stp = stamps ? stamps + ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * kStampsPerCta : nullptr;
+  auto stamp = [&](int i) {
+    if (stp) {
+      uint64_t t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      stp[i] = t;
+    }
+  };
+  if (threadIdx.x == 0) stamp(0);
 
   if (warp == 0) {
     if (lane == 0) {   // ===== TMA producer
@@ -236,16 +259,39 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       int it = 0;
       for (int q = 1; q < nleaf; ++q) {
         const uint32_t acc = tmem + (uint32_t)((q & 1) * 128);
-        if (q >= 2) twait(&xtm[q - 2], 0);   // leaf q-2 no longer reads this accumulator
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        if (q >= 2) {   // leaf q-2 no longer reads accumulator q%2 (its last sub-block is stored)
+          twait(&xsub[4 * (q - 2) + 3], 0);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        }
         bool first = true;
-        for (int j = 0; j <= q - 1; ++j) {
-          const bool ts = j == q - 1;
-          if (ts) {
-            twait(&xtm[q - 1], 0);           // X_{q-1} hi/lo stored in TMEM
-            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          }
+        if (q < 8) stamp(17 + q);
+        for (int j = 0; j <= q - 2; ++j) {   // SS terms: X_j from the panel slot
           for (int kb = 0; kb < kTcLeaf / kTcBK; ++kb, ++it) {
+            const int s = it % kTcStages;
+            twait(&full[s], (uint32_t)((it / kTcStages) & 1));
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            uint8_t* st = ring + s * kTcStageBytes;
+            const uint64_t ahi = sdesc(st), alo = sdesc(st + kTcOpBytes);
+            const uint64_t bhi = sdesc(st + 2 * kTcOpBytes), blo = sdesc(st + 3 * kTcOpBytes);
+#pragma unroll
+            for (int kk = 0; kk < kTcBK / 8; ++kk) {
+              const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+              mma_tf32(acc, alo + adv, bhi + adv, idesc, first ? 0u : 1u);
+              first = false;
+              mma_tf32(acc, ahi + adv, blo + adv, idesc, 1u);
+              mma_tf32(acc, ahi + adv, bhi + adv, idesc, 1u);
+            }
+            mma_commit(&empty[s]);
+          }
+        }
+        // TS term j = q-1, one 32-column sub-block of X_{q-1} at a time as the
+        // substitution produces it (TMEM: hi at 256 + 32u, lo at 384 + 32u)
+        for (int u = 0; u < 4; ++u) {
+          twait(&xsub[4 * (q - 1) + u], 0);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          if (u == 0 && q < 8) stamp(25 + q);
+          const uint32_t xh = tmem + 256u + (uint32_t)(32 * u);
+          for (int h = 0; h < 2; ++h, ++it) {
             const int s = it % kTcStages;
             twait(&full[s], (uint32_t)((it / kTcStages) & 1));
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -254,23 +300,17 @@ __global__ void __launch_bounds__(kTcThreads, 1)
 #pragma unroll
             for (int kk = 0; kk < kTcBK / 8; ++kk) {
               const uint64_t adv = (uint64_t)(kk * 32) >> 4;
-              if (ts) {
-                const uint32_t ahi = tmem + 256u + (uint32_t)(kb * kTcBK + kk * 8), alo = ahi + 128u;
-                mma_ts(acc, alo, bhi + adv, idesc, first ? 0u : 1u);
-                mma_ts(acc, ahi, blo + adv, idesc, 1u);
-                mma_ts(acc, ahi, bhi + adv, idesc, 1u);
-              } else {
-                const uint64_t ahi = sdesc(st), alo = sdesc(st + kTcOpBytes);
-                mma_tf32(acc, alo + adv, bhi + adv, idesc, first ? 0u : 1u);
-                mma_tf32(acc, ahi + adv, blo + adv, idesc, 1u);
-                mma_tf32(acc, ahi + adv, bhi + adv, idesc, 1u);
-              }
+              const uint32_t ahi = xh + (uint32_t)(16 * h + 8 * kk), alo = ahi + 128u;
+              mma_ts(acc, alo, bhi + adv, idesc, first ? 0u : 1u);
               first = false;
+              mma_ts(acc, ahi, blo + adv, idesc, 1u);
+              mma_ts(acc, ahi, bhi + adv, idesc, 1u);
             }
             mma_commit(&empty[s]);
           }
         }
         mma_commit(&tfull[q]);
+        if (q < 8) stamp(33 + q);
       }
     }
     __syncwarp();
@@ -278,7 +318,15 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     const int grp = warp & 3, rr = grp * 32 + lane;
     const uint32_t lane_off = (uint32_t)(grp * 32) << 16;
     const float* brow = A + ((int64_t)yx + rr) * b;   // this row of tile (ti, k): B, then X
-    const float* rd = LsT + kTcLeaf * kLtLd;
+    const float* rd = LsT + kLtRd;
+    // B sub-blocks (32 columns x 128 rows of the tile) through a double
+    // buffer, TMA-loaded one sub-block ahead by the issuer
+    auto bload = [&](int idx) {   // idx = 4 q + s
+      if (idx >= 4 * nleaf) return;
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_expect_tx(&bful[idx & 1], kStgBytes);
+      tma_load_2d(bpre + (idx & 1) * 4096, &tSx, 32 * idx, yx, &bful[idx & 1]);
+    };
     if (issuer) {   // LsT of leaf 0
       mbar_expect_tx(&lsb[0], kLtBytes);
       asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
@@ -286,7 +334,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
                    "l"(lt), "r"(kLtBytes), "r"(saddr(&lsb[0]))
                    : "memory");
     }
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(brow) : "memory");
+    if (issuer) bload(0);
+    int pending = -1;   // leaf whose TMA stores the issuer has not waited for yet
 #pragma unroll 1
     for (int q = 0; q < nleaf; ++q) {
       const int c0 = q * kTcLeaf;
@@ -296,17 +345,22 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         twait(&tfull[q], 0);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       }
+      if (issuer && q < 8) stamp(1 + q);
 #pragma unroll 1
       for (int s = 0; s < 4; ++s) {
+        const int idx = 4 * q + s;
+        if (issuer) bload(idx + 1);
+        twait(&bful[idx & 1], (uint32_t)((idx >> 1) & 1));
         float x[32];
+        {
+          const float* bp = bpre + (idx & 1) * 4096 + rr * 32;
 #pragma unroll
-        for (int u = 0; u < 8; ++u) {   // B (its line was prefetched into L1 one sub-block ahead)
-          const float4 v = *reinterpret_cast<const float4*>(brow + c0 + 32 * s + 4 * u);
-          x[4 * u] = v.x; x[4 * u + 1] = v.y; x[4 * u + 2] = v.z; x[4 * u + 3] = v.w;
+          for (int u = 0; u < 8; ++u) {
+            const float4 v = *reinterpret_cast<const float4*>(bp + ((u ^ (rr & 7)) * 4));
+            x[4 * u] = v.x; x[4 * u + 1] = v.y; x[4 * u + 2] = v.z; x[4 * u + 3] = v.w;
+          }
         }
-        if (c0 + 32 * s + 32 < b)
-          asm volatile("prefetch.global.L1 [%0];" ::"l"(brow + c0 + 32 * s + 32) : "memory");
-        if (q >= 1) {
+        if (q >= 1) {   // x = B - sum_{j<q} X_j L_qj^T
           float a[32];
           tmem_ld32(accq + (uint32_t)(32 * s), a);
 #pragma unroll
@@ -322,7 +376,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             tmem_ld16(accq + (uint32_t)m0, xm);
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
-              const float4* l4 = reinterpret_cast<const float4*>(LsT + (m0 + i) * kLtLd + 32 * s);
+              const float4* l4 =
+                  reinterpret_cast<const float4*>(LsT + kLtU + (s * (s - 1) / 2 + (m0 >> 5)) * 1024 + ((m0 & 31) + i) * 32);
 #pragma unroll
               for (int u = 0; u < 8; ++u) {
                 const float4 l = l4[u];
@@ -338,15 +393,27 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         }
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
-          const float* lc = LsT + (32 * s + c) * kLtLd + 32 * s;   // lc[c2] = L[c0+32s+c2][c0+32s+c]
+          const float* lc = LsT + kLtD + s * 1024 + c * 32;   // lc[c2] = L[c0+32s+c2][c0+32s+c]
           x[c] = div_q(x[c], lc[c], rd[32 * s + c]);
 #pragma unroll
           for (int c2 = c + 1; c2 < 32; ++c2) x[c2] -= x[c] * lc[c2];
         }
         // fp32 x into the consumed accumulator columns, hi/lo for the MMA
         tmem_st32(accq + (uint32_t)(32 * s), x);
+        // hi/lo to TMEM columns 256 / 384 + 32 s (their previous contents, X_{q-1},
+        // were read by acc_q's MMAs, complete before tfull[q])
+        const uint32_t xslot = tmem + 256u + lane_off + (uint32_t)(32 * s);
         // staging (SWIZZLE_128B: 16-B chunk u of row r at chunk u ^ (r & 7)) -> TMA stores
-        if (issuer) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        if (issuer) {
+          if (pending >= 0) {   // the previous leaf's stores: complete, so the producer may load them
+            asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+            asm volatile("fence.proxy.async.global;" ::: "memory");
+            mbar_arrive(&xgl[pending]);
+            pending = -1;
+          } else {
+            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+          }
+        }
         asm volatile("bar.sync 1, 128;" ::: "memory");
 #pragma unroll
         for (int hh = 0; hh < 2; ++hh) {
@@ -356,8 +423,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             h[c] = tf32_rn(x[16 * hh + c]);
             l[c] = tf32_rn(x[16 * hh + c] - h[c]);
           }
-          tmem_st16(tmem + 256u + lane_off + (uint32_t)(32 * s + 16 * hh), h);
-          tmem_st16(tmem + 384u + lane_off + (uint32_t)(32 * s + 16 * hh), l);
+          tmem_st16(xslot + (uint32_t)(16 * hh), h);
+          tmem_st16(xslot + 128u + (uint32_t)(16 * hh), l);
 #pragma unroll
           for (int v = 0; v < 4; ++v) {
             const int u = 4 * hh + v, off = rr * 32 + ((u ^ (rr & 7)) * 4);
@@ -366,6 +433,9 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             *reinterpret_cast<float4*>(stg + 8192 + off) = make_float4(l[4 * v], l[4 * v + 1], l[4 * v + 2], l[4 * v + 3]);
           }
         }
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        mbar_arrive(&xsub[4 * q + s]);   // acc_{q+1}'s MMAs may read this sub-block
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         asm volatile("bar.sync 1, 128;" ::: "memory");
         if (issuer) {
@@ -376,12 +446,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         }
       }
-      // leaf q done: X_q in TMEM (and this accumulator free), LsT free
-      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-      mbar_arrive(&xtm[q]);
+      // leaf q done: LsT free, accumulator q%3 free after the x reads above
+      if (issuer && q < 8) stamp(9 + q);
       asm volatile("bar.sync 1, 128;" ::: "memory");
       if (issuer) {
+        pending = q;
         if (q + 1 < nleaf) {
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           mbar_expect_tx(&lsb[q + 1], kLtBytes);
@@ -391,11 +460,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
               "l"(lt + (int64_t)(q + 1) * kLtFloats), "r"(kLtBytes), "r"(saddr(&lsb[q + 1]))
               : "memory");
         }
-        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // X_q in global: the producer may load it
-        asm volatile("fence.proxy.async.global;" ::: "memory");
-        mbar_arrive(&xgl[q]);
       }
     }
+    if (issuer) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    if (issuer) stamp(41);
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
@@ -425,20 +493,57 @@ __global__ void __launch_bounds__(256) lkk_prep(const float* __restrict__ L, flo
     return;
   }
   const int idx = (int)blockIdx.x - nsplit, q = idx / 16, mi = (idx % 16) / 4, ci = idx % 4;
+  if (mi > ci) return;   // blocks above L's diagonal are never read
   const int c0 = q * kTcLeaf, tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
-  float* dst = lt + (int64_t)q * kLtFloats;
+  float* dst = lt + (int64_t)q * kLtFloats + (mi < ci ? kLtU + (ci * (ci - 1) / 2 + mi) * 1024 : kLtD + ci * 1024);
 #pragma unroll
   for (int j = ty; j < 32; j += 8)   // t[c][m] = L[c0 + 32ci + c][c0 + 32mi + m]
     t[j][tx] = L[(int64_t)(c0 + 32 * ci + j) * b + c0 + 32 * mi + tx];
   __syncthreads();
 #pragma unroll
-  for (int j = ty; j < 32; j += 8)   // LsT[32mi + j][32ci + tx] = t[tx][j]
-    dst[(32 * mi + j) * kLtLd + 32 * ci + tx] = t[tx][j];
+  for (int j = ty; j < 32; j += 8)   // [j][tx] = L[c0 + 32ci + tx][c0 + 32mi + j]
+    dst[j * 32 + tx] = t[tx][j];
   if (mi == ci && threadIdx.x < 32)
-    dst[kTcLeaf * kLtLd + 32 * mi + tx] = __frcp_rn(t[tx][tx]);
+    lt[(int64_t)q * kLtFloats + kLtRd + 32 * mi + tx] = __frcp_rn(t[tx][tx]);
 }
 
 }  // namespace
+
+// MM_TRSM_STAMPS=<file> (diagnostics; eager launches only): every launch
+// appends one line per CTA: k, cta, then the globaltimer stamps relative to
+// the CTA's start: leaf q start (1..8), leaf q end (9..16), acc_q MMA start
+// (17..24), TS term start (25..32), commit (33..40), CTA end (41).
+static uint64_t* trsm_stamps_buffer(cudaStream_t s, size_t n) {
+  static const char* path = getenv("MM_TRSM_STAMPS");
+  if (!path) return nullptr;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(s, &cs);
+  if (cs != cudaStreamCaptureStatusNone) return nullptr;
+  static uint64_t* buf = nullptr;
+  static size_t cap = 0;
+  if (n > cap) {
+    if (buf) cudaFree(buf);
+    if (cudaMalloc(&buf, n * 8) != cudaSuccess) return nullptr;
+    cap = n;
+  }
+  cudaMemsetAsync(buf, 0, n * 8, s);
+  return buf;
+}
+static void trsm_stamps_dump(cudaStream_t s, const uint64_t* d, int gx, int gy, int k) {
+  const size_t n = (size_t)gx * gy * kStampsPerCta;
+  std::vector<uint64_t> h(n);
+  cudaStreamSynchronize(s);
+  cudaMemcpy(h.data(), d, n * 8, cudaMemcpyDeviceToHost);
+  FILE* f = fopen(getenv("MM_TRSM_STAMPS"), "a");
+  if (!f) return;
+  for (int c = 0; c < gx * gy; ++c) {
+    const uint64_t* r = h.data() + (size_t)c * kStampsPerCta;
+    fprintf(f, "%d,%d", k, c);
+    for (int i = 1; i <= 41; ++i) fprintf(f, ",%.3f", r[i] ? (double)(int64_t)(r[i] - r[0]) * 1e-3 : -1.0);
+    fprintf(f, "\n");
+  }
+  fclose(f);
+}
 
 size_t chol_trsm_lt_bytes(int64_t b) { return (size_t)(b / kTcLeaf) * kLtBytes; }
 
@@ -491,9 +596,11 @@ cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32
     job.n = std::min<int32_t>(kCholBatch, n - q0);
     for (int32_t q = 0; q < job.n; ++q) job.ti[q] = ti[q0 + q];
     note_launch();
+    uint64_t* stamps = trsm_stamps_buffer(s, (size_t)(b / kTcRows) * job.n * kStampsPerCta);
     trsm_col<<<dim3((unsigned)(b / kTcRows), (unsigned)job.n), kTcThreads, kTcSmem, s>>>(A, lt, mLhi, mLlo, mSx, mShi,
-                                                                                       mSlo, job);
+                                                                                       mSlo, job, stamps);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (stamps) trsm_stamps_dump(s, stamps, (int)(b / kTcRows), job.n, k);
   }
   for (int32_t q = 0; q < n; ++q) scr->panel[slot0 + ti[q]] = tag;
   return cudaSuccess;
