@@ -63,8 +63,23 @@ struct GemmJob {
   int32_t slot0;           // first slot of this step's parity
   int32_t kx0, n0, ncols;  // mode 2 (mode 3: kx0 = K columns per split)
   int32_t mblk, nblk;      // output tiles per task
+  int32_t tri = 0;         // mode 1, SYRK (ti == tj): only the units on or below the diagonal
   int32_t ti[kCholBatch], tj[kCholBatch];
 };
+
+// Units per task: rows of R = 128 (single CTA) or 256 (pair) by BN columns;
+// `tri` keeps a unit row's n-blocks up to the one holding its last row.
+__host__ __device__ inline int tri_row_units(int r, int R, int bn, int nblk) {
+  const int c = ((r + 1) * R - 1) / bn + 1;
+  return c < nblk ? c : nblk;
+}
+__host__ __device__ inline int units_per_task(const GemmJob& job, bool mc, int bn) {
+  const int rows = mc ? job.mblk / 2 : job.mblk;
+  if (!job.tri) return rows * job.nblk;
+  int n = 0;
+  for (int r = 0; r < rows; ++r) n += tri_row_units(r, mc ? 256 : 128, bn, job.nblk);
+  return n;
+}
 
 
 // Operand coordinates and output of tile `tile` (task-major, n fastest).
@@ -78,10 +93,20 @@ template <int BN, bool MC>
 __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile, int rank) {
   TileGeo g;
   const int mb = MC ? job.mblk / 2 : job.mblk;
-  const int per = mb * job.nblk;
-  const int z = tile / per, rem = tile % per;
-  g.m_blk = MC ? 2 * (rem / job.nblk) + rank : rem / job.nblk;
-  g.n_blk = rem % job.nblk;
+  const int per = job.tri ? units_per_task(job, MC, BN) : mb * job.nblk;
+  const int z = tile / per;
+  int rem = tile % per, row = rem / job.nblk, col = rem % job.nblk;
+  if (job.tri) {
+    row = 0;
+    for (int c = tri_row_units(0, MC ? 256 : 128, BN, job.nblk); rem >= c;
+         c = tri_row_units(row, MC ? 256 : 128, BN, job.nblk)) {
+      rem -= c;
+      ++row;
+    }
+    col = rem;
+  }
+  g.m_blk = MC ? 2 * row + rank : row;
+  g.n_blk = col;
   g.ya = g.m_blk * BM;
   g.yb = g.n_blk * BN;
   g.kx0 = 0;
@@ -476,9 +501,8 @@ cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, cons
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
                         const GemmJob& job, int cap, cudaStream_t s, bool pdl = false) {
   const bool mc = use_mc(job, BN_);
-  const int ntiles = job.mblk * job.nblk * (job.mode >= 1 ? job.n : 1);
-  if (ntiles <= 0) return cudaSuccess;
-  const int units = mc ? ntiles / 2 : ntiles;
+  const int units = units_per_task(job, mc, BN_) * (job.mode >= 1 ? job.n : 1);
+  if (units <= 0) return cudaSuccess;
   const int slots = mc ? 74 : 148;            // CTA (pairs) resident at once
   int grid;
   if (cap > 0) grid = std::min(units, mc ? cap / 2 : cap);
@@ -573,9 +597,11 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
     job.slot0 = (k & 1) * (int32_t)T;
     job.kx0 = job.n0 = 0;
     job.ncols = (int32_t)b;
+    job.tri = 1;   // SYRK batches: every task on the diagonal (its upper triangle is never read)
     for (int32_t q = 0; q < job.n; ++q) {
       job.ti[q] = ijk[3 * (q0 + q)];
       job.tj[q] = ijk[3 * (q0 + q) + 1];
+      if (job.ti[q] != job.tj[q]) job.tri = 0;
     }
     job.mblk = (int32_t)(b / BM);
     job.nblk = (int32_t)(b / BN);
