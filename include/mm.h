@@ -147,6 +147,11 @@ typedef struct {
   int64_t iparam[4];            /* e.g. Cholesky (i, j, k) */
   mm_task_access access[4];
   int32_t n_access;
+  int32_t lane;                 /* 0: the kernel's compute lane (mm_app_set_lane),
+                                   1: compute lane 1 for this task (R31; the
+                                   Cholesky builtin puts SYRK(k+1,k), the update
+                                   of the next diagonal tile, there beside
+                                   POTRF / TRSM) */
 } mm_task_desc;
 
 typedef struct mm_app mm_app;

@@ -90,14 +90,15 @@ def cholesky_tasks(T: int, b: int) -> App:
                               ij=(i, k)))
         for i in range(k + 1, T):
             tasks.append(Task(2, k, tile(i, i), tile(i, i) + 1, [acc(READ, i, k), acc(RW, i, i)],
-                              ij=(i, i)))
+                              ij=(i, i), lane=1 if i == k + 1 else 0))   # SYRK(k+1,k): lane 1
         for j in range(k + 1, T):
             for i in range(j + 1, T):
                 tasks.append(Task(3, k, tile(i, j), tile(i, j) + 1,
                                   [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)], ij=(i, j)))
     ks = [Kernel(nm, 1, 1, 1, []) for nm in ("potrf", "trsm", "syrk", "gemm")]
     edges = [(0, 1), (1, 2), (1, 3), (2, 0), (3, 1), (3, 2), (3, 3)]
-    # POTRF and TRSM (the critical path) on compute lane 1 (R31)
+    # the critical path on compute lane 1 (R31): POTRF, TRSM, and the update of
+    # the next diagonal tile SYRK(k+1,k) (task lane 1)
     return App(buffers=[(4, T * T * bb)], kernels=ks, edges=edges, dag_tasks=tasks, lanes={0: 1, 1: 1})
 
 

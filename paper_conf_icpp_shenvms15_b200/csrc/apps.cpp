@@ -176,10 +176,14 @@ mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
   }
   const int32_t e[7][2] = {{0, 1}, {1, 2}, {1, 3}, {2, 0}, {3, 1}, {3, 2}, {3, 3}};
   for (auto& x : e) mm_app_add_edge(app, x[0], x[1]);
-  // critical path (POTRF, TRSM) on lane 1: step k+1's panel overlaps step k's
-  // trailing updates (lookahead)
+  // critical path on lane 1: POTRF, TRSM and the update of the next
+  // diagonal tile, SYRK(k+1,k), so POTRF(k+1) does not wait behind step k-1's
+  // trailing updates on lane 0 (R31).  MM_CHOL_LOOKAHEAD_LANE: 0 = SYRK(k+1,k)
+  // on lane 0 as well, 2 = also the GEMMs of column k+1 on lane 1 (32768^2:
+  // 62.2 / 61.7 / 65.0 ms for 0 / 1 / 2 — POTRF(k+1) then queues behind them)
   mm_app_set_lane(app, 0, 1);
   mm_app_set_lane(app, 1, 1);
+  static const int lookahead_lane = getenv("MM_CHOL_LOOKAHEAD_LANE") ? atoi(getenv("MM_CHOL_LOOKAHEAD_LANE")) : 1;
   auto tile = [&](int64_t i, int64_t j) { return (i * T + j) * bb; };
   auto task = [&](int32_t kern, int64_t i, int64_t j, int64_t k,
                   std::initializer_list<std::pair<int32_t, std::pair<int64_t, int64_t>>> a) {
@@ -187,6 +191,7 @@ mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
     std::memset(&t, 0, sizeof(t));
     t.kernel = kern;
     t.iparam[0] = i; t.iparam[1] = j; t.iparam[2] = k;
+    t.lane = (j == k + 1 && (kern == 2 ? lookahead_lane >= 1 : kern == 3 && lookahead_lane >= 2)) ? 1 : 0;
     for (auto& x : a) {
       const int64_t lo = tile(x.second.first, x.second.second);
       t.access[t.n_access++] = mm_task_access{A, x.first, lo, lo + bb};

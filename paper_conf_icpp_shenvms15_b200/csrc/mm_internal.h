@@ -46,7 +46,13 @@ struct Task {
   int64_t b = 0, e = 0;     // item range (range apps) / tile id (DAG)
   int64_t ip[4] = {0, 0, 0, 0};
   std::vector<TaskAcc> acc;
+  int32_t lane = 0;         // DAG tasks: 1 = compute lane 1 whatever the kernel's lane
 };
+
+// Compute lane of a task (R31): lane 1 if its kernel or the task itself asks for it.
+struct Kernel;
+struct App;
+int32_t task_lane(const App& app, const Task& t);
 
 struct App {
   std::vector<std::pair<int32_t, int64_t>> buffers;  // (elem_bytes, n_elems)

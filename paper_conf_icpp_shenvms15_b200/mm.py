@@ -70,7 +70,7 @@ class mm_task_access(C.Structure):
 
 class mm_task_desc(C.Structure):
     _fields_ = [("kernel", C.c_int32), ("iparam", C.c_int64 * 4), ("access", mm_task_access * 4),
-                ("n_access", C.c_int32)]
+                ("n_access", C.c_int32), ("lane", C.c_int32)]
 
 
 class mm_app_params(C.Structure):
@@ -312,9 +312,10 @@ def mm_app_set_lane(app: int, kernel: int, lane: int):
 
 
 def mm_app_add_task(app: int, kernel: int, iparam: Sequence[int],
-                    accesses: Sequence[Tuple[int, int, int, int]]):
+                    accesses: Sequence[Tuple[int, int, int, int]], lane: int = 0):
     t = mm_task_desc()
     t.kernel = kernel
+    t.lane = lane
     for i, v in enumerate(iparam):
         t.iparam[i] = v
     for i, (b, m, lo, hi) in enumerate(accesses):

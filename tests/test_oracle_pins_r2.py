@@ -254,19 +254,20 @@ def test_dp_dep_cpp_matches_hand_chains():
 
 # ------------------------------------------------- DP-Perf busy lanes (R31) --
 # 3 x 3 tiles, one device, per-task estimates POTRF 100, TRSM 10, SYRK 1,
-# GEMM 1 ns; POTRF/TRSM on lane 1, SYRK/GEMM on lane 0, each lane its own
-# busy time (same task order t0..t9 as above).  By hand:
+# GEMM 1 ns; POTRF/TRSM and SYRK(k+1,k) (the update of the next diagonal tile)
+# on lane 1, the other SYRK/GEMM on lane 0, each lane its own busy time (same
+# task order t0..t9 as above).  By hand:
 #   t0 POTRF(0)  lane1: 0 + 100                          = 100
 #   t1 TRSM(1,0) lane1: max(100, ready 100) + 10         = 110
 #   t2 TRSM(2,0) lane1: max(110, 100) + 10               = 120
-#   t3 SYRK(1,0) lane0: max(0, ready t1 110) + 1         = 111
-#   t4 SYRK(2,0) lane0: max(111, ready t2 120) + 1       = 121
+#   t3 SYRK(1,0) lane1: max(120, ready t1 110) + 1       = 121   (1 = 0 + 1)
+#   t4 SYRK(2,0) lane0: max(0, ready t2 120) + 1         = 121
 #   t5 GEMM(2,1) lane0: max(121, ready 120) + 1          = 122
-#   t6 POTRF(1)  lane1: max(120, ready t3 111) + 100     = 220
-#   t7 TRSM(2,1) lane1: max(220, ready t6 220, t5 122) + 10 = 230
-#   t8 SYRK(2,1) lane0: max(122, ready t7 230, t4 121) + 1  = 231
-#   t9 POTRF(2)  lane1: max(230, ready t8 231) + 100     = 331
-DP_PERF_LANES_FIN = [100, 110, 120, 111, 121, 122, 220, 230, 231, 331]
+#   t6 POTRF(1)  lane1: max(121, ready t3 121) + 100     = 221
+#   t7 TRSM(2,1) lane1: max(221, ready t6 221, t5 122) + 10 = 231
+#   t8 SYRK(2,1) lane1: max(231, ready t7 231, t4 121) + 1  = 232   (2 = 1 + 1)
+#   t9 POTRF(2)  lane1: max(232, ready t8 232) + 100     = 332
+DP_PERF_LANES_FIN = [100, 110, 120, 121, 121, 122, 221, 231, 232, 332]
 
 
 def test_dp_perf_lanes_by_hand():
