@@ -72,7 +72,9 @@ def cholesky_tasks(T: int, b: int) -> App:
     """Right-looking tiled Cholesky (BASELINE configs[4]) as an explicit task
     DAG over a tile-major matrix (tile (i,j) = elements [(i T + j) b^2, +b^2)).
     Kernels: 0 POTRF, 1 TRSM, 2 SYRK, 3 GEMM.  Creation order is the loop nest
-    k: POTRF(k); i>k: TRSM(i,k); i>k: SYRK(i,k); j>k, i>j: GEMM(i,j,k)."""
+    with the next panel's updates first (lookahead, R34): k: POTRF(k);
+    i>k: TRSM(i,k); SYRK(k+1,k); i>k+1: GEMM(i,k+1,k); i>k+1: SYRK(i,k);
+    j>k+1, i>j: GEMM(i,j,k)."""
     bb = b * b
 
     def tile(i, j):
@@ -88,13 +90,20 @@ def cholesky_tasks(T: int, b: int) -> App:
         for i in range(k + 1, T):
             tasks.append(Task(1, k, tile(i, k), tile(i, k) + 1, [acc(READ, k, k), acc(RW, i, k)],
                               ij=(i, k)))
-        for i in range(k + 1, T):
-            tasks.append(Task(2, k, tile(i, i), tile(i, i) + 1, [acc(READ, i, k), acc(RW, i, i)],
-                              ij=(i, i), lane=1 if i == k + 1 else 0))   # SYRK(k+1,k): lane 1
-        for j in range(k + 1, T):
-            for i in range(j + 1, T):
-                tasks.append(Task(3, k, tile(i, j), tile(i, j) + 1,
-                                  [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)], ij=(i, j)))
+        def syrk(i):
+            return Task(2, k, tile(i, i), tile(i, i) + 1, [acc(READ, i, k), acc(RW, i, i)],
+                        ij=(i, i), lane=1 if i == k + 1 else 0)   # SYRK(k+1,k): lane 1
+
+        def gemm(i, j):
+            return Task(3, k, tile(i, j), tile(i, j) + 1,
+                        [acc(READ, i, k), acc(READ, j, k), acc(RW, i, j)], ij=(i, j))
+
+        if k + 1 < T:   # lookahead: the updates of column k+1
+            tasks.append(syrk(k + 1))
+            tasks.extend(gemm(i, k + 1) for i in range(k + 2, T))
+        tasks.extend(syrk(i) for i in range(k + 2, T))
+        for j in range(k + 2, T):
+            tasks.extend(gemm(i, j) for i in range(j + 1, T))
     ks = [Kernel(nm, 1, 1, 1, []) for nm in ("potrf", "trsm", "syrk", "gemm")]
     edges = [(0, 1), (1, 2), (1, 3), (2, 0), (3, 1), (3, 2), (3, 3)]
     # the critical path on compute lane 1 (R31): POTRF, TRSM, and the update of

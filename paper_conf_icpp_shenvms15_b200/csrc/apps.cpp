@@ -203,11 +203,21 @@ mm_status cholesky_app(const mm_app_params& p, mm_app* app) {
     if (st) return st;
     for (int64_t i = k + 1; i < T; ++i)
       if ((st = task(1, i, k, k, {{MM_READ, {k, k}}, {MM_RW, {i, k}}}))) return st;
-    for (int64_t i = k + 1; i < T; ++i)
-      if ((st = task(2, i, i, k, {{MM_READ, {i, k}}, {MM_RW, {i, i}}}))) return st;
-    for (int64_t j = k + 1; j < T; ++j)
+    // the updates of column k+1 first (lookahead, R34), then the rest
+    auto syrk = [&](int64_t i) { return task(2, i, i, k, {{MM_READ, {i, k}}, {MM_RW, {i, i}}}); };
+    auto gemm = [&](int64_t i, int64_t j) {
+      return task(3, i, j, k, {{MM_READ, {i, k}}, {MM_READ, {j, k}}, {MM_RW, {i, j}}});
+    };
+    if (k + 1 < T) {
+      if ((st = syrk(k + 1))) return st;
+      for (int64_t i = k + 2; i < T; ++i)
+        if ((st = gemm(i, k + 1))) return st;
+    }
+    for (int64_t i = k + 2; i < T; ++i)
+      if ((st = syrk(i))) return st;
+    for (int64_t j = k + 2; j < T; ++j)
       for (int64_t i = j + 1; i < T; ++i)
-        if ((st = task(3, i, j, k, {{MM_READ, {i, k}}, {MM_READ, {j, k}}, {MM_RW, {i, j}}}))) return st;
+        if ((st = gemm(i, j))) return st;
   }
   return MM_OK;
 }

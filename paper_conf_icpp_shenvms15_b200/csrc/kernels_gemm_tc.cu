@@ -63,19 +63,22 @@ struct GemmJob {
   int32_t slot0;           // first slot of this step's parity
   int32_t kx0, n0, ncols;  // mode 2 (mode 3: kx0 = K columns per split)
   int32_t mblk, nblk;      // output tiles per task
-  int32_t tri = 0;         // mode 1, SYRK (ti == tj): only the units on or below the diagonal
+  int32_t tri = 0;         // mode 1: tasks on the diagonal (SYRK, ti == tj) keep only the
+                           // units on or below it (the upper triangle is never read);
+                           // task z's units start at uoff[z]
   int32_t ti[kCholBatch], tj[kCholBatch];
+  int32_t uoff[kCholBatch + 1];
 };
 
 // Units per task: rows of R = 128 (single CTA) or 256 (pair) by BN columns;
-// `tri` keeps a unit row's n-blocks up to the one holding its last row.
+// a triangular task keeps a unit row's n-blocks up to the one holding its last row.
 __host__ __device__ inline int tri_row_units(int r, int R, int bn, int nblk) {
   const int c = ((r + 1) * R - 1) / bn + 1;
   return c < nblk ? c : nblk;
 }
-__host__ __device__ inline int units_per_task(const GemmJob& job, bool mc, int bn) {
+__host__ __device__ inline int units_per_task(const GemmJob& job, bool mc, int bn, bool tri = false) {
   const int rows = mc ? job.mblk / 2 : job.mblk;
-  if (!job.tri) return rows * job.nblk;
+  if (!tri) return rows * job.nblk;
   int n = 0;
   for (int r = 0; r < rows; ++r) n += tri_row_units(r, mc ? 256 : 128, bn, job.nblk);
   return n;
@@ -93,10 +96,23 @@ template <int BN, bool MC>
 __device__ __forceinline__ TileGeo tile_geo(const GemmJob& job, float* C, int tile, int rank) {
   TileGeo g;
   const int mb = MC ? job.mblk / 2 : job.mblk;
-  const int per = job.tri ? units_per_task(job, MC, BN) : mb * job.nblk;
-  const int z = tile / per;
-  int rem = tile % per, row = rem / job.nblk, col = rem % job.nblk;
-  if (job.tri) {
+  int z, rem;
+  if (job.tri) {   // task of unit `tile`: the last z with uoff[z] <= tile
+    int lo = 0, hi = job.n;
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (job.uoff[mid] <= tile) lo = mid;
+      else hi = mid;
+    }
+    z = lo;
+    rem = tile - job.uoff[z];
+  } else {
+    const int per = mb * job.nblk;
+    z = tile / per;
+    rem = tile % per;
+  }
+  int row = rem / job.nblk, col = rem % job.nblk;
+  if (job.tri && job.ti[z] == job.tj[z]) {
     row = 0;
     for (int c = tri_row_units(0, MC ? 256 : 128, BN, job.nblk); rem >= c;
          c = tri_row_units(row, MC ? 256 : 128, BN, job.nblk)) {
@@ -501,7 +517,7 @@ cudaError_t launch_gemm(const CUtensorMap& ta_hi, const CUtensorMap& ta_lo, cons
                         const CUtensorMap& tb_lo, float* C, int64_t N, int64_t row0, int64_t mrows, int nkb,
                         const GemmJob& job, int cap, cudaStream_t s, bool pdl = false) {
   const bool mc = use_mc(job, BN_);
-  const int units = units_per_task(job, mc, BN_) * (job.mode >= 1 ? job.n : 1);
+  const int units = job.tri ? job.uoff[job.n] : units_per_task(job, mc, BN_) * (job.mode >= 1 ? job.n : 1);
   if (units <= 0) return cudaSuccess;
   const int slots = mc ? 74 : 148;            // CTA (pairs) resident at once
   int grid;
@@ -597,14 +613,16 @@ cudaError_t chol_update_tc(float* A, int64_t T, int64_t b, const int32_t* ijk, i
     job.slot0 = (k & 1) * (int32_t)T;
     job.kx0 = job.n0 = 0;
     job.ncols = (int32_t)b;
-    job.tri = 1;   // SYRK batches: every task on the diagonal (its upper triangle is never read)
+    job.tri = 1;   // SYRK tasks (ti == tj): lower units only; SYRK and GEMM may share a batch
+    job.mblk = (int32_t)(b / BM);
+    job.nblk = (int32_t)(b / BN);
+    const bool mc = use_mc(job);
+    job.uoff[0] = 0;
     for (int32_t q = 0; q < job.n; ++q) {
       job.ti[q] = ijk[3 * (q0 + q)];
       job.tj[q] = ijk[3 * (q0 + q) + 1];
-      if (job.ti[q] != job.tj[q]) job.tri = 0;
+      job.uoff[q + 1] = job.uoff[q] + units_per_task(job, mc, BN, job.ti[q] == job.tj[q]);
     }
-    job.mblk = (int32_t)(b / BM);
-    job.nblk = (int32_t)(b / BN);
     launch_gemm<BN>(ta_hi, ta_lo, tb_hi, tb_lo, A, b, 0, b, (int)(b / BK), job, 0, s);
   }
   return cudaGetLastError();

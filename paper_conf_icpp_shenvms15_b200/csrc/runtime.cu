@@ -239,6 +239,7 @@ struct PlanRt {
 bool is_batchable_op(int32_t op) {
   return op == MM_OP_CHOL_TRSM || op == MM_OP_CHOL_SYRK || op == MM_OP_CHOL_GEMM;
 }
+bool is_chol_update(int32_t op) { return op == MM_OP_CHOL_SYRK || op == MM_OP_CHOL_GEMM; }
 
 // Group consecutive independent kernel ops of one device and one kernel into
 // one launch (MK-DAG steps: all TRSMs / SYRKs / GEMMs of a step on a device).
@@ -248,10 +249,12 @@ bool is_batchable_op(int32_t op) {
 // Batch key: tasks of one batch must share it.  Cholesky lookahead: the GEMM
 // updates of column k+1 and SYRK(k+1, k) run as their own launches, so step
 // k+1's POTRF / TRSM (lane 1) wait only for the updates they read; the rest
-// of step k's GEMMs is one launch (no per-column waves of partial occupancy).
+// of step k's SYRKs and GEMMs is one launch (no per-column waves of partial
+// occupancy; the task order puts them next to each other, R34).
 int64_t batch_key(const Kernel& k, const Task& t) {
-  if (k.op == MM_OP_CHOL_GEMM) return t.ip[2] * 2 + (t.ip[1] == t.ip[2] + 1 ? 1 : 0);
-  if (k.op == MM_OP_CHOL_SYRK) return t.ip[2] * 2 + (t.ip[0] == t.ip[2] + 1 ? 1 : 0);
+  static const int merge = getenv("MM_CHOL_MERGE_SYRK") ? atoi(getenv("MM_CHOL_MERGE_SYRK")) : 1;
+  if (k.op == MM_OP_CHOL_GEMM) return t.ip[2] * 4 + (t.ip[1] == t.ip[2] + 1 ? 1 : 0);
+  if (k.op == MM_OP_CHOL_SYRK) return t.ip[2] * 4 + (t.ip[0] == t.ip[2] + 1 ? 1 : (merge ? 0 : 2));
   return t.ip[2];
 }
 
@@ -278,8 +281,10 @@ void compute_batches(const Plan& plan, PlanRt* rt) {
     const Task& t = plan.tasks[op.task];
     const Kernel& kern = plan.app.kernels[op.kernel];
     int64_t h = open[sid];
-    bool ok = h >= 0 && plan.ops[h].kernel == op.kernel && (int64_t)rt->members[h].size() + 1 < kCholBatch &&
-              batch_key(kern, plan.tasks[plan.ops[h].task]) == batch_key(kern, t);
+    const Kernel& hk = plan.app.kernels[h >= 0 ? plan.ops[h].kernel : op.kernel];
+    const bool same = h >= 0 && (plan.ops[h].kernel == op.kernel || (is_chol_update(hk.op) && is_chol_update(kern.op)));
+    bool ok = same && (int64_t)rt->members[h].size() + 1 < kCholBatch &&
+              batch_key(hk, plan.tasks[plan.ops[h].task]) == batch_key(kern, t);
     if (ok)
       for (auto& w : plan.waits[i])
         if (w.op >= h) ok = false;

@@ -212,15 +212,17 @@ def test_pipelined_staged_program_moves_each_element_once(P, passes):
 
 # ------------------------------------------------------------ DP-Dep (R30) --
 # Hand-traced chains of the 3 x 3-tile Cholesky DAG.  Creation order (P119
-# breadth-first; loop nest k, then TRSM i, SYRK i, GEMM j<i):
-#   t0 POTRF(0)  t1 TRSM(1,0)  t2 TRSM(2,0)  t3 SYRK(1,0)  t4 SYRK(2,0)
-#   t5 GEMM(2,1,0)  t6 POTRF(1)  t7 TRSM(2,1)  t8 SYRK(2,1)  t9 POTRF(2)
-# t0 new chain; t1 continues t0 (RAW on tile 00); t2: t0 closed -> new chain;
-# t3 continues t1 (RAW 10); t4 continues t2 (RAW 20); t5: t1, t2 closed ->
-# new chain; t6 continues t3 (WAW 11); t7 continues t5 (WAW 21); t8 continues
-# t4 (WAW 22); t9 continues t8 (WAW 22).
-DP_DEP_CHOL3 = {2: [0, 0, 1, 0, 1, 0, 0, 0, 1, 1],
-                3: [0, 0, 1, 0, 1, 2, 0, 2, 1, 1]}
+# breadth-first; loop nest k, TRSM i, then the lookahead updates of column
+# k+1, then the rest, R34):
+#   t0 POTRF(0)  t1 TRSM(1,0)  t2 TRSM(2,0)  t3 SYRK(1,0)  t4 GEMM(2,1,0)
+#   t5 SYRK(2,0)  t6 POTRF(1)  t7 TRSM(2,1)  t8 SYRK(2,1)  t9 POTRF(2)
+# t0 new chain (device 0); t1 continues t0 (RAW on tile 00, t0 closed); t2:
+# no open predecessor -> new chain (device 1); t3 continues t1 (RAW 10, t1
+# closed); t4 continues t2 (RAW 20; t1 is closed; t2 closed); t5: t2 closed
+# -> new chain (device 0 of 2 / 2 of 3); t6 continues t3 (WAW 11); t7
+# continues t4 (WAW 21); t8 continues t5 (WAW 22); t9 continues t8 (WAW 22).
+DP_DEP_CHOL3 = {2: [0, 0, 1, 0, 1, 0, 0, 1, 0, 0],
+                3: [0, 0, 1, 0, 1, 2, 0, 1, 2, 2]}
 
 
 @pytest.mark.parametrize("G", [2, 3])
@@ -261,11 +263,11 @@ def test_dp_dep_cpp_matches_hand_chains():
 #   t1 TRSM(1,0) lane1: max(100, ready 100) + 10         = 110
 #   t2 TRSM(2,0) lane1: max(110, 100) + 10               = 120
 #   t3 SYRK(1,0) lane1: max(120, ready t1 110) + 1       = 121   (1 = 0 + 1)
-#   t4 SYRK(2,0) lane0: max(0, ready t2 120) + 1         = 121
-#   t5 GEMM(2,1) lane0: max(121, ready 120) + 1          = 122
+#   t4 GEMM(2,1) lane0: max(0, ready t2 120, t1 110) + 1 = 121
+#   t5 SYRK(2,0) lane0: max(121, ready t2 120) + 1       = 122
 #   t6 POTRF(1)  lane1: max(121, ready t3 121) + 100     = 221
-#   t7 TRSM(2,1) lane1: max(221, ready t6 221, t5 122) + 10 = 231
-#   t8 SYRK(2,1) lane1: max(231, ready t7 231, t4 121) + 1  = 232   (2 = 1 + 1)
+#   t7 TRSM(2,1) lane1: max(221, ready t6 221, t4 121) + 10 = 231
+#   t8 SYRK(2,1) lane1: max(231, ready t7 231, t5 122) + 1  = 232   (2 = 1 + 1)
 #   t9 POTRF(2)  lane1: max(232, ready t8 232) + 100     = 332
 DP_PERF_LANES_FIN = [100, 110, 120, 121, 121, 122, 221, 231, 232, 332]
 

@@ -1,6 +1,6 @@
 cd /root/repo
 for r in 1 2; do
-for la in 2 0 1; do
-MM_CHOL_LOOKAHEAD_LANE=$la timeout 300 python bench.py --app cholesky --steps 3 --warmup 2 --kernel-timing none --no-cpu-baseline --no-e2e --no-strategies > gpurun_out/ab.log 2>&1
-echo "la=$la $(grep -o '"ms_per_step": [0-9.]*' gpurun_out/ab.log | head -1) $(grep -o '"sm_mhz": [0-9.]*' gpurun_out/ab.log)" >> gpurun_out/ab.txt
+for cfg in "MM_CHOL_MERGE_SYRK=1" "MM_CHOL_MERGE_SYRK=0"; do
+env $cfg timeout 300 python bench.py --app cholesky --steps 3 --warmup 2 --kernel-timing none --no-cpu-baseline --no-e2e --no-strategies > gpurun_out/ab.log 2>&1
+echo "$cfg $(grep -o '"ms_per_step": [0-9.]*' gpurun_out/ab.log | head -1) $(grep -o '"sm_mhz": [0-9.]*' gpurun_out/ab.log)" >> gpurun_out/ab.txt
 done; done
