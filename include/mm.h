@@ -430,7 +430,11 @@ typedef struct {
                                 stream (mm_ctx_stream), so later runs and a caller stream set by
                                 mm_ctx_set_stream are ordered after it; device_ms = -1; host
                                 buffers must not be touched before that stream completes */
-  int32_t _pad;
+  int32_t repeat;            /* run the op program this many times back to back (0/1 = once;
+                                with use_graph ONE graph holds all of them, so the runs pay
+                                one launch); stats count every run, kernel_ms (time_kernels,
+                                which use_graph then captures as event nodes) is the last
+                                run's */
 } mm_run_opts;
 
 /* One adaptive DP-Perf decision: the snapshot it was taken on.  All times in

@@ -610,6 +610,16 @@ void* flush_target(mm_ctx* ctx, const Plan& plan, const mm_run_opts* o, int32_t 
 }
 
 // Issue the op program of an in-process ctx (world == 1) onto the streams.
+// Kernel-timing events: inside a stream capture a plain cudaEventRecord only
+// orders streams; the external flag makes it an event record node of the
+// graph, so graph replays carry the timing too.
+cudaError_t rec_kev(cudaEvent_t ev, cudaStream_t s) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaStreamIsCapturing(s, &cs);
+  return cudaEventRecordWithFlags(ev, s, cs == cudaStreamCaptureStatusActive ? cudaEventRecordExternal
+                                                                             : cudaEventRecordDefault);
+}
+
 mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run_opts* o, bool timing,
                       mm_run_stats* st) {
   PlanRt* rt = static_cast<PlanRt*>(plan.rt);
@@ -654,17 +664,17 @@ mm_status issue_local(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_ru
     if (op.kind == MM_OPK_KERNEL && !rt->members[i].empty()) {
       for (int64_t m : rt->members[i])
         for (auto& w : plan.waits[m]) CU_OK(cudaStreamWaitEvent(s, rt->ev[w.op], 0));
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i], s));
       mm_status r = launch_batch(ctx, plan, rt, (int64_t)i, d, buffers, s);
       if (r) return r;
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i + 1], s));
       for (int64_t m : rt->members[i])
         if (plan.needs_event[m]) CU_OK(cudaEventRecord(rt->ev[m], s));
     } else if (op.kind == MM_OPK_KERNEL) {
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i], s));
       mm_status r = launch_task(ctx, app, plan.tasks[op.task], d, buffers, s);
       if (r) return r;
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i + 1], s));
     } else if (op.kind == MM_OPK_XFER) {
       const int64_t eb = app.buffers[op.buffer].first;
       const size_t bytes = (size_t)((op.r.end - op.r.begin) * eb);
@@ -731,11 +741,11 @@ mm_status issue_dist(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run
     }
     if (op.kind == MM_OPK_KERNEL) {
       if (op.device != me || rt->batch_head[i] >= 0) continue;
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i], s));
       mm_status r = rt->members[i].empty() ? launch_task(ctx, app, plan.tasks[op.task], me, buffers, s)
                                             : launch_batch(ctx, plan, rt, (int64_t)i, me, buffers, s);
       if (r) return r;
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i + 1], s));
       continue;
     }
     const int64_t eb = app.buffers[op.buffer].first;
@@ -876,11 +886,11 @@ mm_status issue_ipc(mm_ctx* ctx, Plan& plan, void* const* buffers, const mm_run_
         if (mm_status r = add_waits((size_t)m)) return r;
     if (mm_status r = flush_waits(s)) return r;
     if (op.kind == MM_OPK_KERNEL) {
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i], s));
       mm_status r = rt->members[i].empty() ? launch_task(ctx, app, plan.tasks[op.task], d, buffers, s)
                                            : launch_batch(ctx, plan, rt, (int64_t)i, d, buffers, s);
       if (r) return r;
-      if (timing) CU_OK(cudaEventRecord(rt->kev[2 * i + 1], s));
+      if (timing) CU_OK(rec_kev(rt->kev[2 * i + 1], s));
       for (int64_t m : rt->members[i]) {
         if (plan.needs_event[m]) CU_OK(cudaEventRecord(rt->ev[m], s));
         if (rt->remote_sig[m]) CU_OK(ipc_signal(ch->flags, kIpcOp0 + m, s));
@@ -1553,7 +1563,9 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
   mm_run_stats* S = st ? st : &local;
   *S = mm_run_stats{};
   const bool timing = o && o->time_kernels;
-  const bool graph = o && o->use_graph && !timing && (ctx->world == 1 || ctx->ipc);
+  const bool graph = o && o->use_graph && (ctx->world == 1 || ctx->ipc);
+  const int32_t reps = (o && o->repeat > 1) ? o->repeat : 1;
+  if (o && o->repeat < 0) MM_FAIL(MM_EINVAL, "run: repeat %d < 0", o->repeat);
   mm_status r = ensure_rt(ctx, plan, timing);
   if (r) return r;
   if ((r = join_external(ctx, true))) return r;
@@ -1612,6 +1624,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       key.push_back(o && o->host ? o->host[b] : nullptr);
     for (void* p : ctx->flush_scratch) key.push_back(p);
     for (char* p : ctx->ipc_bufs) key.push_back(p);
+    key.push_back(reinterpret_cast<void*>((intptr_t)reps));
+    key.push_back(reinterpret_cast<void*>((intptr_t)(timing ? 1 : 0)));
     if (!rt->gexec || key != rt->graph_bufs) {
       if (rt->gexec) cudaGraphExecDestroy(rt->gexec);
       if (rt->graph) cudaGraphDestroy(rt->graph);
@@ -1621,7 +1635,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
       CU_OK(cudaStreamBeginCapture(rs, cudaStreamCaptureModeThreadLocal));
       mm_run_stats cap{};
       const int64_t l0 = g_kernel_launches.load();
-      r = ctx->ipc ? issue_ipc(ctx, plan, buffers, o, false, &cap) : issue_local(ctx, plan, buffers, o, false, &cap);
+      for (int32_t rep = 0; rep < reps && !r; ++rep)   // kernel timing: event record nodes
+        r = ctx->ipc ? issue_ipc(ctx, plan, buffers, o, timing, &cap) : issue_local(ctx, plan, buffers, o, timing, &cap);
       const int64_t captured = g_kernel_launches.load() - l0;
       g_kernel_launches.fetch_sub(captured, std::memory_order_relaxed);   // counted per replay
       cudaGraph_t g = nullptr;
@@ -1653,9 +1668,11 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     CU_OK(set_dev(ctx, root));
     CU_OK(cudaEventRecord(rt->t_start, rs));
     const int64_t l0 = g_kernel_launches.load();
-    if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
-    else if (ctx->ipc) r = issue_ipc(ctx, plan, buffers, o, timing, S);
-    else r = issue_dist(ctx, plan, buffers, o, timing, S);
+    for (int32_t rep = 0; rep < reps && !r; ++rep) {
+      if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
+      else if (ctx->ipc) r = issue_ipc(ctx, plan, buffers, o, timing, S);
+      else r = issue_dist(ctx, plan, buffers, o, timing, S);
+    }
     S->n_launches = g_kernel_launches.load() - l0;
     if (r) return r;
     CU_OK(set_dev(ctx, root));
@@ -1670,7 +1687,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     S->device_ms = -1.0;
     for (size_t i = 0; i < plan.ops.size(); ++i)
       if (plan.ops[i].kind == MM_OPK_KERNEL && ctx->dev[plan.ops[i].device].mine)
-        S->kernel_launches[plan.ops[i].device][plan.ops[i].kernel]++;
+        S->kernel_launches[plan.ops[i].device][plan.ops[i].kernel] += reps;
     return MM_OK;
   }
   CU_OK(cudaEventSynchronize(rt->t_stop));
@@ -1697,8 +1714,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
                 a, z);
       }
     }
-    S->kernel_launches[op.device][op.kernel]++;
-    if (timing && rt->kev[2 * i] && rt->batch_head[i] < 0) {   // batch members: timed with their head
+    S->kernel_launches[op.device][op.kernel] += reps;
+    if (timing && rt->kev[2 * i] && rt->batch_head[i] < 0) {   // batch members: timed with their head (last run)
       float k = 0.f;
       CU_OK(cudaEventElapsedTime(&k, rt->kev[2 * i], rt->kev[2 * i + 1]));
       S->kernel_ms[op.device][op.kernel] += k;

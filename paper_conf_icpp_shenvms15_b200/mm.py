@@ -122,7 +122,7 @@ class mm_profile_opts(C.Structure):
 class mm_run_opts(C.Structure):
     _fields_ = [("use_graph", C.c_int32), ("time_kernels", C.c_int32), ("adaptive", C.c_int32),
                 ("max_inflight", C.c_int32), ("host", C.POINTER(C.c_void_p)), ("no_wait", C.c_int32),
-                ("_pad", C.c_int32)]
+                ("repeat", C.c_int32)]
 
 
 class mm_decision(C.Structure):
@@ -560,8 +560,9 @@ def mm_profile_run(ctx: int, app: int, buffers: Sequence[int], reps: int = 5, dp
 
 def mm_run(ctx: int, plan: int, buffers: Optional[Sequence[int]], use_graph: bool = False, time_kernels: bool = False,
            host: Optional[Sequence[int]] = None, adaptive: bool = False, max_inflight: int = 0,
-           no_wait: bool = False) -> mm_run_stats:
+           no_wait: bool = False, repeat: int = 1) -> mm_run_stats:
     o = mm_run_opts()
+    o.repeat = int(repeat)
     o.use_graph = int(use_graph)
     o.no_wait = int(no_wait)
     o.time_kernels = int(time_kernels)

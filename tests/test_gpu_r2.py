@@ -321,3 +321,32 @@ def test_stencil_reduction_halo_split(R):
     assert np.array_equal(got, T)
     import math
     assert abs(math.fsum(rowsum) - rs[-1]) <= 1e-12 * abs(rs[-1])
+
+
+# ------------------------------------------------- repeated runs (mm_run repeat) --
+@pytest.mark.parametrize("graph", [False, True])
+@pytest.mark.parametrize("timing", [False, True])
+def test_run_repeat_equals_sequential_runs(R, graph, timing):
+    """mm_run_opts.repeat = 3 runs the op program three times back to back (in
+    one CUDA graph with use_graph; kernel-timing events become event nodes of
+    that graph): STREAM's arrays evolve as after 3 passes, bit for bit; the
+    stats count every run; kernel_ms is the last run's (> 0 when timed)."""
+    mm, runner = R
+    n = 100003
+    a0, b0, c0 = synthgen.stream_random(n)
+    ref = on.stream_run(a0, b0, c0, 3)
+    with runner.session(mm.MM_APP_STREAM, [n, 1, 1, 32, 1], G=2) as s:
+        s.fill()
+        prof = mm.make_profile(2, [[1000, 1300, 900, 1100]] * 2, [[10 ** 5] * 4] * 2, [10 ** 11] * 2)
+        plan = s.plan(mm.MM_SP_UNIFIED, prof)
+        one = s.run(plan)
+        s.fill()
+        st = s.run(plan, use_graph=graph, time_kernels=timing, repeat=3)
+        for slot in range(3):
+            assert np.array_equal(s.collect(plan, slot), ref[slot]), slot
+        assert st.n_launches == 3 * one.n_launches
+        launches = sum(st.kernel_launches[d][k] for d in range(2) for k in range(4))
+        assert launches == 3 * sum(one.kernel_launches[d][k] for d in range(2) for k in range(4))
+        ms = sum(st.kernel_ms[d][k] for d in range(2) for k in range(4))
+        assert (ms > 0) == timing
+        assert st.device_ms > 0
