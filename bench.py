@@ -271,6 +271,10 @@ def main():
     ap.add_argument("--halo-split", default="auto", choices=["auto", "on", "off"],
                     help="R33: SP ranges of halo-reading kernels run interior-first so the interior overlaps "
                          "the halo pulls (auto = on when the job spans more than one device)")
+    ap.add_argument("--one-graph", action="store_true",
+                    help="time the K steps as ONE mm_run with repeat = K (one graph of K copies of the op "
+                         "program); measured no faster than K replays, and slower with kernel timing, whose "
+                         "event nodes then sit in every copy")
     ap.add_argument("--no-graph", action="store_true",
                     help="timed steps issue the op program eagerly instead of replaying a CUDA graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -383,10 +387,16 @@ def main():
     # every kernel for the roofline (--kernel-timing)
     graph_ok = world == 1 or os.environ.get("MM_TRANSPORT") != "nccl"
     fast = dict(use_graph=graph_ok and not args.no_graph, no_wait=True)
+    # apps that do not restore their input between steps run all K timed steps
+    # as ONE mm_run with repeat = K (see the timed loop); its graph is captured
+    # in the last warm-up step, outside the timed region
+    one_graph = not pristine and fast["use_graph"] and args.one_graph and args.kernel_timing != "all"
     for w in range(args.warmup):
         restore()
         if w == 0:
             step(plan, time_kernels=True)
+        elif one_graph and w == args.warmup - 1:
+            step(plan, use_graph=True, time_kernels=args.kernel_timing != "none", repeat=args.steps)
         else:
             step(plan, **fast)
     barrier()
@@ -400,8 +410,29 @@ def main():
     # enqueued back to back), so timing more steps would add host round trips
     # to the measured region
     n_last = 1
+    # one_graph: one CUDA graph holding K copies of the op program
+    # (kernel-timing events are event nodes of that graph, read for the last
+    # copy), so the steps pay one launch instead of K
     with ClockSampler(local) as clk:
-        for i in range(args.steps):
+        if one_graph:
+            barrier()
+            ev0 = torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            for _ in range(args.steps - 1):   # the host control plane of every step
+                c = mm.mm_classify(sess.app)
+                mm.mm_rank(c, mm.mm_needs_sync(sess.app))
+                if best in (mm.MM_SP_SINGLE, mm.MM_SP_UNIFIED, mm.MM_SP_VARIED):
+                    mm.mm_split(sess.app, prof, best)
+            st = step(plan, use_graph=True, time_kernels=args.kernel_timing != "none", repeat=args.steps)
+            for d in range(G):
+                for k in range(K):
+                    kms[d][k] += st.kernel_ms[d][k]
+            launches += st.n_launches
+            ev1 = torch.cuda.Event(enable_timing=True)
+            ev1.record(stream)
+            barrier()
+            spans.append((ev0, ev1))
+        for i in range(0 if not one_graph else args.steps, args.steps):
             if pristine or i == 0:
                 restore()
                 barrier()
@@ -629,9 +660,12 @@ def main():
                        "strategy": mm.mm_strategy_name(best), "logical_devices": G,
                        "l2": "inputs larger than L2 (1 GiB arrays); no flush",
                        "kernel_timing": {"all": "per-kernel CUDA events in every timed step",
-                                         "last": f"per-kernel CUDA events in the last {n_last} of {args.steps} timed steps",
+                                         "last": f"per-kernel CUDA events in the last {n_last} of {args.steps} timed steps"
+                                                 + (" (graph event nodes)" if one_graph else ""),
                                          "none": "no per-kernel events"}[args.kernel_timing],
-                       "issue": ("other timed steps: the op program replayed as a CUDA graph, enqueued back to back"
+                       "issue": ("all timed steps in ONE CUDA graph (mm_run repeat = K: K copies of the op program, "
+                                 "kernel-timing events as graph nodes, read for the last copy)" if one_graph else
+                                 "other timed steps: the op program replayed as a CUDA graph, enqueued back to back"
                                  if fast["use_graph"] else "other timed steps: eager issue, enqueued back to back"),
                        "split": mm.mm_plan_ranges(plan)[:G], "parallelism": f"row/element split over {G}",
                        "halo_split": halo_split,

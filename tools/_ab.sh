@@ -1,6 +1,9 @@
 cd /root/repo
-for r in 1 2; do
-for cfg in "MM_CHOL_MERGE_SYRK=1" "MM_CHOL_MERGE_SYRK=0"; do
-env $cfg timeout 300 python bench.py --app cholesky --steps 3 --warmup 2 --kernel-timing none --no-cpu-baseline --no-e2e --no-strategies > gpurun_out/ab.log 2>&1
-echo "$cfg $(grep -o '"ms_per_step": [0-9.]*' gpurun_out/ab.log | head -1) $(grep -o '"sm_mhz": [0-9.]*' gpurun_out/ab.log)" >> gpurun_out/ab.txt
+for app in matmul1k stream; do
+for f in "--kernel-timing none" "--kernel-timing none --no-repeat" "--kernel-timing last" "--kernel-timing last --no-repeat"; do
+timeout 600 python bench.py --app $app --steps 20 --warmup 5 --no-strategies --no-cpu-baseline --no-e2e $f > gpurun_out/ab.log 2>&1
+python3 -c "
+import json
+d=[json.loads(l) for l in open('gpurun_out/ab.log') if l.startswith('{')][-1]
+print('$app', '$f', round(d['ms_per_step'],4), round(d['value'],2), d['unit'], d['gpu_launches'], d['clocks']['sm_mhz'])" >> gpurun_out/ab.txt
 done; done
