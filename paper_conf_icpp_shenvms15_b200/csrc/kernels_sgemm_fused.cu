@@ -27,8 +27,15 @@
 //              barrier before exit.
 // 1024^2 (S = 2, 128 CTAs in clusters of 4): 23.5 us (ncu, cold) against 33 us
 // for the split -> GEMM -> reduce chain.  globaltimer stamps: set-up 0.8 us,
-// first MMA at 1.9 us, ~490 ns per k-step (MMA-issue-bound: the converters
-// run up to 3 steps ahead), reduction ~4 us (DSMEM moves ~20 B/clk per SM).
+// first MMA at 1.9 us, ~490 ns per k-step (the converters of both CTAs run
+// 2-3 steps ahead), reduction ~4 us (DSMEM moves ~20 B/clk per SM).  The 6
+// MMAs of a k-step need 384 clk at the measured full rate (tools/mma_rates.cu:
+// 64 clk per 256 x 128 x 8 pair MMA, TS or SS, also with streamed operand
+// stages); the rest of the ~940 clk per k-step is per-step overhead that
+// neither an 8-stage split ring, 4 converter groups, two stages per
+// wait/commit round nor issuing without waiting for split_full removed
+// (all measured unchanged; doubling the MMAs of a step added exactly their
+// 64 clk each).
 // Tried and dropped: 256-wide pairs with S = 3 (24.9 us, both operands in
 // smem: 26 us), a cp.async.bulk push of the partial slices and a reduction
 // through L2 (both slower than the DSMEM pull).
