@@ -40,7 +40,7 @@ class Session:
     def __init__(self, app: int, G: int = 1, cuda_devices: Optional[Sequence[int]] = None,
                  sm_budgets: Optional[Sequence[int]] = None, rank: int = 0, world: int = 1,
                  nccl_id: Optional[bytes] = None, owned: Optional[Sequence[int]] = None,
-                 app_id: int = 0):
+                 app_id: int = 0, register: bool = True):
         self.app = app
         self.app_id = app_id
         self.G = G
@@ -67,10 +67,12 @@ class Session:
                                                     device=f"cuda:{cuda_devices[d]}")
         # register the buffers once (mm_buffer_register): runs then pass no
         # pointer array (mm_run with buffers == NULL)
+        # (register=False: the caller registers, or passes pointers per run)
         ptrs = self.ptrs()
-        for slot in range(self.nbuf):
+        for slot in range(self.nbuf if register else 0):
             eb, n = mm.mm_app_buffer_info(app, slot)
             mm.mm_buffer_register(self.ctx, eb, n, ptrs[slot * G:(slot + 1) * G])
+        self.registered = register
         self.plans: List[int] = []
         self.tile = 0   # Cholesky tile size (set by session())
 
@@ -151,7 +153,7 @@ class Session:
         return p
 
     def run(self, plan: int, **kw) -> mm.mm_run_stats:
-        return mm.mm_run(self.ctx, plan, None, **kw)   # the registered buffers
+        return mm.mm_run(self.ctx, plan, None if self.registered else self.ptrs(), **kw)
 
     def tune_chunks(self, strategy: int, prof: mm.mm_profile, candidates=(1, 2, 4, 8, 16, 32), reps: int = 3,
                     **opts):

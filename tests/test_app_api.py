@@ -53,7 +53,7 @@ def test_registered_buffers(R, strategy):
     n = 100003
     a0, b0, c0 = synthgen.stream_random(n)
     ref = on.stream_run(a0, b0, c0, 1)
-    with runner.session(mm.MM_APP_STREAM, [n, 1, 0, 32, 1], G=2) as s:
+    with runner.session(mm.MM_APP_STREAM, [n, 1, 0, 32, 1], G=2, register=False) as s:
         s.fill()
         for slot in range(3):
             assert mm.mm_buffer_register(s.ctx, 4, n, [s.bufs[(slot, d)].data_ptr() for d in range(2)]) == slot
@@ -71,7 +71,7 @@ def test_registered_buffers(R, strategy):
 @pytest.mark.gpu
 def test_registered_buffer_shape_mismatch(R):
     _, runner = R
-    with runner.session(mm.MM_APP_STREAM, [4096, 1, 0, 32, 1], G=1) as s:
+    with runner.session(mm.MM_APP_STREAM, [4096, 1, 0, 32, 1], G=1, register=False) as s:
         for slot in range(3):
             mm.mm_buffer_register(s.ctx, 4, 4096 if slot < 2 else 1024, [s.bufs[(slot, 0)].data_ptr()])
         plan = s.plan(mm.MM_SP_UNIFIED)
