@@ -12,7 +12,7 @@
 //   leaf q: X_q = (B_q - acc_q) L_qq^{-T}    substitution, thread = row, four
 //                                            32-column sub-blocks in registers
 //
-// Warp roles (192 threads, one CTA per SM):
+// Warp roles (320 threads, one CTA per SM):
 //   warp 0   TMA producer: operand stages of the j <= q-2 terms (X_j hi/lo
 //            from the step's panel slot, written back by this CTA's earlier
 //            leaves; L_qj hi/lo from the L_kk slot) and the B half of the
@@ -21,7 +21,10 @@
 //            single-thread MMA issuer; the j = q-1 term reads X_{q-1} straight
 //            from TMEM (TS form), so the critical hand-off leaf q-1 -> acc_q
 //            never goes through global memory
-//   warps 2-5 the substitution (TMEM lane = row).  A sub-block: x = B -
+//   warps 2-9 the substitution (TMEM lane = row; warps w and w+4 share a
+//            row group, each taking 16 of a sub-block's 32 columns: the first
+//            solves its 16 and hands them to the second through TMEM, so the
+//            arithmetic and its order are one thread's).  A sub-block: x = B -
 //            acc (tcgen05.ld), minus the earlier sub-blocks of the leaf
 //            (accumulated first, ascending, as in the leaf kernels), then the
 //            32-column forward substitution with div_rcp quotients; the
@@ -57,7 +60,7 @@ namespace {
 
 using namespace tcx;
 
-constexpr int kTcRows = 128, kTcLeaf = 128, kTcBK = 16, kTcStages = 3, kTcThreads = 192;
+constexpr int kTcRows = 128, kTcLeaf = 128, kTcBK = 16, kTcStages = 3, kTcThreads = 320;
 constexpr int kTcOpBytes = kTcRows * kTcBK * 4;            // 8 KB: one operand box (16 fp32 x 128 rows)
 constexpr int kTcStageBytes = 4 * kTcOpBytes;               // A hi, A lo, B hi, B lo
 // The leaf's L block, packed as the 32 x 32 blocks the substitution reads
@@ -201,7 +204,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       mbar_init(&tfull[q], 1);
       mbar_init(&xgl[q], 1);
       mbar_init(&lsb[q], 1);
-      for (int u = 0; u < 4; ++u) mbar_init(&xsub[4 * q + u], 128);
+      for (int u = 0; u < 4; ++u) mbar_init(&xsub[4 * q + u], 256);
     }
     mbar_init(&bful[0], 1);
     mbar_init(&bful[1], 1);
@@ -314,8 +317,10 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
     }
     __syncwarp();
-  } else {   // ===== substitution: warps 2..5, row = TMEM lane
-    const int grp = warp & 3, rr = grp * 32 + lane;
+  } else {   // ===== substitution: warps 2..9, row = TMEM lane, two warps per row group
+    // (warps w and w + 4 share TMEM lanes 32 (w % 4) ..: half hf = 0 / 1 takes
+    // columns 16 hf .. 16 hf + 15 of every sub-block)
+    const int grp = warp & 3, rr = grp * 32 + lane, hf = (warp - 2) >> 2, cb = 16 * hf;
     const uint32_t lane_off = (uint32_t)(grp * 32) << 16;
     const float* brow = A + ((int64_t)yx + rr) * b;   // this row of tile (ti, k): B, then X
     const float* rd = LsT + kLtRd;
@@ -351,35 +356,35 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         const int idx = 4 * q + s;
         if (issuer) bload(idx + 1);
         twait(&bful[idx & 1], (uint32_t)((idx >> 1) & 1));
-        float x[32];
+        float x[16];
         {
           const float* bp = bpre + (idx & 1) * 4096 + rr * 32;
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {
-            const float4 v = *reinterpret_cast<const float4*>(bp + ((u ^ (rr & 7)) * 4));
-            x[4 * u] = v.x; x[4 * u + 1] = v.y; x[4 * u + 2] = v.z; x[4 * u + 3] = v.w;
+          for (int v = 0; v < 4; ++v) {
+            const float4 t = *reinterpret_cast<const float4*>(bp + (((4 * hf + v) ^ (rr & 7)) * 4));
+            x[4 * v] = t.x; x[4 * v + 1] = t.y; x[4 * v + 2] = t.z; x[4 * v + 3] = t.w;
           }
         }
         if (q >= 1) {   // x = B - sum_{j<q} X_j L_qj^T
-          float a[32];
-          tmem_ld32(accq + (uint32_t)(32 * s), a);
+          float a[16];
+          tmem_ld16(accq + (uint32_t)(32 * s + cb), a);
 #pragma unroll
-          for (int c = 0; c < 32; ++c) x[c] -= a[c];
+          for (int c = 0; c < 16; ++c) x[c] -= a[c];
         }
         if (s > 0) {   // earlier sub-blocks of this leaf: accumulate ascending, subtract once
-          float acc[32];
+          float acc[16];
 #pragma unroll
-          for (int c = 0; c < 32; ++c) acc[c] = 0.f;
+          for (int c = 0; c < 16; ++c) acc[c] = 0.f;
 #pragma unroll 1
           for (int m0 = 0; m0 < 32 * s; m0 += 16) {
             float xm[16];
             tmem_ld16(accq + (uint32_t)m0, xm);
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
-              const float4* l4 =
-                  reinterpret_cast<const float4*>(LsT + kLtU + (s * (s - 1) / 2 + (m0 >> 5)) * 1024 + ((m0 & 31) + i) * 32);
+              const float4* l4 = reinterpret_cast<const float4*>(
+                  LsT + kLtU + (s * (s - 1) / 2 + (m0 >> 5)) * 1024 + ((m0 & 31) + i) * 32 + cb);
 #pragma unroll
-              for (int u = 0; u < 8; ++u) {
+              for (int u = 0; u < 4; ++u) {
                 const float4 l = l4[u];
                 acc[4 * u + 0] = fmaf(xm[i], l.x, acc[4 * u + 0]);
                 acc[4 * u + 1] = fmaf(xm[i], l.y, acc[4 * u + 1]);
@@ -389,17 +394,41 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             }
           }
 #pragma unroll
-          for (int c = 0; c < 32; ++c) x[c] -= acc[c];
+          for (int c = 0; c < 16; ++c) x[c] -= acc[c];
         }
+        // the 32-column substitution: half 0 solves columns 0..15 and hands
+        // them over through TMEM (fp32, the consumed accumulator columns);
+        // half 1 applies them, then solves 16..31 — the operations and their
+        // order are those of one thread doing all 32
+        const float* Ds = LsT + kLtD + s * 1024;   // Ds[c * 32 + c2] = L[c0+32s+c2][c0+32s+c]
+        if (hf == 0) {
 #pragma unroll
-        for (int c = 0; c < 32; ++c) {
-          const float* lc = LsT + kLtD + s * 1024 + c * 32;   // lc[c2] = L[c0+32s+c2][c0+32s+c]
-          x[c] = div_q(x[c], lc[c], rd[32 * s + c]);
+          for (int c = 0; c < 16; ++c) {
+            x[c] = div_q(x[c], Ds[c * 32 + c], rd[32 * s + c]);
 #pragma unroll
-          for (int c2 = c + 1; c2 < 32; ++c2) x[c2] -= x[c] * lc[c2];
+            for (int c2 = c + 1; c2 < 16; ++c2) x[c2] -= x[c] * Ds[c * 32 + c2];
+          }
+          tmem_st16(accq + (uint32_t)(32 * s), x);
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          asm volatile("bar.sync %0, 64;" ::"r"(2 + grp) : "memory");
+        } else {
+          asm volatile("bar.sync %0, 64;" ::"r"(2 + grp) : "memory");
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          float x0[16];
+          tmem_ld16(accq + (uint32_t)(32 * s), x0);
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+#pragma unroll
+            for (int c = 0; c < 16; ++c) x[c] -= x0[i] * Ds[i * 32 + 16 + c];
+#pragma unroll
+          for (int c = 0; c < 16; ++c) {
+            x[c] = div_q(x[c], Ds[(16 + c) * 32 + 16 + c], rd[32 * s + 16 + c]);
+#pragma unroll
+            for (int c2 = c + 1; c2 < 16; ++c2) x[c2] -= x[c] * Ds[(16 + c) * 32 + 16 + c2];
+          }
+          tmem_st16(accq + (uint32_t)(32 * s + 16), x);
         }
-        // fp32 x into the consumed accumulator columns, hi/lo for the MMA
-        tmem_st32(accq + (uint32_t)(32 * s), x);
         // hi/lo to TMEM columns 256 / 384 + 32 s (their previous contents, X_{q-1},
         // were read by acc_q's MMAs, complete before tfull[q])
         const uint32_t xslot = tmem + 256u + lane_off + (uint32_t)(32 * s);
@@ -414,21 +443,20 @@ __global__ void __launch_bounds__(kTcThreads, 1)
             asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
           }
         }
-        asm volatile("bar.sync 1, 128;" ::: "memory");
-#pragma unroll
-        for (int hh = 0; hh < 2; ++hh) {
+        asm volatile("bar.sync 1, 256;" ::: "memory");
+        {
           float h[16], l[16];
 #pragma unroll
           for (int c = 0; c < 16; ++c) {
-            h[c] = tf32_rn(x[16 * hh + c]);
-            l[c] = tf32_rn(x[16 * hh + c] - h[c]);
+            h[c] = tf32_rn(x[c]);
+            l[c] = tf32_rn(x[c] - h[c]);
           }
-          tmem_st16(xslot + (uint32_t)(16 * hh), h);
-          tmem_st16(xslot + 128u + (uint32_t)(16 * hh), l);
+          tmem_st16(xslot + (uint32_t)cb, h);
+          tmem_st16(xslot + 128u + (uint32_t)cb, l);
 #pragma unroll
           for (int v = 0; v < 4; ++v) {
-            const int u = 4 * hh + v, off = rr * 32 + ((u ^ (rr & 7)) * 4);
-            *reinterpret_cast<float4*>(stg + off) = make_float4(x[4 * u], x[4 * u + 1], x[4 * u + 2], x[4 * u + 3]);
+            const int u = 4 * hf + v, off = rr * 32 + ((u ^ (rr & 7)) * 4);
+            *reinterpret_cast<float4*>(stg + off) = make_float4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
             *reinterpret_cast<float4*>(stg + 4096 + off) = make_float4(h[4 * v], h[4 * v + 1], h[4 * v + 2], h[4 * v + 3]);
             *reinterpret_cast<float4*>(stg + 8192 + off) = make_float4(l[4 * v], l[4 * v + 1], l[4 * v + 2], l[4 * v + 3]);
           }
@@ -437,7 +465,8 @@ __global__ void __launch_bounds__(kTcThreads, 1)
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(&xsub[4 * q + s]);   // acc_{q+1}'s MMAs may read this sub-block
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        asm volatile("bar.sync 1, 128;" ::: "memory");
+        asm volatile("bar.sync 1, 256;" ::: "memory");
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");   // the other half's x columns
         if (issuer) {
           const int32_t xc = c0 + 32 * s;
           tma_store_2d(&tSx, xc, yx, stg);
@@ -448,7 +477,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       }
       // leaf q done: LsT free, accumulator q%3 free after the x reads above
       if (issuer && q < 8) stamp(9 + q);
-      asm volatile("bar.sync 1, 128;" ::: "memory");
+      asm volatile("bar.sync 1, 256;" ::: "memory");
       if (issuer) {
         pending = q;
         if (q + 1 < nleaf) {
