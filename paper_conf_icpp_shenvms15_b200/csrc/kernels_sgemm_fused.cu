@@ -33,9 +33,13 @@
 // 64 clk per 256 x 128 x 8 pair MMA, TS or SS, also with streamed operand
 // stages); the rest of the ~940 clk per k-step is per-step overhead that
 // neither an 8-stage split ring, 4 converter groups, two stages per
-// wait/commit round nor issuing without waiting for split_full removed
-// (all measured unchanged; doubling the MMAs of a step added exactly their
-// 64 clk each).
+// wait/commit round, the MMA warp as the highest warp id of its
+// sub-partition nor issuing without waiting for split_full removed (all
+// measured unchanged; doubling the MMAs of a step added exactly their 64 clk
+// each).  Issuing all 192 MMAs without any wait still takes 14.5 us (~148 clk
+// per MMA) here, while the microbenchmark of the same issue pattern (pair, TS,
+// streamed stages, fence + multicast commit per step) runs at 79 clk and at
+// 96 clk with three warps per CTA storing to TMEM beside it.
 // Tried and dropped: 256-wide pairs with S = 3 (24.9 us, both operands in
 // smem: 26 us), a cp.async.bulk push of the partial slices and a reduction
 // through L2 (both slower than the DSMEM pull).

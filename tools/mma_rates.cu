@@ -134,15 +134,41 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1) k_mma2(long 
   cluster_sync_all();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = tslot;
+  __shared__ int stop2;
+  if (threadIdx.x == 0) stop2 = 0;
+  __syncthreads();
+  cluster_sync_all();
+  if (C == 6 && warp >= 1) {
+    const int lane = threadIdx.x & 31;
+    float v[16];
+    for (int c = 0; c < 16; ++c) v[c] = lane * 1.f + c;
+    int it = 0;
+    while (!*(volatile int*)&stop2 && it < 400000) {
+      asm volatile(
+          "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+              tmem + ((uint32_t)((warp & 3) * 32) << 16) + 128u + (uint32_t)((it & 7) * 16)),
+          "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]), "f"(v[8]), "f"(v[9]),
+          "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15])
+          : "memory");
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      ++it;
+      if (rank == 1 && (it & 255) == 0) {   // the peer stops when the leader does
+        uint32_t v2;
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v2) : "r"(peer_addr(&stop2, 0)) : "memory");
+        if (v2) break;
+      }
+    }
+  }
   if (threadIdx.x == 0 && rank == 0) {
     const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
     const uint64_t a = sdesc(base), b = sdesc(base + 8192);
     long long t0 = clock64();
     for (int i = 0; i < R; ++i) {
       const uint64_t adv = (uint64_t)((i & 1) * 32) >> 4;
-      if (C == 3 || C == 4) {   // fused-kernel pattern: 6 MMAs per k-step, stage = k-step % 8 (C=4: stage 0 only)
+      if (C >= 3) {   // fused-kernel pattern: 6 MMAs per k-step, stage = k-step % 8 (C=4: stage 0 only)
         if (i % 6) continue;
-        const int st = C == 3 ? (i / 6) % 8 : 0;
+        const int st = C != 4 ? (i / 6) % 8 : 0;
+        if (C >= 5) asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint64_t bhi = sdesc(base + 8192 + st * 8192), blo = sdesc(base + 8192 + st * 8192 + 4096);
         const uint32_t ahi = tmem + 128u + (uint32_t)(st * 32), alo = ahi + 16u;
 #pragma unroll
@@ -152,6 +178,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1) k_mma2(long 
           mma_ts2(tmem, ahi + 8u * kk, blo + ad, idesc);
           mma_ts2(tmem, ahi + 8u * kk, bhi + ad, idesc);
         }
+        if (C >= 5) mma_commit_pair(&sbar[(i / 6) & 3]);
       } else if (TS) {
         asm volatile(
             "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
@@ -171,6 +198,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(128, 1) k_mma2(long 
     mbar_wait(&bar, 0);
     long long t1 = clock64();
     out[blockIdx.x / 2] = (t1 - t0);
+    stop2 = 1;
   }
   if (threadIdx.x == 0 && rank == 1) mbar_wait(&bar, 0);
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -216,6 +244,8 @@ int main() {
   run<128, false, 2>("SS128+sts", 4096, d, 148);
   run2<128, true, 3>("2TS128stm", 4098, d, 74);
   run2<128, true, 4>("2TS128st0", 4098, d, 74);
+  run2<128, true, 5>("2TS128fus", 4098, d, 74);
+  run2<128, true, 6>("2TS128f+d", 4098, d, 74);
   run2<128, true, 1>("2TS128+cm", 4098, d, 74);
   run2<128, true, 2>("2TS128+cmf", 4098, d, 74);
   for (int pairs : {1, 74}) {
