@@ -55,6 +55,22 @@ def test_cholesky_exact_factor_bench_tile(R, b, strategy, G):
         assert np.all(np.triu(L[k * b:(k + 1) * b, k * b:(k + 1) * b], 1) == 0)
 
 
+@pytest.mark.parametrize("b", [2048, 4096, 256])
+def test_cholesky_exact_factor_wide_tiles(R, b):
+    """The column TRSM's leaf count b/128 at its extremes (2, 16, 32 leaves;
+    kernels_chol_trsm.cu kMaxLeaves = 32): n = 2 b (or 8192 for b = 256),
+    exact-factor input, the factor is L0 bit for bit."""
+    mm, runner = R
+    n = 2 * b if b > 256 else 8192
+    A, L0 = synthgen.cholesky_exact_factor(n)
+    with runner.session(mm.MM_APP_CHOLESKY, [n, b], G=1) as s:
+        s.load(0, _to_tiles(A, b))
+        plan = s.plan(mm.MM_DP_PERF, _prof(mm, 1, 4))
+        s.run(plan)
+        L = _from_tiles(s.collect(plan, 0), n, b)
+    assert np.array_equal(np.tril(L), L0)
+
+
 def test_cholesky_random_spd_bench_tile(R):
     """Random SPD n = 4096 at b = 1024 (4 x 4 tiles, the bench's kernels and
     batching) against the FP64 oracle (unblocked Cholesky-Banachiewicz):
