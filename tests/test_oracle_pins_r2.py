@@ -442,3 +442,55 @@ def test_halo_split_cpp_matches_oracle(G, tb):
     assert ops_as_tuples(plan) == oc.op_program(oapp, G, tasks, dev, oc.SP_SINGLE)
     mm.mm_plan_destroy(plan)
     mm.mm_app_destroy(capp)
+
+
+# ------------------------------------------- per-task compute lane (R31) ------
+def _lane_dag(lanes):
+    """Two kernels over 4 tiles of 16 elements: t0, t1 (kernel 0) write tiles
+    0, 1; t2, t3 (kernel 1) read tiles 0, 1 and write tiles 2, 3; `lanes` =
+    the task lanes (mm_task_desc.lane)."""
+    def acc(mode, t):
+        return oc.TaskAccess(0, mode, 16 * t, 16 * t + 16, 16 * t, 16 * t + 16)
+    tasks = [oc.Task(0, 0, 0, 1, [acc(oc.WRITE, 0)], lane=lanes[0]),
+             oc.Task(0, 0, 16, 17, [acc(oc.WRITE, 1)], lane=lanes[1]),
+             oc.Task(1, 0, 32, 33, [acc(oc.READ, 0), acc(oc.WRITE, 2)], lane=lanes[2]),
+             oc.Task(1, 0, 48, 49, [acc(oc.READ, 1), acc(oc.WRITE, 3)], lane=lanes[3])]
+    return oc.App(buffers=[(4, 64)], kernels=[oc.Kernel("a", 1, 1, 1, []), oc.Kernel("b", 1, 1, 1, [])],
+                  edges=[(0, 1)], dag_tasks=tasks)
+
+
+# One device, estimates kernel 0: 100 ns, kernel 1: 10 ns.  By hand:
+#   all on lane 0: t0 100, t1 200, t2 max(200, 100) + 10 = 210, t3 220
+#   t1, t3 on lane 1: t0 100 | t1 100 (lane 1 free); t2 max(100, 100) + 10 = 110 |
+#                     t3 max(100, ready t1 100) + 10 = 110
+LANE_DAG_FIN = {(0, 0, 0, 0): [100, 200, 210, 220], (0, 1, 0, 1): [100, 100, 110, 110]}
+
+
+@pytest.mark.parametrize("lanes", sorted(LANE_DAG_FIN))
+def test_dp_perf_task_lanes_by_hand(lanes):
+    prof = oc.Profile(G=1, fs_item=[[1, 1]], chunk_est_ns=[[100, 10]], link_Bps=[10 ** 9])
+    _, dev, fin = oc.dp_perf(_lane_dag(lanes), prof)
+    assert dev == [0] * 4 and fin == LANE_DAG_FIN[lanes]
+
+
+@pytest.mark.parametrize("lanes", sorted(LANE_DAG_FIN))
+def test_dp_perf_task_lanes_cpp(lanes):
+    """The same DAG through the C ABI (mm_app_add_task with mm_task_desc.lane)."""
+    mm = pytest.importorskip("paper_conf_icpp_shenvms15_b200.mm")
+    app = mm.mm_app_create()
+    mm.mm_app_add_buffer(app, 4, 64)
+    for nm in ("a", "b"):
+        # a builtin op as a stand-in: the test only plans (a custom op needs a launch callback)
+        mm.mm_app_add_kernel(app, mm.kernel_desc(nm, mm.MM_OP_STREAM_COPY, 1, [], granule=1))
+    mm.mm_app_add_edge(app, 0, 1)
+    spec = [(0, [(0, mm.MM_WRITE, 0, 16)]), (0, [(0, mm.MM_WRITE, 16, 32)]),
+            (1, [(0, mm.MM_READ, 0, 16), (0, mm.MM_WRITE, 32, 48)]),
+            (1, [(0, mm.MM_READ, 16, 32), (0, mm.MM_WRITE, 48, 64)])]
+    for (k, acc), ln in zip(spec, lanes):
+        mm.mm_app_add_task(app, k, [0, 0, 0, 0], acc, lane=ln)
+    mm.mm_app_finalize(app)
+    prof = mm.make_profile(1, [[1, 1]], [[100, 10]], [10 ** 9])
+    plan = mm.mm_plan_build(app, prof, mm.plan_opts(mm.MM_DP_PERF))
+    assert [c.finish_ns for c in mm.mm_plan_chunks(plan)] == LANE_DAG_FIN[lanes]
+    mm.mm_plan_destroy(plan)
+    mm.mm_app_destroy(app)
