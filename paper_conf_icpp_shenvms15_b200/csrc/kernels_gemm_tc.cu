@@ -447,6 +447,35 @@ __global__ void __launch_bounds__(256) split_ab(const float* __restrict__ A, flo
   }
 }
 
+// B (K x N, row-major) -> B_hi^T, B_lo^T (N x Kp, K-major), one 32 (k) x 128
+// (n) block per CTA: float4 row loads into a padded smem tile, then each warp
+// writes 128-B runs of k for its n rows (both sides coalesced).  K % 32 == 0,
+// N % 4 == 0.
+__global__ void __launch_bounds__(256) split_bT(const float* __restrict__ B, float* __restrict__ bhi,
+                                                float* __restrict__ blo, int64_t N, int64_t Kp, int ntn) {
+  __shared__ float t[32][128 + 1];
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const int64_t k0 = (int64_t)(blockIdx.x / ntn) * 32, n0 = (int64_t)(blockIdx.x % ntn) * 128;
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {            // 32 rows x 32 float4
+    const int e = tid + 256 * j, r = e >> 5, c4 = (e & 31) * 4;
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (n0 + c4 < N) v = *reinterpret_cast<const float4*>(B + (k0 + r) * N + n0 + c4);
+    t[r][c4] = v.x; t[r][c4 + 1] = v.y; t[r][c4 + 2] = v.z; t[r][c4 + 3] = v.w;
+  }
+  __syncthreads();
+  const int lane = tid & 31, w = tid >> 5;
+#pragma unroll 4
+  for (int nn = w; nn < 128; nn += 8) {    // output row n0 + nn: k0 .. k0 + 31 (lane = k)
+    if (n0 + nn >= N) break;
+    float h, l;
+    split2(t[lane][nn], h, l);
+    bhi[(n0 + nn) * Kp + k0 + lane] = h;
+    blo[(n0 + nn) * Kp + k0 + lane] = l;
+  }
+}
+
 // Split panel tiles: tile (list[t].i, k) of the tile-major matrix -> slot
 // slot0 + i of the hi/lo panel buffers (b x b each, row-major = K-major rows).
 __global__ void split_tiles(const float* __restrict__ A, float* __restrict__ hi, float* __restrict__ lo,
@@ -733,6 +762,9 @@ size_t sgemm_tf32x3_scratch(int64_t N, int64_t K, int64_t mrows) {
 int sgemm_fused_splits(const float* A, const float* B, float* C, int64_t mrows, int64_t N, int64_t K, int64_t r0);
 cudaError_t sgemm_fused_rows(const float* A, const float* B, float* C, int64_t N, int64_t K, int64_t r0,
                              int64_t mrows, int S, cudaStream_t s);
+bool sgemm_fused_presplit_b();
+cudaError_t sgemm_fused_presplit_rows(const float* A, const float* bhi, const float* blo, int64_t Kp, float* C,
+                                      int64_t N, int64_t K, int64_t r0, int64_t mrows, int S, cudaStream_t s);
 
 cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t M, int64_t N, int64_t K,
                               int64_t r0, int64_t r1, cudaStream_t s, int sms, Scratch* scr, bool b_readonly) {
@@ -744,6 +776,20 @@ cudaError_t sgemm_tf32x3_rows(const float* A, const float* B, float* C, int64_t 
     // in shared memory and reduces its K splits inside the cluster
     // (kernels_sgemm_fused.cu) instead of split -> GEMM -> reduce below
     const int S = sgemm_fused_splits(A, B, C, mrows, N, K, r0);
+    const int64_t Kp0 = (K + KPAD - 1) / KPAD * KPAD;
+    if (S > 1 && sgemm_fused_presplit_b() && K % KPAD == 0 && (N & 3) == 0 && scr && scr->ptr &&
+        scr->bytes >= sgemm_tf32x3_scratch(N, K, mrows)) {
+      // B split + transposed by one launch (its B part of split_ab), then the
+      // fused kernel converts only A (the B transposition dominated it)
+      float* bh = static_cast<float*>(scr->ptr);
+      float* bl = bh + N * Kp0;
+      const int ntn = (int)((N + 127) / 128);
+      note_launch();
+      split_bT<<<(unsigned)((int64_t)ntn * (Kp0 / 32)), 256, 0, s>>>(B, bh, bl, N, Kp0, ntn);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return e;
+      return sgemm_fused_presplit_rows(A, bh, bl, Kp0, C, N, K, r0, mrows, S, s);
+    }
     if (S > 1) return sgemm_fused_rows(A, B, C, N, K, r0, mrows, S, s);
   }
   if (!scr || !scr->ptr || scr->bytes < sgemm_tf32x3_scratch(N, K, mrows)) return cudaErrorNotSupported;

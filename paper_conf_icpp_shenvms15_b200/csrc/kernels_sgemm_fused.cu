@@ -1,5 +1,19 @@
 // Small-SGEMM path of MatrixMul (BASELINE configs[0], 1024^2; P311 C = A x B,
-// row-wise split) in ONE launch: no operand-split pass, no reduction pass.
+// row-wise split): fused kernels with no reduction pass.  Three variants
+// (MM_SGEMM_FUSED = 1 / 2 / 3, default 3):
+//  3  split_bT (kernels_gemm_tc.cu) writes B_hi^T / B_lo^T once, then
+//     sgemm_fused2: single-SM 128 x 256 tiles (tcgen05 M = 128, N = 256), S = 4
+//     K splits per cluster; TMA brings raw A and the split B, the converter
+//     warps only split A into TMEM.  1024^2: split_bT 4.9 us + sgemm_fused2
+//     19.0 us (ncu, serialised; PDL overlaps them in the stream), bench step
+//     30.2 us.  globaltimer: main loop 7.6 us for 16 k-steps (~82 % of the
+//     MMA time), TMEM -> smem 1.5 us, cluster barrier 0.8 us, DSMEM reduction
+//     of 4 partials 3.9 us.
+//  2  sgemm_fused1: the same tiles with B transposed and split in-kernel by
+//     the converter warps (25.4 us: the B transposition keeps the main loop
+//     at ~15 us).
+//  1  the pair design below (25.3 us).
+// Variant 1, the original fused kernel, in ONE launch: no operand-split pass.
 //
 // A cluster of 2 S CTAs computes one 256 x 128 output tile pair over S K
 // splits (S in 2..4, the largest whose clusters are all resident at once):
@@ -406,6 +420,457 @@ __global__ void __launch_bounds__(kFThreads, 1)
   }
 }
 
+// ---------------------------------------------------------------------------
+// Single-SM variant (round 2): one CTA = 128 rows x 256 columns (M = 128,
+// N = 256 tcgen05.mma.cta_group::1, twice the work per instruction of the
+// pair's 256 x 128), S K splits in a cluster of S CTAs reduced through DSMEM.
+// Same stage pipeline: raw TMA ring -> converter warps (A to TMEM, B
+// transposed into the K-major SWIZZLE_64B smem layout) -> MMA thread.
+constexpr int G1N = 256;                                       // output columns per CTA (MMA N)
+constexpr int RAW1_A = FBM * FBK * 4, RAW1_B = G1N * FBK * 4;  // 8 KB + 16 KB
+constexpr int RAW1_BYTES = RAW1_A + RAW1_B;
+constexpr int kRaw1 = 6, kSplit1 = 2;
+constexpr int SPLIT1_BYTES = 2 * RAW1_B;                       // B_hi, B_lo
+constexpr int kRing1 = kRaw1 * RAW1_BYTES + kSplit1 * SPLIT1_BYTES;   // 208 KB
+constexpr int RED1_LD = G1N + 4;
+constexpr int kTmem1 = 512;                                    // 256 accumulator + kSplit1 x 32 A columns
+static_assert(G1N + kSplit1 * 32 <= kTmem1, "TMEM columns");
+static_assert(FBM * RED1_LD * 4 <= kRing1, "partial buffer");
+constexpr int kFused1Smem = kRing1 + 1024 + 256;
+
+__device__ __forceinline__ void mma_tf32_ts1(uint32_t tmem_d, uint32_t tmem_a, uint64_t b, uint32_t idesc,
+                                             uint32_t acc) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(b), "r"(idesc), "r"(acc));
+}
+
+__global__ void __launch_bounds__(kFThreads, 1)
+    sgemm_fused1(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tB, float* __restrict__ C,
+                 int64_t N, int64_t row0, int64_t mrows, int nblk, int S, int nkb_all) {
+  uint32_t z;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(z));
+  const int cl = (int)(blockIdx.x / S);
+  const int m_blk = cl / nblk, nb = cl % nblk;
+  const int kb0 = (int)z * nkb_all / S, nkb = ((int)z + 1) * nkb_all / S - kb0;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = smem_raw + ((1024u - (saddr(smem_raw) & 1023u)) & 1023u);
+  uint8_t* raw = base;
+  uint8_t* spl = base + kRaw1 * RAW1_BYTES;
+  uint64_t* raw_full = reinterpret_cast<uint64_t*>(base + kRing1);
+  uint64_t* raw_empty = raw_full + kRaw1;
+  uint64_t* split_full = raw_empty + kRaw1;    // this CTA's 4 converter warps of the stage's group
+  uint64_t* split_empty = split_full + kSplit1;
+  uint64_t* tfull = split_empty + kSplit1;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (warp == 0 && lane == 0) {
+    for (int q = 0; q < kRaw1; ++q) {
+      mbar_init(&raw_full[q], 1);
+      mbar_init(&raw_empty[q], 4);
+    }
+    for (int q = 0; q < kSplit1; ++q) {
+      mbar_init(&split_full[q], 4);
+      mbar_init(&split_empty[q], 1);
+    }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tB) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)), "n"(kTmem1));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tslot;
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+
+  if (warp == 0) {
+    if (lane == 0) {   // ===== producer: raw A (16 k x 128 rows) and B (16 k-rows x 256 columns)
+      const int32_t ya = m_blk * FBM, xb = nb * G1N;
+      for (int i = 0; i < nkb; ++i) {
+        const int q = i % kRaw1;
+        if (i >= kRaw1) fwait(&raw_empty[q], (uint32_t)(((i / kRaw1) - 1) & 1));
+        uint8_t* st = raw + q * RAW1_BYTES;
+        const int32_t kx = (kb0 + i) * FBK;
+        mbar_expect_tx(&raw_full[q], RAW1_BYTES);
+        tma_load_2d(st, &tA, kx, ya, &raw_full[q]);
+#pragma unroll
+        for (int j = 0; j < G1N / 32; ++j) tma_load_2d(st + RAW1_A + j * 2048, &tB, xb + 32 * j, kx, &raw_full[q]);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0) {   // ===== MMA issuer (every CTA is its own issuer)
+      const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(G1N >> 3) << 17) |
+                             ((uint32_t)(FBM >> 4) << 24);
+      for (int i = 0; i < nkb; ++i) {
+        const int q = i % kSplit1;
+        fwait(&split_full[q], (uint32_t)((i / kSplit1) & 1));
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        uint8_t* st = spl + q * SPLIT1_BYTES;
+        const uint64_t bhi = sdesc(st), blo = sdesc(st + RAW1_B);
+        const uint32_t ahi = tmem + (uint32_t)G1N + (uint32_t)(q * 32), alo = ahi + 16u;
+#pragma unroll
+        for (int kk = 0; kk < FBK / 8; ++kk) {
+          const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+          mma_tf32_ts1(tmem, alo + 8u * kk, bhi + adv, idesc, (i | kk) != 0);
+          mma_tf32_ts1(tmem, ahi + 8u * kk, blo + adv, idesc, 1u);
+          mma_tf32_ts1(tmem, ahi + 8u * kk, bhi + adv, idesc, 1u);
+        }
+        mma_commit(&split_empty[q]);
+      }
+      mma_commit(tfull);
+    }
+    __syncwarp();
+  } else {   // ===== converters (warps 2..9, two groups alternating k-steps), then the epilogue
+    const int cg = (warp - 2) / 4;
+    const int ct = (threadIdx.x - 64) & 127;
+    for (int i = cg; i < nkb; i += kConvGroups) {
+      const int q = i % kRaw1, p = i % kSplit1;
+      fwait(&raw_full[q], (uint32_t)((i / kRaw1) & 1));
+      if (i >= kSplit1) fwait(&split_empty[p], (uint32_t)(((i / kSplit1) - 1) & 1));
+      const uint8_t* rs = raw + q * RAW1_BYTES;
+      uint8_t* dst = spl + p * SPLIT1_BYTES;
+      const int ar = (warp & 3) * 32 + lane;
+      float4 v[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        v[c] = *reinterpret_cast<const float4*>(rs + ar * 64 + ((c ^ ((ar >> 1) & 3)) << 4));
+      constexpr int NB4 = G1N * 4 / 128;   // 8 B output float4 per converter thread
+#pragma unroll 2
+      for (int j0 = 0; j0 < NB4; j0 += 2) {
+        float4 w[2];
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const int o = ct + 128 * (j0 + j), n = o % G1N, k0 = 4 * (o / G1N);
+          const uint8_t* box = rs + RAW1_A + (n >> 5) * 2048 + (n & 3) * 4;
+          const int c16 = (n & 31) >> 2;
+          float t[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const int k = k0 + u;
+            t[u] = *reinterpret_cast<const float*>(box + k * 128 + ((c16 ^ (k & 7)) << 4));
+          }
+          w[j] = make_float4(t[0], t[1], t[2], t[3]);
+        }
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          float4 hi, lo;
+          const int o = ct + 128 * (j0 + j), n = o % G1N, kc4 = o / G1N;
+          const int boff = n * 64 + ((kc4 ^ ((n >> 1) & 3)) << 4);
+          split2(w[j].x, hi.x, lo.x);
+          split2(w[j].y, hi.y, lo.y);
+          split2(w[j].z, hi.z, lo.z);
+          split2(w[j].w, hi.w, lo.w);
+          *reinterpret_cast<float4*>(dst + boff) = hi;
+          *reinterpret_cast<float4*>(dst + RAW1_B + boff) = lo;
+        }
+      }
+      {
+        float ah[16], al[16];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          split2(v[c].x, ah[4 * c], al[4 * c]);
+          split2(v[c].y, ah[4 * c + 1], al[4 * c + 1]);
+          split2(v[c].z, ah[4 * c + 2], al[4 * c + 2]);
+          split2(v[c].w, ah[4 * c + 3], al[4 * c + 3]);
+        }
+        const uint32_t ta = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)G1N + (uint32_t)(p * 32);
+        tmem_st16(ta, ah);
+        tmem_st16(ta + 16u, al);
+      }
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) {
+        mbar_arrive(&raw_empty[q]);
+        mbar_arrive(&split_full[p]);
+      }
+    }
+    // ---- epilogue: accumulator -> this CTA's smem partial (or C when S = 1)
+    const int grp = warp & 3;
+    fwait(tfull, 0);
+    asm volatile("bar.sync 1, %0;" ::"n"(128 * kConvGroups) : "memory");
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int r = grp * 32 + lane;
+    const int64_t grow = (int64_t)m_blk * FBM + r;
+    float* red = reinterpret_cast<float*>(base);
+    for (int c = cg * (G1N / kConvGroups); c < (cg + 1) * (G1N / kConvGroups); c += 16) {
+      uint32_t v[16];
+      const uint32_t ta = tmem + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+          : "r"(ta));
+      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      if (S > 1) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          *reinterpret_cast<float4*>(red + r * RED1_LD + c + 4 * u) =
+              make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]), __uint_as_float(v[4 * u + 2]),
+                          __uint_as_float(v[4 * u + 3]));
+      } else if (grow < mrows) {
+        const int64_t n0 = (int64_t)nb * G1N + c;
+        float* crow = C + (row0 + grow) * N;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (n0 + 4 * u < N)
+            *reinterpret_cast<float4*>(crow + n0 + 4 * u) =
+                make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                            __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+      }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  }
+  __syncthreads();
+  if (S > 1) {
+    cluster_sync_all();   // every partial of the cluster is in shared memory
+    // CTA z reduces float4 columns [z G1N/4 / S, (z+1) G1N/4 / S) of the 128
+    // rows over the S partials in split order ((p0 + p1) + p2) + p3
+    const int c4a = (int)z * (G1N / 4) / S, c4n = ((int)z + 1) * (G1N / 4) / S - c4a;
+    const float* red = reinterpret_cast<const float*>(base);
+    uint32_t peer[4];
+#pragma unroll
+    for (int zz = 0; zz < 4; ++zz) peer[zz] = peer_addr(red, (uint32_t)(zz < S ? zz : 0));
+    for (int e = threadIdx.x; e < FBM * c4n; e += kFThreads) {
+      const int rr = e / c4n, cc = 4 * (c4a + e % c4n);
+      const uint32_t off = (uint32_t)((rr * RED1_LD + cc) * 4);
+      float4 pp[4];
+#pragma unroll
+      for (int zz = 0; zz < 4; ++zz)
+        if (zz < S) pp[zz] = ld_dsmem_f4(peer[zz] + off);
+      float4 a = pp[0];
+#pragma unroll
+      for (int zz = 1; zz < 4; ++zz)
+        if (zz < S) {
+          a.x += pp[zz].x; a.y += pp[zz].y; a.z += pp[zz].z; a.w += pp[zz].w;
+        }
+      const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * G1N + cc;
+      if (grow < mrows && n0 < N) *reinterpret_cast<float4*>(C + (row0 + grow) * N + n0) = a;
+    }
+    cluster_arrive_relaxed_wait();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmem1));
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Pre-split-B variant: as the single-SM variant, but B arrives already split
+// and K-major (split_ab, one launch before, PDL) by TMA, so the converter
+// warps only split A into TMEM (the B transposition was the converters' main
+// load).  Single-SM variant (round 2): one CTA = 128 rows x 256 columns (M = 128,
+// N = 256 tcgen05.mma.cta_group::1, twice the work per instruction of the
+// pair's 256 x 128), S K splits in a cluster of S CTAs reduced through DSMEM.
+// Same stage pipeline: raw TMA ring -> converter warps (A to TMEM, B
+// transposed into the K-major SWIZZLE_64B smem layout) -> MMA thread.
+constexpr int G2N = 256;                                       // output columns per CTA (MMA N)
+constexpr int RAW2_A = FBM * FBK * 4, RAW2_B = G2N * FBK * 4;  // 8 KB + 16 KB (x2: hi, lo)
+constexpr int RAW2_BYTES = RAW2_A + 2 * RAW2_B;
+constexpr int kRaw2 = 5, kSplit2 = 8;                          // raw stages; A stages in TMEM
+constexpr int kRing2 = kRaw2 * RAW2_BYTES;                     // 200 KB
+constexpr int RED2_LD = G2N + 4;
+constexpr int kTmem2 = 512;                                    // 256 accumulator + kSplit2 x 32 A columns
+static_assert(G2N + kSplit2 * 32 <= kTmem2, "TMEM columns");
+static_assert(FBM * RED2_LD * 4 <= kRing2, "partial buffer");
+constexpr int kFused2Smem = kRing2 + 1024 + 256;
+
+__global__ void __launch_bounds__(kFThreads, 1)
+    sgemm_fused2(const __grid_constant__ CUtensorMap tA, const __grid_constant__ CUtensorMap tBh,
+                 const __grid_constant__ CUtensorMap tBl, float* __restrict__ C,
+                 int64_t N, int64_t row0, int64_t mrows, int nblk, int S, int nkb_all) {
+  uint32_t z;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(z));
+  const int cl = (int)(blockIdx.x / S);
+  const int m_blk = cl / nblk, nb = cl % nblk;
+  const int kb0 = (int)z * nkb_all / S, nkb = ((int)z + 1) * nkb_all / S - kb0;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* base = smem_raw + ((1024u - (saddr(smem_raw) & 1023u)) & 1023u);
+  uint8_t* raw = base;
+  uint64_t* raw_full = reinterpret_cast<uint64_t*>(base + kRing2);
+  uint64_t* raw_empty = raw_full + kRaw2;
+  uint64_t* split_full = raw_empty + kRaw2;    // this CTA's 4 converter warps of the stage's group
+  uint64_t* split_empty = split_full + kSplit2;
+  uint64_t* tfull = split_empty + kSplit2;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tfull + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (warp == 0 && lane == 0) {
+    for (int q = 0; q < kRaw2; ++q) {
+      mbar_init(&raw_full[q], 1);
+      mbar_init(&raw_empty[q], 1);          // the MMA commit (B is read by the MMAs in place)
+    }
+    for (int q = 0; q < kSplit2; ++q) {
+      mbar_init(&split_full[q], 4);
+      mbar_init(&split_empty[q], 1);
+    }
+    mbar_init(tfull, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBh) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tBl) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(saddr(tslot)), "n"(kTmem2));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tslot;
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+
+  if (warp == 0) {
+    if (lane == 0) {   // ===== producer: raw A (16 k x 128 rows) and B (16 k-rows x 256 columns)
+      const int32_t ya = m_blk * FBM, xb = nb * G2N;
+      for (int i = 0; i < nkb; ++i) {
+        const int q = i % kRaw2;
+        if (i >= kRaw2) fwait(&raw_empty[q], (uint32_t)(((i / kRaw2) - 1) & 1));
+        uint8_t* st = raw + q * RAW2_BYTES;
+        const int32_t kx = (kb0 + i) * FBK;
+        mbar_expect_tx(&raw_full[q], RAW2_BYTES);
+        tma_load_2d(st, &tA, kx, ya, &raw_full[q]);
+        tma_load_2d(st + RAW2_A, &tBh, kx, xb, &raw_full[q]);            // B_hi^T rows n, 16 k (K-major)
+        tma_load_2d(st + RAW2_A + RAW2_B, &tBl, kx, xb, &raw_full[q]);
+      }
+    }
+    __syncwarp();
+  } else if (warp == 1) {
+    if (lane == 0) {   // ===== MMA issuer (every CTA is its own issuer)
+      const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(G2N >> 3) << 17) |
+                             ((uint32_t)(FBM >> 4) << 24);
+      for (int i = 0; i < nkb; ++i) {
+        const int q = i % kRaw2, p = i % kSplit2;
+        fwait(&raw_full[q], (uint32_t)((i / kRaw2) & 1));      // B of this k-step
+        fwait(&split_full[p], (uint32_t)((i / kSplit2) & 1));  // A of this k-step in TMEM
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        uint8_t* st = raw + q * RAW2_BYTES;
+        const uint64_t bhi = sdesc(st + RAW2_A), blo = sdesc(st + RAW2_A + RAW2_B);
+        const uint32_t ahi = tmem + (uint32_t)G2N + (uint32_t)(p * 32), alo = ahi + 16u;
+#pragma unroll
+        for (int kk = 0; kk < FBK / 8; ++kk) {
+          const uint64_t adv = (uint64_t)(kk * 32) >> 4;
+          mma_tf32_ts1(tmem, alo + 8u * kk, bhi + adv, idesc, (i | kk) != 0);
+          mma_tf32_ts1(tmem, ahi + 8u * kk, blo + adv, idesc, 1u);
+          mma_tf32_ts1(tmem, ahi + 8u * kk, bhi + adv, idesc, 1u);
+        }
+        mma_commit(&raw_empty[q]);     // the converters finished reading this stage's A before split_full
+        mma_commit(&split_empty[p]);
+      }
+      mma_commit(tfull);
+    }
+    __syncwarp();
+  } else {   // ===== converters (warps 2..9, two groups alternating k-steps), then the epilogue
+    const int cg = (warp - 2) / 4;
+    const int ct = (threadIdx.x - 64) & 127;
+    (void)ct;
+    for (int i = cg; i < nkb; i += kConvGroups) {
+      const int q = i % kRaw2, p = i % kSplit2;
+      fwait(&raw_full[q], (uint32_t)((i / kRaw2) & 1));
+      if (i >= kSplit2) fwait(&split_empty[p], (uint32_t)(((i / kSplit2) - 1) & 1));
+      const uint8_t* rs = raw + q * RAW2_BYTES;
+      const int ar = (warp & 3) * 32 + lane;
+      float4 v[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        v[c] = *reinterpret_cast<const float4*>(rs + ar * 64 + ((c ^ ((ar >> 1) & 3)) << 4));
+      float ah[16], al[16];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        split2(v[c].x, ah[4 * c], al[4 * c]);
+        split2(v[c].y, ah[4 * c + 1], al[4 * c + 1]);
+        split2(v[c].z, ah[4 * c + 2], al[4 * c + 2]);
+        split2(v[c].w, ah[4 * c + 3], al[4 * c + 3]);
+      }
+      const uint32_t ta = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)G2N + (uint32_t)(p * 32);
+      tmem_st16(ta, ah);
+      tmem_st16(ta + 16u, al);
+      asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&split_full[p]);
+    }
+    // ---- epilogue: accumulator -> this CTA's smem partial (or C when S = 1)
+    const int grp = warp & 3;
+    fwait(tfull, 0);
+    asm volatile("bar.sync 1, %0;" ::"n"(128 * kConvGroups) : "memory");
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int r = grp * 32 + lane;
+    const int64_t grow = (int64_t)m_blk * FBM + r;
+    float* red = reinterpret_cast<float*>(base);
+    for (int c = cg * (G2N / kConvGroups); c < (cg + 1) * (G2N / kConvGroups); c += 16) {
+      uint32_t v[16];
+      const uint32_t ta = tmem + ((uint32_t)(grp * 32) << 16) + (uint32_t)c;
+      asm volatile(
+          "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+          : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+            "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+          : "r"(ta));
+      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      if (S > 1) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          *reinterpret_cast<float4*>(red + r * RED2_LD + c + 4 * u) =
+              make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]), __uint_as_float(v[4 * u + 2]),
+                          __uint_as_float(v[4 * u + 3]));
+      } else if (grow < mrows) {
+        const int64_t n0 = (int64_t)nb * G2N + c;
+        float* crow = C + (row0 + grow) * N;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (n0 + 4 * u < N)
+            *reinterpret_cast<float4*>(crow + n0 + 4 * u) =
+                make_float4(__uint_as_float(v[4 * u]), __uint_as_float(v[4 * u + 1]),
+                            __uint_as_float(v[4 * u + 2]), __uint_as_float(v[4 * u + 3]));
+      }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  }
+  __syncthreads();
+  if (S > 1) {
+    cluster_sync_all();   // every partial of the cluster is in shared memory
+    // CTA z reduces float4 columns [z G2N/4 / S, (z+1) G2N/4 / S) of the 128
+    // rows over the S partials in split order ((p0 + p1) + p2) + p3
+    const int c4a = (int)z * (G2N / 4) / S, c4n = ((int)z + 1) * (G2N / 4) / S - c4a;
+    const float* red = reinterpret_cast<const float*>(base);
+    uint32_t peer[4];
+#pragma unroll
+    for (int zz = 0; zz < 4; ++zz) peer[zz] = peer_addr(red, (uint32_t)(zz < S ? zz : 0));
+    for (int e = threadIdx.x; e < FBM * c4n; e += kFThreads) {
+      const int rr = e / c4n, cc = 4 * (c4a + e % c4n);
+      const uint32_t off = (uint32_t)((rr * RED2_LD + cc) * 4);
+      float4 pp[4];
+#pragma unroll
+      for (int zz = 0; zz < 4; ++zz)
+        if (zz < S) pp[zz] = ld_dsmem_f4(peer[zz] + off);
+      float4 a = pp[0];
+#pragma unroll
+      for (int zz = 1; zz < 4; ++zz)
+        if (zz < S) {
+          a.x += pp[zz].x; a.y += pp[zz].y; a.z += pp[zz].z; a.w += pp[zz].w;
+        }
+      const int64_t grow = (int64_t)m_blk * FBM + rr, n0 = (int64_t)nb * G2N + cc;
+      if (grow < mrows && n0 < N) *reinterpret_cast<float4*>(C + (row0 + grow) * N + n0) = a;
+    }
+    cluster_arrive_relaxed_wait();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmem2));
+  }
+}
+
 }  // namespace
 
 int max_active_clusters(int csize);
@@ -414,9 +879,27 @@ int max_active_clusters(int csize);
 // least 8 k-blocks per split whose clusters of 2 S CTAs all fit on the GPU at
 // once (one wave: cudaOccupancyMaxActiveClusters), 0 = use the two-pass path
 // (the tile pairs alone fill the GPU, or the operands are not 16-B aligned).
+static int fused_variant() {   // 1: 2-SM pairs (256 x 128), 2: single-SM 128 x 256 tiles, 3: 2 + pre-split B
+  static const int env = getenv("MM_SGEMM_FUSED") ? atoi(getenv("MM_SGEMM_FUSED")) : 3;
+  return env;
+}
+bool sgemm_fused_presplit_b() { return fused_variant() == 3; }
+int max_active_clusters1(int csize);
+
 int sgemm_fused_splits(const float* A, const float* B, float* C, int64_t mrows, int64_t N, int64_t K, int64_t r0) {
-  static const int env = getenv("MM_SGEMM_FUSED") ? atoi(getenv("MM_SGEMM_FUSED")) : 1;
+  const int env = fused_variant();
   if (!env || (K & 3) || (N & 3)) return 0;
+  if (env >= 2) {
+    if ((reinterpret_cast<uintptr_t>(A + r0 * K) | reinterpret_cast<uintptr_t>(B) | reinterpret_cast<uintptr_t>(C)) &
+        15)
+      return 0;
+    const int64_t tiles = (mrows + FBM - 1) / FBM * ((N + G1N - 1) / G1N);
+    const int64_t nkb = (K + FBK - 1) / FBK;
+    if (tiles > 148 / 2) return 0;
+    for (int S = 4; S >= 2; --S)
+      if (nkb / S >= 8 && max_active_clusters1(S) >= tiles) return S;
+    return 0;
+  }
   if ((reinterpret_cast<uintptr_t>(A + r0 * K) | reinterpret_cast<uintptr_t>(B) | reinterpret_cast<uintptr_t>(C)) & 15)
     return 0;
   const int64_t pairs = ((mrows + FBM - 1) / FBM + 1) / 2 * ((N + FBN - 1) / FBN);
@@ -451,8 +934,97 @@ int max_active_clusters(int csize) {
   return n;
 }
 
+int max_active_clusters1(int csize) {
+  static int cache[9] = {-1, -1, -1, -1, -1, -1, -1, -1, -1};
+  if (csize < 1 || csize > 8) return 0;
+  if (cache[csize] >= 0) return cache[csize];
+  if (cudaFuncSetAttribute(sgemm_fused1, cudaFuncAttributeMaxDynamicSharedMemorySize, kFused1Smem) != cudaSuccess)
+    return 0;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(csize * 16));
+  cfg.blockDim = dim3(kFThreads);
+  cfg.dynamicSmemBytes = kFused1Smem;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)csize;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, (void*)sgemm_fused1, &cfg) != cudaSuccess) n = 0;
+  cache[csize] = n;
+  return n;
+}
+
+static cudaError_t sgemm_fused1_rows(const float* A, const float* B, float* C, int64_t N, int64_t K, int64_t r0,
+                                     int64_t mrows, int S, cudaStream_t s) {
+  CUtensorMap tA, tB;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(&tA, A + r0 * K, K, mrows, K * 4, FBK, FBM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tB, B, N, K, N * 4, 32, FBK)) != cudaSuccess) return e;
+  static std::atomic<uint64_t> attr{0};
+  e = once_per_device(attr, [] {
+    return cudaFuncSetAttribute(sgemm_fused1, cudaFuncAttributeMaxDynamicSharedMemorySize, kFused1Smem);
+  });
+  if (e != cudaSuccess) return e;
+  const int mblk = (int)((mrows + FBM - 1) / FBM);
+  const int nblk = (int)((N + G1N - 1) / G1N);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(mblk * nblk * S));
+  cfg.blockDim = dim3(kFThreads);
+  cfg.dynamicSmemBytes = kFused1Smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)S;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  note_launch();
+  return cudaLaunchKernelEx(&cfg, sgemm_fused1, tA, tB, C, N, r0, mrows, nblk, S, (int)((K + FBK - 1) / FBK));
+}
+
+// B already split and K-major (bhi / blo: N x Kp, written by the previous
+// launch on the stream); PDL lets the set-up overlap that launch.
+cudaError_t sgemm_fused_presplit_rows(const float* A, const float* bhi, const float* blo, int64_t Kp, float* C,
+                                      int64_t N, int64_t K, int64_t r0, int64_t mrows, int S, cudaStream_t s) {
+  CUtensorMap tA, tBh, tBl;
+  cudaError_t e;
+  if ((e = encode_tmap_2d_f32(&tA, A + r0 * K, K, mrows, K * 4, FBK, FBM)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tBh, bhi, Kp, N, Kp * 4, FBK, G2N)) != cudaSuccess) return e;
+  if ((e = encode_tmap_2d_f32(&tBl, blo, Kp, N, Kp * 4, FBK, G2N)) != cudaSuccess) return e;
+  static std::atomic<uint64_t> attr{0};
+  e = once_per_device(attr, [] {
+    return cudaFuncSetAttribute(sgemm_fused2, cudaFuncAttributeMaxDynamicSharedMemorySize, kFused2Smem);
+  });
+  if (e != cudaSuccess) return e;
+  const int mblk = (int)((mrows + FBM - 1) / FBM);
+  const int nblk = (int)((N + G2N - 1) / G2N);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(mblk * nblk * S));
+  cfg.blockDim = dim3(kFThreads);
+  cfg.dynamicSmemBytes = kFused2Smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = (unsigned)S;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  note_launch();
+  return cudaLaunchKernelEx(&cfg, sgemm_fused2, tA, tBh, tBl, C, N, r0, mrows, nblk, S, (int)((K + FBK - 1) / FBK));
+}
+
 cudaError_t sgemm_fused_rows(const float* A, const float* B, float* C, int64_t N, int64_t K, int64_t r0,
                              int64_t mrows, int S, cudaStream_t s) {
+  if (fused_variant() >= 2) return sgemm_fused1_rows(A, B, C, N, K, r0, mrows, S, s);
   CUtensorMap tA, tB;
   cudaError_t e;
   if ((e = encode_tmap_2d_f32(&tA, A + r0 * K, K, mrows, K * 4, FBK, FBM)) != cudaSuccess) return e;
