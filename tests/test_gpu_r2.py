@@ -366,3 +366,45 @@ def test_run_repeat_equals_sequential_runs(R, graph, timing):
         ms = sum(st.kernel_ms[d][k] for d in range(2) for k in range(4))
         assert (ms > 0) == timing
         assert st.device_ms > 0
+
+
+_FUSED_SCRIPT = r"""
+import sys, numpy as np
+sys.path.insert(0, {root!r})
+import synthgen
+from oracle import numeric as on
+from paper_conf_icpp_shenvms15_b200 import mm, runner
+M, N, K = {M}, {N}, {K}
+out = {{}}
+for integer in (True, False):
+    A, B = (synthgen.matmul_integer if integer else synthgen.matmul_uniform)(M, K, N)
+    ref = on.sgemm(A, B)
+    with runner.session(mm.MM_APP_SGEMM, [M, N, K, 2, 16, 1], G=1) as s:
+        s.fill(integer=integer)
+        plan = s.plan(1, mm.make_profile(1, [[1000]], [[10 ** 5]], [10 ** 10]))
+        s.run(plan)
+        got = s.collect(plan, 2).reshape(M, N)
+    if integer:
+        assert np.array_equal(got, ref), "integer"
+    else:
+        assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-4, "uniform"
+print("ok")
+"""
+
+
+@pytest.mark.parametrize("variant", ["1", "2", "3"])
+@pytest.mark.parametrize("shape", [(1024, 1024, 1024), (300, 520, 768)])
+def test_sgemm_fused_variants(gpu, variant, shape):
+    """The three small-SGEMM kernels (MM_SGEMM_FUSED = 1 pair tiles, 2 single-SM
+    tiles with in-kernel B transposition, 3 split_bT + single-SM tiles; a
+    fresh process each): integer inputs bit-exact, uniform within 1e-4 of the
+    FP64 oracle, including ragged M and N."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MM_SGEMM_FUSED=variant)
+    M, N, K = shape
+    r = subprocess.run([sys.executable, "-c", _FUSED_SCRIPT.format(root=root, M=M, N=N, K=K)], env=env, cwd=root,
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
