@@ -271,12 +271,13 @@ def test_graph_staged_new_host_buffers(R):
 
 def test_launch_counter_counts_kernels(R):
     """n_launches and mm_kernel_launch_count count kernels, not ops, eagerly
-    and per graph replay: the 3xTF32 SGEMM of 1024 x 1024 x 1024 is ONE fused
-    launch (in-smem operand split + in-cluster split-K reduction), 512 x 4096
-    x 1024 (enough tile pairs, no K split) issues the operand split and the GEMM (2 kernels for
-    one op); STREAM issues one kernel per op."""
+    and per graph replay: the 3xTF32 SGEMM of 1024 x 1024 x 1024 is the B
+    split (split_bT) and ONE fused launch (A split in the kernel, in-cluster
+    split-K reduction); 2048 x 2048 x 1024 (enough tile pairs, no K split)
+    issues the operand split and the GEMM — 2 kernels for one op either way;
+    STREAM issues one kernel per op."""
     mm, runner = R
-    for (M, N, K), want in (((1024, 1024, 1024), 1), ((2048, 2048, 1024), 2)):
+    for (M, N, K), want in (((1024, 1024, 1024), 2), ((2048, 2048, 1024), 2)):
         with runner.session(mm.MM_APP_SGEMM, [M, N, K, 2, 128, 1], G=1) as s:
             s.fill()
             plan = s.plan(mm.MM_SP_SINGLE, _prof(mm, 1, 1))
