@@ -411,9 +411,11 @@ __global__ void __launch_bounds__(kTcThreads, 1)
           tmem_st16(accq + (uint32_t)(32 * s), x);
           asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
           asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-          asm volatile("bar.sync %0, 64;" ::"r"(2 + grp) : "memory");
-        } else {
-          asm volatile("bar.sync %0, 64;" ::"r"(2 + grp) : "memory");
+        }
+        // the row group's two warps meet at ONE barrier instruction (per-warp
+        // aligned barriers reached from two code sites count as divergent)
+        asm volatile("bar.sync %0, 64;" ::"r"(2 + grp) : "memory");
+        if (hf == 1) {
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           float x0[16];
           tmem_ld16(accq + (uint32_t)(32 * s), x0);
