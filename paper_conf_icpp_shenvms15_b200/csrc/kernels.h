@@ -63,7 +63,19 @@ struct Scratch {
   uint64_t b_epoch = 0;
   uint64_t epoch = 1;
   std::vector<uint64_t> panel;   // Cholesky: split tag (epoch, step) per panel slot
+  // Cholesky: the last POTRF launched on this scratch (step, stream, epoch):
+  // it also wrote L_kk's split and packed leaves and counts finished blocks
+  // per 128-row block, so a TRSM of that step on that stream may start early
+  int64_t potrf_k = -1;
+  const void* potrf_stream = nullptr;
+  uint64_t potrf_epoch = 0;
 };
+
+// Packed 128 x 128 leaf blocks of L_kk for the column TRSM (per leaf q, floats):
+//   U[s(s-1)/2 + mb][i][c] = L[c0+32s+c][c0+32mb+i]   s = 1..3, mb < s   at kLtU
+//   D[s][c][c2]            = L[c0+32s+c2][c0+32s+c]   s = 0..3           at kLtD
+//   rd[m]                  = RN(1 / L[c0+m][c0+m])                       at kLtRd
+constexpr int kLtU = 0, kLtD = 6 * 1024, kLtRd = 10 * 1024, kLtFloats = kLtRd + 128;
 
 struct Launch {
   const Kernel* k;          // kernel descriptor (op, params)
@@ -126,6 +138,11 @@ void chol_mark_split(Scratch* scr, int64_t T, int32_t k, const int32_t* tiles, i
 // == 0, 256 <= b <= 4096, else cudaErrorNotSupported); MM_TRSM_COL=0 selects
 // the leaf path.  Its transposed L_kk leaves live after the POTRF flags.
 bool chol_trsm_col_enabled();
+// MM_TRSM_OVERLAP=0: no POTRF -> column TRSM overlap (the TRSM then waits for
+// the whole POTRF and splits L_kk itself)
+bool chol_trsm_overlap_enabled();
+// per-128-row-block finished-block counts of the last POTRF on this scratch
+int* chol_potrf_rowcnt(Scratch* scr, int64_t T, int64_t b);
 size_t chol_trsm_lt_bytes(int64_t b);
 cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32_t* ti, int32_t n, cudaStream_t s,
                           Scratch* scr);

@@ -68,9 +68,7 @@ constexpr int kTcStageBytes = 4 * kTcOpBytes;               // A hi, A lo, B hi,
 //   U[s(s-1)/2 + mb][i][c] = L[c0+32s+c][c0+32mb+i]   s = 1..3, mb < s
 //   D[s][c][c2]            = L[c0+32s+c2][c0+32s+c]   s = 0..3
 //   rd[m]                  = RN(1 / L[c0+m][c0+m])
-constexpr int kLtU = 0, kLtD = 6 * 1024, kLtRd = 10 * 1024;
-constexpr int kLtFloats = kLtRd + kTcLeaf;
-constexpr int kLtBytes = kLtFloats * 4;                     // 41472
+constexpr int kLtBytes = kLtFloats * 4;                     // 41472 (layout: kernels.h)
 constexpr int kStgBytes = kTcRows * 32 * 4;                 // 16 KB: 128 rows x 32 fp32 (SWIZZLE_128B)
 constexpr int kMaxLeaves = 32;                              // b <= 4096
 constexpr int kSmRing = 0, kSmStg = kTcStages * kTcStageBytes, kSmBpre = kSmStg + 3 * kStgBytes;
@@ -103,6 +101,25 @@ __device__ __forceinline__ void twait(uint64_t* b, uint32_t parity) {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     if (t - t0 > 4000000000ull) __trap();
   }
+}
+
+// rowcnt != NULL (launched as a programmatic dependent of the step's POTRF):
+// the rows of leaf q of L_kk, with their split and packed block, are final
+// once POTRF counted all 16 q + 10 of their 32 x 32 blocks
+__device__ __forceinline__ void wait_rows(const int* rowcnt, int q) {
+  if (!rowcnt) return;
+  uint64_t t0 = 0;
+  for (;;) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(rowcnt + q) : "memory");
+    if (v >= 16 * q + 10) break;
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (!t0) t0 = t;
+    else if (t - t0 > 4000000000ull) __trap();
+    __nanosleep(64);
+  }
+  asm volatile("fence.proxy.async.global;" ::: "memory");   // POTRF's generic stores -> our TMA / bulk loads
 }
 
 __device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc, uint32_t acc) {
@@ -168,7 +185,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
     trsm_col(float* __restrict__ A, const float* __restrict__ lt, const __grid_constant__ CUtensorMap tLhi,
              const __grid_constant__ CUtensorMap tLlo, const __grid_constant__ CUtensorMap tSx,
              const __grid_constant__ CUtensorMap tShi, const __grid_constant__ CUtensorMap tSlo,
-             const __grid_constant__ ColJob job, uint64_t* __restrict__ stamps) {
+             const __grid_constant__ ColJob job, const int* __restrict__ rowcnt, uint64_t* __restrict__ stamps) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   // 1024-B aligned (SWIZZLE_64B / 128B atoms), pointer arithmetic on the
   // shared array so the accesses stay LDS/STS
@@ -235,6 +252,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       int it = 0;
       for (int q = 1; q < nleaf; ++q) {
         const int32_t yb = yl + q * kTcLeaf;
+        wait_rows(rowcnt, q);   // L_qj (j < q): row block q of L_kk
         for (int j = 0; j <= q - 1; ++j) {
           const bool ts = j == q - 1;                 // X_{q-1} comes from TMEM
           if (!ts && j == q - 2) twait(&xgl[j], 0);   // X_j of this CTA's leaf j is in global memory
@@ -333,6 +351,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       tma_load_2d(bpre + (idx & 1) * 4096, &tSx, 32 * idx, yx, &bful[idx & 1]);
     };
     if (issuer) {   // LsT of leaf 0
+      wait_rows(rowcnt, 0);
       mbar_expect_tx(&lsb[0], kLtBytes);
       asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                        saddr(LsT)),
@@ -483,6 +502,7 @@ __global__ void __launch_bounds__(kTcThreads, 1)
       if (issuer) {
         pending = q;
         if (q + 1 < nleaf) {
+          wait_rows(rowcnt, q + 1);
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           mbar_expect_tx(&lsb[q + 1], kLtBytes);
           asm volatile(
@@ -578,6 +598,11 @@ static void trsm_stamps_dump(cudaStream_t s, const uint64_t* d, int gx, int gy, 
 
 size_t chol_trsm_lt_bytes(int64_t b) { return (size_t)(b / kTcLeaf) * kLtBytes; }
 
+bool chol_trsm_overlap_enabled() {
+  static const int env = getenv("MM_TRSM_OVERLAP") ? atoi(getenv("MM_TRSM_OVERLAP")) : 1;
+  return env != 0;
+}
+
 bool chol_trsm_col_enabled() {
   static const int env = getenv("MM_TRSM_COL") ? atoi(getenv("MM_TRSM_COL")) : 1;
   return env != 0;
@@ -602,6 +627,12 @@ cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32
   if (e != cudaSuccess) return e;
   if (scr->panel.size() != (size_t)(2 * T)) scr->panel.assign(2 * T, 0);
   const uint64_t tag = (scr->epoch << 20) | (uint64_t)(k + 1);   // = kernels_gemm_tc.cu split_tag
+  // the step's POTRF ran right before on this stream and wrote L_kk's split
+  // and packed leaves itself: overlap it (PDL launch, per-leaf row counts)
+  const bool overlap = chol_trsm_overlap_enabled() && scr->potrf_k == k && scr->potrf_stream == (const void*)s &&
+                       scr->potrf_epoch == scr->epoch;
+  const int* rowcnt = overlap ? chol_potrf_rowcnt(scr, T, b) : nullptr;
+  if (overlap) scr->panel[slot0 + k] = tag;
   if (scr->panel[slot0 + k] != tag) {
     scr->panel[slot0 + k] = tag;
     const int nsplit = 64;
@@ -626,11 +657,21 @@ cudaError_t chol_trsm_col(float* A, int64_t T, int64_t b, int32_t k, const int32
   for (int32_t q0 = 0; q0 < n; q0 += kCholBatch) {
     job.n = std::min<int32_t>(kCholBatch, n - q0);
     for (int32_t q = 0; q < job.n; ++q) job.ti[q] = ti[q0 + q];
-    note_launch();
     uint64_t* stamps = trsm_stamps_buffer(s, (size_t)(b / kTcRows) * job.n * kStampsPerCta);
-    trsm_col<<<dim3((unsigned)(b / kTcRows), (unsigned)job.n), kTcThreads, kTcSmem, s>>>(A, lt, mLhi, mLlo, mSx, mShi,
-                                                                                       mSlo, job, stamps);
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    note_launch();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(b / kTcRows), (unsigned)job.n);
+    cfg.blockDim = dim3(kTcThreads);
+    cfg.dynamicSmemBytes = kTcSmem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = rowcnt ? 1 : 0;
+    if ((e = cudaLaunchKernelEx(&cfg, trsm_col, A, (const float*)lt, mLhi, mLlo, mSx, mShi, mSlo, job, rowcnt,
+                                stamps)) != cudaSuccess)
+      return e;
     if (stamps) trsm_stamps_dump(s, stamps, (int)(b / kTcRows), job.n, k);
   }
   for (int32_t q = 0; q < n; ++q) scr->panel[slot0 + ti[q]] = tag;
