@@ -104,17 +104,21 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
 // kTbAhead rows ahead; levels 1..H-1 keep their 3-row windows in registers
 // (slot = row index mod 3, compile-time because the row loop is unrolled by
 // 3).  Horizontal neighbours come from warp shuffles.  The 4 cells of a lane
-// are updated as two f32x2 pairs (FADD2/FMUL2: same round-to-nearest ops in
+// are updated as two f32x2 pairs (FADD2/FFMA2: same round-to-nearest ops in
 // the oracle's order, half the issue slots).  Rows outside the grid are
 // never stored and halo columns lose one valid column per level and are not
 // stored, so every stored cell went through exactly H applications of the
 // R16 update: bit-identical to H single-step launches.
-constexpr int kTbWarps = 4;                      // warps per CTA
+//
+// One CTA of 12 warps per SM (3 per SM sub-partition: the register-bound
+// residency at ~150 registers); every warp of a CTA runs the same number of
+// steps.  Measured at 8192^2 x 1000 (h = 8): 41.8 ms vs 45.8 ms with three
+// 4-warp CTAs per SM, whose SMs averaged 9.3 of 12 active warps (ncu) — the
+// warps of one sub-partition drifted apart and the last ones ran alone,
+// latency-bound on their level chains.  CTAs of 4 or 6 warps: 45.6 / 46.2 ms;
+// CTA barriers every 6-48 steps: slower.
+constexpr int kTbWarps = 12;                     // warps per CTA (MM_TB_WARPS = 4 | 6 | 12 CTAs of 12 / NW per SM)
 constexpr int kTbAhead = 5;                      // cp.async prefetch distance (rows)
-#ifndef TB_MIN_BLOCKS
-#define TB_MIN_BLOCKS 3
-#endif
-constexpr int kTbMinBlocks = TB_MIN_BLOCKS;       // resident CTAs per SM (4 = 128 registers: spills, measured slower)
 
 template <int H>
 struct TbCfg {
@@ -146,29 +150,32 @@ __device__ __forceinline__ f2 sub2(f2 a, f2 b) {
   return r;
 }
 
-// products as two scalar __fmul_rn: ptxas contracts mul.rn.f32x2 followed by
-// add.rn.f32x2 into FFMA2 (single rounding), which would break R16's order
-__device__ __forceinline__ f2 mul2s(f2 a, float b) {
-  float x, y;
-  upk(a, x, y);
-  return pk(__fmul_rn(x, b), __fmul_rn(y, b));
+// products: ptxas contracts mul.rn.f32x2 followed by add.rn.f32x2 into FFMA2
+// (single rounding), which would break R16's order, and folds a literal -0
+// addend the same way.  fma.rn.f32x2(a, b, z) with z = -0 held in a register
+// that comes from a kernel argument (opaque to ptxas) is RN(a*b + -0) =
+// RN(a*b) for every a, b (an exact zero product keeps its sign, -0 + -0 = -0,
+// +0 + -0 = +0): the R16 product bit for bit, one FFMA2 issue for two cells.
+__device__ __forceinline__ f2 mul2s(f2 a, f2 b, f2 nz) {
+  f2 r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r.v) : "l"(a.v), "l"(b.v), "l"(nz.v));
+  return r;
 }
 
 struct HotCoef2 {
-  float ry1, rx1, rz1, sdc;
-  f2 amb;
+  f2 ry1, rx1, rz1, sdc;
+  f2 amb, nz;
 };
 
 // cell() on two cells at once (R16 order, every op rounded to nearest), with
 // the horizontal sums e + w already formed
-__device__ __forceinline__ f2 cell2h(f2 c, f2 n, f2 s, f2 ew, f2 p, float ry1, float rx1, float rz1, f2 amb,
-                                     float sdc) {
+__device__ __forceinline__ f2 cell2h(f2 c, f2 n, f2 s, f2 ew, f2 p, const HotCoef2& k) {
   const f2 two = add2(c, c);
-  const f2 dv = mul2s(sub2(add2(s, n), two), ry1);
-  const f2 dh = mul2s(sub2(ew, two), rx1);
-  const f2 dz = mul2s(sub2(amb, c), rz1);
+  const f2 dv = mul2s(sub2(add2(s, n), two), k.ry1, k.nz);
+  const f2 dh = mul2s(sub2(ew, two), k.rx1, k.nz);
+  const f2 dz = mul2s(sub2(k.amb, c), k.rz1, k.nz);
   const f2 sum = add2(add2(add2(p, dv), dh), dz);
-  return add2(c, mul2s(sum, sdc));
+  return add2(c, mul2s(sum, k.sdc, k.nz));
 }
 
 // Four cells of a lane as the pairs (x, y), (z, w).  The east + west sums
@@ -179,10 +186,8 @@ __device__ __forceinline__ f2 cell2h(f2 c, f2 n, f2 s, f2 ew, f2 p, float ry1, f
 __device__ __forceinline__ float4 cell4(float4 cu, float4 up, float4 dn, float w, float e, float4 p, const HotCoef2& k) {
   const f2 ewa = pk(__fadd_rn(cu.y, w), __fadd_rn(cu.z, cu.x));
   const f2 ewb = pk(__fadd_rn(cu.w, cu.y), __fadd_rn(e, cu.z));
-  const f2 a = cell2h(pk(cu.x, cu.y), pk(up.x, up.y), pk(dn.x, dn.y), ewa, pk(p.x, p.y), k.ry1, k.rx1, k.rz1, k.amb,
-                      k.sdc);
-  const f2 b = cell2h(pk(cu.z, cu.w), pk(up.z, up.w), pk(dn.z, dn.w), ewb, pk(p.z, p.w), k.ry1, k.rx1, k.rz1, k.amb,
-                      k.sdc);
+  const f2 a = cell2h(pk(cu.x, cu.y), pk(up.x, up.y), pk(dn.x, dn.y), ewa, pk(p.x, p.y), k);
+  const f2 b = cell2h(pk(cu.z, cu.w), pk(up.z, up.w), pk(dn.z, dn.w), ewb, pk(p.z, p.w), k);
   float4 o;
   upk(a, o.x, o.y);
   upk(b, o.z, o.w);
@@ -268,19 +273,22 @@ __device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3], float
     tb_levels<H, PH, true>(W, tr, pr, a, r, k);
 }
 
-template <int H>
-__global__ void __launch_bounds__(32 * kTbWarps, kTbMinBlocks) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
+template <int H, int NW>
+__global__ void __launch_bounds__(32 * NW, 12 / NW) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
                                                              float* __restrict__ tout, int rows, int cols, int r0, int r1,
-                                                             HotCoef kc, int nwx, int SR) {
+                                                             HotCoef kc, int nwx, int SR, float nz) {
   using C = TbCfg<H>;
   extern __shared__ float4 tb_smem[];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int gw = blockIdx.x * kTbWarps + wid;
+  const int gw = blockIdx.x * NW + wid;
   const int wx = gw % nwx, wy = gw / nwx;
   TbArgs<H> a;
   a.tin = tin; a.pw = pw; a.tout = tout; a.rows = rows; a.cols = cols; a.lane = lane;
-  const int64_t y0 = (int64_t)r0 + (int64_t)wy * SR;
-  if (y0 >= r1) return;                           // whole warp exits together
+  // every warp of the CTA runs the same SR + 2H - 1 steps (a strip past r1
+  // or shorter than SR fetches nothing and stores nothing there), so the
+  // CTA barriers below are reached by all of them
+  int64_t y0 = (int64_t)r0 + (int64_t)wy * SR;
+  if (y0 > r1) y0 = r1;
   a.Y0 = (int)y0;
   a.Y1 = a.Y0 + SR < r1 ? a.Y0 + SR : r1;
   const int X0 = wx * C::OW;                      // first output column
@@ -292,8 +300,9 @@ __global__ void __launch_bounds__(32 * kTbWarps, kTbMinBlocks) hotspot_tb(const 
   float4* tr = tb_smem + (size_t)wid * (C::RT + C::RP) * 32;
   float4* pr = tr + C::RT * 32;
   HotCoef2 k;
-  k.ry1 = kc.ry1; k.rx1 = kc.rx1; k.rz1 = kc.rz1; k.sdc = kc.sdc;
+  k.ry1 = pk(kc.ry1, kc.ry1); k.rx1 = pk(kc.rx1, kc.rx1); k.rz1 = pk(kc.rz1, kc.rz1); k.sdc = pk(kc.sdc, kc.sdc);
   k.amb = pk(kc.amb, kc.amb);
+  k.nz = pk(nz, nz);
   float4 W[H > 1 ? H - 1 : 1][3];
 #pragma unroll
   for (int i = 0; i < (H > 1 ? H - 1 : 1); ++i)
@@ -306,7 +315,7 @@ __global__ void __launch_bounds__(32 * kTbWarps, kTbMinBlocks) hotspot_tb(const 
   // prologue: rows rs .. rs + kTbAhead in flight (step r fetches r + kTbAhead)
 #pragma unroll
   for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H>(tr, pr, a, rs + q);
-  const int rb = rs + 1, rend = a.re;
+  const int rb = rs + 1, rend = rb + SR + 2 * H - 1;
   for (int r = rb; r < rend; r += 3) {
     tb_step<H, 0>(W, tr, pr, a, r, k);
     if (r + 1 < rend) tb_step<H, 1>(W, tr, pr, a, r + 1, k);
@@ -315,20 +324,20 @@ __global__ void __launch_bounds__(32 * kTbWarps, kTbMinBlocks) hotspot_tb(const 
   cp_wait<0>();
 }
 
-template <int H>
-cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
+template <int H, int NW>
+cudaError_t launch_tb_nw(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
                       int64_t r1, HotCoef c, cudaStream_t s, int sms) {
   using C = TbCfg<H>;
   if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
-  const size_t smem = (size_t)kTbWarps * (C::RT + C::RP) * 32 * sizeof(float4);
+  const size_t smem = (size_t)NW * (C::RT + C::RP) * 32 * sizeof(float4);
   static std::atomic<uint64_t> attr{0};
   static std::atomic<int> per_sm{0};   // resident CTAs per SM (registers bound it; same on every B200)
   cudaError_t e = once_per_device(attr, [&] {
-    cudaError_t r = cudaFuncSetAttribute(hotspot_tb<H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t r = cudaFuncSetAttribute(hotspot_tb<H, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (r != cudaSuccess) return r;
     int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, hotspot_tb<H>, 32 * kTbWarps, smem) != cudaSuccess || n < 1)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, hotspot_tb<H, NW>, 32 * NW, smem) != cudaSuccess || n < 1)
       n = 1;
     per_sm.store(n);
     return cudaSuccess;
@@ -336,18 +345,30 @@ cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t ro
   if (e != cudaSuccess) return e;
   // exactly one wave of resident warps (a partial second wave left SMs
   // idle); strips at least 8H rows tall (vertical redundancy (2H+1)/SR)
-  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm.load() * kTbWarps;
+  const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm.load() * NW;
   const int64_t nr = r1 - r0;
   int64_t nstrip = (target + nwx - 1) / nwx;
   int64_t SR = (nr + nstrip - 1) / nstrip;
   if (SR < 8 * H) SR = 8 * H;
   nstrip = (nr + SR - 1) / SR;
   const int64_t warps = nwx * nstrip;
-  if (warps + kTbWarps >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
+  if (warps + NW >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   note_launch();
-  hotspot_tb<H><<<(unsigned)((warps + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, smem, s>>>(
-      tin, pw, tout, (int)rows, (int)cols, (int)r0, (int)r1, c, (int)nwx, (int)SR);
+  hotspot_tb<H, NW><<<(unsigned)((warps + NW - 1) / NW), 32 * NW, smem, s>>>(
+      tin, pw, tout, (int)rows, (int)cols, (int)r0, (int)r1, c, (int)nwx, (int)SR, -0.0f);
   return cudaGetLastError();
+}
+
+template <int H>
+cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
+                      int64_t r1, HotCoef c, cudaStream_t s, int sms) {
+  static const int nw = [] {
+    const char* e = getenv("MM_TB_WARPS");
+    return e ? atoi(e) : kTbWarps;
+  }();
+  if (nw == 4) return launch_tb_nw<H, 4>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+  if (nw == 6) return launch_tb_nw<H, 6>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+  return launch_tb_nw<H, 12>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
 }
 
 // Generic shapes: one thread per cell.
