@@ -117,13 +117,14 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
 // warps of one sub-partition drifted apart and the last ones ran alone,
 // latency-bound on their level chains.  CTAs of 4 or 6 warps: 45.6 / 46.2 ms;
 // CTA barriers every 6-48 steps: slower.
-constexpr int kTbWarps = 12;                     // warps per CTA (MM_TB_WARPS = 4 | 6 | 12 CTAs of 12 / NW per SM)
+constexpr int kTbWarps = 12;                     // warps per CTA
 constexpr int kTbAhead = 5;                      // cp.async prefetch distance (rows)
 
-template <int H>
+template <int H, int CL>
 struct TbCfg {
-  static constexpr int HC = 4 * ((H + 3) / 4);   // halo columns per side (float4-aligned)
-  static constexpr int OW = 128 - 2 * HC;        // output columns per warp
+  static constexpr int LW = 4 * CL;              // columns per lane (CL float4 groups)
+  static constexpr int HC = LW * ((H + LW - 1) / LW);  // halo columns per side (whole lanes)
+  static constexpr int OW = 32 * LW - 2 * HC;    // output columns per warp
   // ring rows (powers of 2): T rows r-2 .. r+ahead (level 1 only), P rows
   // r-H .. r+ahead (every level)
   static constexpr int RT = (kTbAhead + 3) <= 8 ? 8 : 16;
@@ -202,7 +203,6 @@ __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_grou
 template <int N>
 __device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-template <int H>
 struct TbArgs {
   const float* tin;
   const float* pw;
@@ -212,14 +212,18 @@ struct TbArgs {
   int lane;
 };
 
-// issue the copies of level-0 row q (T and P) into the ring, one commit group
-template <int H>
-__device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs<H>& a, int q) {
-  constexpr int RT = TbCfg<H>::RT, RP = TbCfg<H>::RP;
+// issue the copies of level-0 row q (T and P) into the ring, one commit group;
+// ring slot layout [group j][lane] so the lanes' 16-B reads are contiguous
+template <int H, int CL>
+__device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs& a, int q) {
+  constexpr int RT = TbCfg<H, CL>::RT, RP = TbCfg<H, CL>::RP;
   if (q < a.re && q >= 0 && q < a.rows && a.inx) {
     const int64_t off = (int64_t)q * a.cols + a.x0;
-    cp16(tr + (q & (RT - 1)) * 32 + a.lane, a.tin + off);
-    cp16(pr + (q & (RP - 1)) * 32 + a.lane, a.pw + off);
+#pragma unroll
+    for (int j = 0; j < CL; ++j) {
+      cp16(tr + ((q & (RT - 1)) * CL + j) * 32 + a.lane, a.tin + off + 4 * j);
+      cp16(pr + ((q & (RP - 1)) * CL + j) * 32 + a.lane, a.pw + off + 4 * j);
+    }
   }
   cp_commit();
 }
@@ -227,148 +231,154 @@ __device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs<H>
 // One step r: level s = 1..H computes row r - s.  EDGE = some row of the
 // step is the grid's first or last row (warp-uniform, so interior steps run
 // without the boundary selects).
-template <int H, int PH, bool EDGE>
-__device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3], const float4* tr, const float4* pr,
-                                          const TbArgs<H>& a, int r, const HotCoef2& k) {
-  constexpr int RT = TbCfg<H>::RT, RP = TbCfg<H>::RP;
+template <int H, int CL, int PH, bool EDGE>
+__device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
+                                          const TbArgs& a, int r, const HotCoef2& k) {
+  constexpr int RT = TbCfg<H, CL>::RT, RP = TbCfg<H, CL>::RP;
 #pragma unroll
   for (int s = 1; s <= H; ++s) {
     const int y = r - s;
-    float4 cu, up, dn;
-    if (s == 1) {                                 // level 0 rows from the ring
-      cu = tr[((r - 1) & (RT - 1)) * 32 + a.lane];
-      up = tr[((r - 2) & (RT - 1)) * 32 + a.lane];
-      dn = tr[(r & (RT - 1)) * 32 + a.lane];
-    } else {
-      cu = W[s - 2][((PH - s) % 3 + 3) % 3];
-      up = W[s - 2][((PH - s - 1) % 3 + 3) % 3];
-      dn = W[s - 2][((PH - s + 1) % 3 + 3) % 3];
+    float4 cu[CL], up[CL], dn[CL], p[CL];
+#pragma unroll
+    for (int j = 0; j < CL; ++j) {
+      if (s == 1) {                               // level 0 rows from the ring
+        cu[j] = tr[(((r - 1) & (RT - 1)) * CL + j) * 32 + a.lane];
+        up[j] = tr[(((r - 2) & (RT - 1)) * CL + j) * 32 + a.lane];
+        dn[j] = tr[((r & (RT - 1)) * CL + j) * 32 + a.lane];
+      } else {
+        cu[j] = W[s - 2][((PH - s) % 3 + 3) % 3][j];
+        up[j] = W[s - 2][((PH - s - 1) % 3 + 3) % 3][j];
+        dn[j] = W[s - 2][((PH - s + 1) % 3 + 3) % 3][j];
+      }
+      if (EDGE) {
+        if (y <= 0) up[j] = cu[j];                // chip edge: neighbour = the cell itself
+        if (y + 1 >= a.rows) dn[j] = cu[j];
+      }
+      p[j] = pr[(((r - s) & (RP - 1)) * CL + j) * 32 + a.lane];
     }
-    if (EDGE) {
-      if (y <= 0) up = cu;                        // chip edge: neighbour = the cell itself
-      if (y + 1 >= a.rows) dn = cu;
-    }
-    const float4 p = pr[((r - s) & (RP - 1)) * 32 + a.lane];
-    float w = __shfl_up_sync(0xffffffffu, cu.w, 1);
-    float e = __shfl_down_sync(0xffffffffu, cu.x, 1);
-    if (a.wedge) w = cu.x;
-    if (a.eedge) e = cu.w;
-    const float4 o = cell4(cu, up, dn, w, e, p, k);
-    if (s < H) {
-      W[s - 1][((PH - s) % 3 + 3) % 3] = o;
-    } else if (a.store_x && y >= a.Y0 && y < a.Y1) {
-      __stcs(reinterpret_cast<float4*>(a.tout + (int64_t)y * a.cols + a.x0), o);
+    float w = __shfl_up_sync(0xffffffffu, cu[CL - 1].w, 1);
+    float e = __shfl_down_sync(0xffffffffu, cu[0].x, 1);
+    if (a.wedge) w = cu[0].x;
+    if (a.eedge) e = cu[CL - 1].w;
+#pragma unroll
+    for (int j = 0; j < CL; ++j) {
+      const float wj = j > 0 ? cu[j - 1].w : w;
+      const float ej = j + 1 < CL ? cu[j + 1].x : e;
+      const float4 o = cell4(cu[j], up[j], dn[j], wj, ej, p[j], k);
+      if (s < H) {
+        W[s - 1][((PH - s) % 3 + 3) % 3][j] = o;
+      } else if (a.store_x && y >= a.Y0 && y < a.Y1) {
+        __stcs(reinterpret_cast<float4*>(a.tout + (int64_t)y * a.cols + a.x0 + 4 * j), o);
+      }
     }
   }
 }
 
-template <int H, int PH>
-__device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3], float4* tr, float4* pr, const TbArgs<H>& a,
-                                        int r, const HotCoef2& k) {
-  tb_fetch<H>(tr, pr, a, r + kTbAhead);
+template <int H, int CL, int PH>
+__device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], float4* tr, float4* pr,
+                                        const TbArgs& a, int r, const HotCoef2& k) {
+  tb_fetch<H, CL>(tr, pr, a, r + kTbAhead);
   cp_wait<kTbAhead>();                            // rows <= r landed (each lane reads only its own copies)
   if (r - H - 1 >= 0 && r + 1 < a.rows)
-    tb_levels<H, PH, false>(W, tr, pr, a, r, k);
+    tb_levels<H, CL, PH, false>(W, tr, pr, a, r, k);
   else
-    tb_levels<H, PH, true>(W, tr, pr, a, r, k);
+    tb_levels<H, CL, PH, true>(W, tr, pr, a, r, k);
 }
 
-template <int H, int NW>
-__global__ void __launch_bounds__(32 * NW, 12 / NW) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
-                                                             float* __restrict__ tout, int rows, int cols, int r0, int r1,
-                                                             HotCoef kc, int nwx, int SR, float nz) {
-  using C = TbCfg<H>;
+template <int H, int CL, int NW>
+__global__ void __launch_bounds__(32 * NW, 1) hotspot_tb(const float* __restrict__ tin, const float* __restrict__ pw,
+                                                        float* __restrict__ tout, int rows, int cols, int r0, int r1,
+                                                        HotCoef kc, int nwx, int SR, float nz) {
+  using C = TbCfg<H, CL>;
   extern __shared__ float4 tb_smem[];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int gw = blockIdx.x * NW + wid;
   const int wx = gw % nwx, wy = gw / nwx;
-  TbArgs<H> a;
+  TbArgs a;
   a.tin = tin; a.pw = pw; a.tout = tout; a.rows = rows; a.cols = cols; a.lane = lane;
   // every warp of the CTA runs the same SR + 2H - 1 steps (a strip past r1
-  // or shorter than SR fetches nothing and stores nothing there), so the
-  // CTA barriers below are reached by all of them
+  // or shorter than SR fetches nothing and stores nothing there)
   int64_t y0 = (int64_t)r0 + (int64_t)wy * SR;
   if (y0 > r1) y0 = r1;
   a.Y0 = (int)y0;
   a.Y1 = a.Y0 + SR < r1 ? a.Y0 + SR : r1;
   const int X0 = wx * C::OW;                      // first output column
-  a.x0 = X0 - C::HC + 4 * lane;                   // this lane's 4 columns
-  a.inx = a.x0 >= 0 && a.x0 < cols;
+  a.x0 = X0 - C::HC + C::LW * lane;               // this lane's LW columns
+  a.inx = a.x0 >= 0 && a.x0 < cols;               // cols % LW == 0: all or none of them
   a.store_x = a.inx && a.x0 >= X0 && a.x0 < X0 + C::OW;
   a.wedge = a.x0 == 0;
-  a.eedge = a.x0 + 4 == cols;
-  float4* tr = tb_smem + (size_t)wid * (C::RT + C::RP) * 32;
-  float4* pr = tr + C::RT * 32;
+  a.eedge = a.x0 + C::LW == cols;
+  float4* tr = tb_smem + (size_t)wid * (C::RT + C::RP) * CL * 32;
+  float4* pr = tr + C::RT * CL * 32;
   HotCoef2 k;
   k.ry1 = pk(kc.ry1, kc.ry1); k.rx1 = pk(kc.rx1, kc.rx1); k.rz1 = pk(kc.rz1, kc.rz1); k.sdc = pk(kc.sdc, kc.sdc);
   k.amb = pk(kc.amb, kc.amb);
   k.nz = pk(nz, nz);
-  float4 W[H > 1 ? H - 1 : 1][3];
+  float4 W[H > 1 ? H - 1 : 1][3][CL];
 #pragma unroll
   for (int i = 0; i < (H > 1 ? H - 1 : 1); ++i)
 #pragma unroll
-    for (int j = 0; j < 3; ++j) W[i][j] = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int j = 0; j < 3; ++j)
+#pragma unroll
+      for (int g = 0; g < CL; ++g) W[i][j][g] = make_float4(0.f, 0.f, 0.f, 0.f);
   // level-0 rows [rs, re) = [Y0 - H, Y1 + H); at step r level s computes row
   // r - s, so steps r in [rs + 1, re) end with level H row Y1 - 1
   const int rs = a.Y0 - H;
   a.re = a.Y1 + H;
   // prologue: rows rs .. rs + kTbAhead in flight (step r fetches r + kTbAhead)
 #pragma unroll
-  for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H>(tr, pr, a, rs + q);
+  for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H, CL>(tr, pr, a, rs + q);
   const int rb = rs + 1, rend = rb + SR + 2 * H - 1;
   for (int r = rb; r < rend; r += 3) {
-    tb_step<H, 0>(W, tr, pr, a, r, k);
-    if (r + 1 < rend) tb_step<H, 1>(W, tr, pr, a, r + 1, k);
-    if (r + 2 < rend) tb_step<H, 2>(W, tr, pr, a, r + 2, k);
+    tb_step<H, CL, 0>(W, tr, pr, a, r, k);
+    if (r + 1 < rend) tb_step<H, CL, 1>(W, tr, pr, a, r + 1, k);
+    if (r + 2 < rend) tb_step<H, CL, 2>(W, tr, pr, a, r + 2, k);
   }
   cp_wait<0>();
 }
 
-template <int H, int NW>
+template <int H, int CL, int NW>
 cudaError_t launch_tb_nw(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
-                      int64_t r1, HotCoef c, cudaStream_t s, int sms) {
-  using C = TbCfg<H>;
+                         int64_t r1, HotCoef c, cudaStream_t s, int sms) {
+  using C = TbCfg<H, CL>;
   if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
-  const size_t smem = (size_t)NW * (C::RT + C::RP) * 32 * sizeof(float4);
+  const size_t smem = (size_t)NW * (C::RT + C::RP) * CL * 32 * sizeof(float4);
   static std::atomic<uint64_t> attr{0};
   static std::atomic<int> per_sm{0};   // resident CTAs per SM (registers bound it; same on every B200)
   cudaError_t e = once_per_device(attr, [&] {
-    cudaError_t r = cudaFuncSetAttribute(hotspot_tb<H, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t r = cudaFuncSetAttribute(hotspot_tb<H, CL, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (r != cudaSuccess) return r;
     int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, hotspot_tb<H, NW>, 32 * NW, smem) != cudaSuccess || n < 1)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, hotspot_tb<H, CL, NW>, 32 * NW, smem) != cudaSuccess || n < 1)
       n = 1;
     per_sm.store(n);
     return cudaSuccess;
   });
   if (e != cudaSuccess) return e;
-  // exactly one wave of resident warps (a partial second wave left SMs
+  // at most one wave of resident warps (a partial second wave left SMs
   // idle); strips at least 8H rows tall (vertical redundancy (2H+1)/SR)
   const int64_t target = (int64_t)(sms > 0 ? sms : 148) * per_sm.load() * NW;
   const int64_t nr = r1 - r0;
-  int64_t nstrip = (target + nwx - 1) / nwx;
+  int64_t nstrip = target / nwx > 1 ? target / nwx : 1;
   int64_t SR = (nr + nstrip - 1) / nstrip;
   if (SR < 8 * H) SR = 8 * H;
   nstrip = (nr + SR - 1) / SR;
   const int64_t warps = nwx * nstrip;
   if (warps + NW >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   note_launch();
-  hotspot_tb<H, NW><<<(unsigned)((warps + NW - 1) / NW), 32 * NW, smem, s>>>(
+  hotspot_tb<H, CL, NW><<<(unsigned)((warps + NW - 1) / NW), 32 * NW, smem, s>>>(
       tin, pw, tout, (int)rows, (int)cols, (int)r0, (int)r1, c, (int)nwx, (int)SR, -0.0f);
   return cudaGetLastError();
 }
 
+// CL = 2 (256-column warp tiles, half the halo share, 246 registers, one
+// 8-warp CTA per SM) measured 46.2 ms vs 41.8 ms for CL = 1 at 8192^2 x 1000:
+// two warps per sub-partition do not hide the level chains' latency.
 template <int H>
 cudaError_t launch_tb(const float* tin, const float* pw, float* tout, int64_t rows, int64_t cols, int64_t r0,
                       int64_t r1, HotCoef c, cudaStream_t s, int sms) {
-  static const int nw = [] {
-    const char* e = getenv("MM_TB_WARPS");
-    return e ? atoi(e) : kTbWarps;
-  }();
-  if (nw == 4) return launch_tb_nw<H, 4>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
-  if (nw == 6) return launch_tb_nw<H, 6>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
-  return launch_tb_nw<H, 12>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
+  return launch_tb_nw<H, 1, kTbWarps>(tin, pw, tout, rows, cols, r0, r1, c, s, sms);
 }
 
 // Generic shapes: one thread per cell.
