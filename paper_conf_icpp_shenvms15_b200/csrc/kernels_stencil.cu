@@ -118,17 +118,24 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
 // latency-bound on their level chains.  CTAs of 4 or 6 warps: 45.6 / 46.2 ms;
 // CTA barriers every 6-48 steps: slower.
 constexpr int kTbWarps = 12;                     // warps per CTA
-constexpr int kTbAhead = 5;                      // cp.async prefetch distance (rows)
+constexpr int kTbAhead = 3;                      // cp.async prefetch distance (rows, beyond a 3-step group)
 
+// Level-0 rings in shared memory, [row slot][group j][lane] so the lanes'
+// 16-B reads are contiguous.  T rows r-2 .. r+ahead+2 (level 1 only) in RT
+// slots, P rows r-H .. r+ahead+2 (every level) in RP slots.  Each ring
+// sits M slots above the start of its array, and a row whose slot is among
+// the ring's last M is also written R slots lower (M = 2 for T, H for P), so
+// the rows a step reads are contiguous at fixed offsets below one per-step
+// base (array slot(r) + M): no per-level index arithmetic.
 template <int H, int CL>
 struct TbCfg {
   static constexpr int LW = 4 * CL;              // columns per lane (CL float4 groups)
   static constexpr int HC = LW * ((H + LW - 1) / LW);  // halo columns per side (whole lanes)
   static constexpr int OW = 32 * LW - 2 * HC;    // output columns per warp
-  // ring rows (powers of 2): T rows r-2 .. r+ahead (level 1 only), P rows
-  // r-H .. r+ahead (every level)
-  static constexpr int RT = (kTbAhead + 3) <= 8 ? 8 : 16;
-  static constexpr int RP = (H + kTbAhead + 1) <= 8 ? 8 : 16;
+  static constexpr int RT = 8, MT = 2;
+  static constexpr int RP = 16, MP = H;
+  static_assert(kTbAhead + 5 <= RT && H + kTbAhead + 3 <= RP, "ring capacity");
+  static constexpr int ROWS = RT + MT + RP + MP; // float4 rows of 32 x CL per warp
 };
 
 struct f2 {
@@ -195,46 +202,59 @@ __device__ __forceinline__ float4 cell4(float4 cu, float4 up, float4 dn, float w
   return o;
 }
 
-__device__ __forceinline__ void cp16(float4* dst, const float* src) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src) : "memory");
-}
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+// Per-lane state of a warp's strip.  The global row pointers advance by one
+// row per fetch and the store pointer by one row per step, so neither the
+// fetches nor the stores recompute 64-bit addresses.
 struct TbArgs {
-  const float* tin;
-  const float* pw;
-  float* tout;
-  int rows, cols, x0, Y0, Y1, re;   // 32-bit: rows, cols < 2^31 (checked at launch)
-  bool inx, store_x, wedge, eedge;  // lane in the grid; lane stores; chip-edge lanes
-  int lane;
+  const char* gT;                   // T and P bytes of the next row to fetch (lane's columns)
+  const char* gP;
+  float* so;                        // output row r - H of the current step (lane's columns)
+  int64_t rowB;                     // row stride in bytes
+  uint32_t trs, prs;                // shared addresses of the T / P arrays (+ lane)
+  int rows, cols;                   // 32-bit: rows, cols < 2^31 (checked at launch)
+  int qlo, qn;                      // rows q in [qlo, qlo + qn) are fetched (empty if the lane is off the grid)
+  int sr0, sn;                      // step r stores row r - H iff r - sr0 in [0, sn)
+  int eh;                           // step r has no grid-edge row iff r - H - 1 in [0, eh)
+  bool wedge, eedge;                // chip-edge lanes
 };
 
-// issue the copies of level-0 row q (T and P) into the ring, one commit group;
-// ring slot layout [group j][lane] so the lanes' 16-B reads are contiguous
+__device__ __forceinline__ void cp16s(uint32_t dst, const char* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+
+// issue the copies of level-0 row q (T and P) into the rings (and their
+// mirrors), one commit group; rows are fetched in order, one per call
 template <int H, int CL>
-__device__ __forceinline__ void tb_fetch(float4* tr, float4* pr, const TbArgs& a, int q) {
-  constexpr int RT = TbCfg<H, CL>::RT, RP = TbCfg<H, CL>::RP;
-  if (q < a.re && q >= 0 && q < a.rows && a.inx) {
-    const int64_t off = (int64_t)q * a.cols + a.x0;
+__device__ __forceinline__ void tb_fetch(TbArgs& a, int q) {
+  using C = TbCfg<H, CL>;
+  constexpr uint32_t SLOT = CL * 32 * 16;         // bytes per ring slot
+  if ((unsigned)(q - a.qlo) < (unsigned)a.qn) {
+    const int st = q & (C::RT - 1), sp = q & (C::RP - 1);
+    const uint32_t dt = a.trs + (uint32_t)(st + C::MT) * SLOT, dp = a.prs + (uint32_t)(sp + C::MP) * SLOT;
 #pragma unroll
     for (int j = 0; j < CL; ++j) {
-      cp16(tr + ((q & (RT - 1)) * CL + j) * 32 + a.lane, a.tin + off + 4 * j);
-      cp16(pr + ((q & (RP - 1)) * CL + j) * 32 + a.lane, a.pw + off + 4 * j);
+      cp16s(dt + j * 512, a.gT + 16 * j);
+      cp16s(dp + j * 512, a.gP + 16 * j);
+      if (st >= C::RT - C::MT) cp16s(dt - C::RT * SLOT + j * 512, a.gT + 16 * j);
+      if (sp >= C::RP - C::MP) cp16s(dp - C::RP * SLOT + j * 512, a.gP + 16 * j);
     }
   }
   cp_commit();
+  a.gT += a.rowB;
+  a.gP += a.rowB;
 }
 
 // One step r: level s = 1..H computes row r - s.  EDGE = some row of the
-// step is the grid's first or last row (warp-uniform, so interior steps run
-// without the boundary selects).
-template <int H, int CL, int PH, bool EDGE>
-__device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
+// step is the grid's first or last row; CE = the warp holds the chip's first
+// or last column (both warp-uniform, so interior steps of interior warps run
+// without boundary selects).  tb = T row r, pb = P row r (ring bases).
+template <int H, int CL, int PH, bool EDGE, bool CE>
+__device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tb, const float4* pb,
                                           const TbArgs& a, int r, const HotCoef2& k) {
-  constexpr int RT = TbCfg<H, CL>::RT, RP = TbCfg<H, CL>::RP;
 #pragma unroll
   for (int s = 1; s <= H; ++s) {
     const int y = r - s;
@@ -242,9 +262,9 @@ __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL],
 #pragma unroll
     for (int j = 0; j < CL; ++j) {
       if (s == 1) {                               // level 0 rows from the ring
-        cu[j] = tr[(((r - 1) & (RT - 1)) * CL + j) * 32 + a.lane];
-        up[j] = tr[(((r - 2) & (RT - 1)) * CL + j) * 32 + a.lane];
-        dn[j] = tr[((r & (RT - 1)) * CL + j) * 32 + a.lane];
+        cu[j] = tb[(j - CL) * 32];
+        up[j] = tb[(j - 2 * CL) * 32];
+        dn[j] = tb[j * 32];
       } else {
         cu[j] = W[s - 2][((PH - s) % 3 + 3) % 3][j];
         up[j] = W[s - 2][((PH - s - 1) % 3 + 3) % 3][j];
@@ -254,12 +274,14 @@ __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL],
         if (y <= 0) up[j] = cu[j];                // chip edge: neighbour = the cell itself
         if (y + 1 >= a.rows) dn[j] = cu[j];
       }
-      p[j] = pr[(((r - s) & (RP - 1)) * CL + j) * 32 + a.lane];
+      p[j] = pb[(j - s * CL) * 32];
     }
     float w = __shfl_up_sync(0xffffffffu, cu[CL - 1].w, 1);
     float e = __shfl_down_sync(0xffffffffu, cu[0].x, 1);
-    if (a.wedge) w = cu[0].x;
-    if (a.eedge) e = cu[CL - 1].w;
+    if (CE) {
+      if (a.wedge) w = cu[0].x;
+      if (a.eedge) e = cu[CL - 1].w;
+    }
 #pragma unroll
     for (int j = 0; j < CL; ++j) {
       const float wj = j > 0 ? cu[j - 1].w : w;
@@ -267,22 +289,47 @@ __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL],
       const float4 o = cell4(cu[j], up[j], dn[j], wj, ej, p[j], k);
       if (s < H) {
         W[s - 1][((PH - s) % 3 + 3) % 3][j] = o;
-      } else if (a.store_x && y >= a.Y0 && y < a.Y1) {
-        __stcs(reinterpret_cast<float4*>(a.tout + (int64_t)y * a.cols + a.x0 + 4 * j), o);
+      } else if ((unsigned)(r - a.sr0) < (unsigned)a.sn) {
+        __stcs(reinterpret_cast<float4*>(a.so) + j, o);
       }
     }
   }
 }
 
-template <int H, int CL, int PH>
-__device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], float4* tr, float4* pr,
-                                        const TbArgs& a, int r, const HotCoef2& k) {
-  tb_fetch<H, CL>(tr, pr, a, r + kTbAhead);
-  cp_wait<kTbAhead>();                            // rows <= r landed (each lane reads only its own copies)
-  if (r - H - 1 >= 0 && r + 1 < a.rows)
-    tb_levels<H, CL, PH, false>(W, tr, pr, a, r, k);
+// The first step of each unrolled 3-step group fetches rows r + kTbAhead ..
+// r + kTbAhead + 2 and waits for rows <= r + 2, so the other two steps carry
+// no cp.async instructions (asm volatile, memory clobber) that would keep
+// ptxas from interleaving the steps' level chains (measured: 40.8 vs 41.6 ms
+// with a fetch + wait in every step).
+template <int H, int CL, int PH, bool CE>
+__device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
+                                        TbArgs& a, int r, const HotCoef2& k) {
+  using C = TbCfg<H, CL>;
+  if (PH == 0) {
+    tb_fetch<H, CL>(a, r + kTbAhead);
+    tb_fetch<H, CL>(a, r + kTbAhead + 1);
+    tb_fetch<H, CL>(a, r + kTbAhead + 2);
+    cp_wait<kTbAhead>();                          // rows <= r + 2 landed (each lane reads only its own copies)
+  }
+  const float4* tb = tr + ((r & (C::RT - 1)) + C::MT) * CL * 32;
+  const float4* pb = pr + ((r & (C::RP - 1)) + C::MP) * CL * 32;
+  if ((unsigned)(r - H - 1) < (unsigned)a.eh)
+    tb_levels<H, CL, PH, false, CE>(W, tb, pb, a, r, k);
   else
-    tb_levels<H, CL, PH, true>(W, tr, pr, a, r, k);
+    tb_levels<H, CL, PH, true, CE>(W, tb, pb, a, r, k);
+  a.so += a.cols;
+}
+
+// steps r = rb, rb + 1, ... in whole 3-step groups (steps past the strip
+// fetch and store nothing)
+template <int H, int CL, bool CE>
+__device__ __forceinline__ void tb_run(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
+                                       TbArgs& a, int rb, int ngroups, const HotCoef2& k) {
+  for (int g = 0, r = rb; g < ngroups; ++g, r += 3) {
+    tb_step<H, CL, 0, CE>(W, tr, pr, a, r, k);
+    tb_step<H, CL, 1, CE>(W, tr, pr, a, r + 1, k);
+    tb_step<H, CL, 2, CE>(W, tr, pr, a, r + 2, k);
+  }
 }
 
 template <int H, int CL, int NW>
@@ -294,22 +341,39 @@ __global__ void __launch_bounds__(32 * NW, 1) hotspot_tb(const float* __restrict
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int gw = blockIdx.x * NW + wid;
   const int wx = gw % nwx, wy = gw / nwx;
-  TbArgs a;
-  a.tin = tin; a.pw = pw; a.tout = tout; a.rows = rows; a.cols = cols; a.lane = lane;
-  // every warp of the CTA runs the same SR + 2H - 1 steps (a strip past r1
+  // every warp of the CTA runs the same number of steps (a strip past r1
   // or shorter than SR fetches nothing and stores nothing there)
-  int64_t y0 = (int64_t)r0 + (int64_t)wy * SR;
-  if (y0 > r1) y0 = r1;
-  a.Y0 = (int)y0;
-  a.Y1 = a.Y0 + SR < r1 ? a.Y0 + SR : r1;
+  int64_t y0l = (int64_t)r0 + (int64_t)wy * SR;
+  if (y0l > r1) y0l = r1;
+  const int Y0 = (int)y0l;
+  const int Y1 = Y0 + SR < r1 ? Y0 + SR : r1;
   const int X0 = wx * C::OW;                      // first output column
-  a.x0 = X0 - C::HC + C::LW * lane;               // this lane's LW columns
-  a.inx = a.x0 >= 0 && a.x0 < cols;               // cols % LW == 0: all or none of them
-  a.store_x = a.inx && a.x0 >= X0 && a.x0 < X0 + C::OW;
-  a.wedge = a.x0 == 0;
-  a.eedge = a.x0 + C::LW == cols;
-  float4* tr = tb_smem + (size_t)wid * (C::RT + C::RP) * CL * 32;
-  float4* pr = tr + C::RT * CL * 32;
+  const int x0 = X0 - C::HC + C::LW * lane;       // this lane's LW columns
+  const bool inx = x0 >= 0 && x0 < cols;          // cols % LW == 0: all or none of them
+  const bool store_x = inx && x0 >= X0 && x0 < X0 + C::OW;
+  // level-0 rows [rs, re) = [Y0 - H, Y1 + H); at step r level s computes row
+  // r - s, so steps r in [rs + 1, re) end with level H row Y1 - 1
+  const int rs = Y0 - H, re = Y1 + H;
+  const int rb = rs + 1;
+  TbArgs a;
+  a.rows = rows;
+  a.cols = cols;
+  a.rowB = (int64_t)cols * 4;
+  a.gT = reinterpret_cast<const char*>(tin + (int64_t)rs * cols + x0);
+  a.gP = reinterpret_cast<const char*>(pw + (int64_t)rs * cols + x0);
+  a.so = tout + (int64_t)(rb - H) * cols + x0;
+  a.qlo = rs > 0 ? rs : 0;
+  const int qhi = re < rows ? re : rows;
+  a.qn = inx && qhi > a.qlo ? qhi - a.qlo : 0;
+  a.sr0 = Y0 + H;
+  a.sn = store_x ? Y1 - Y0 : 0;
+  a.eh = rows - H - 2 > 0 ? rows - H - 2 : 0;
+  a.wedge = x0 == 0;
+  a.eedge = x0 + C::LW == cols;
+  const float4* tr = tb_smem + (size_t)wid * C::ROWS * CL * 32 + lane;
+  const float4* pr = tr + (C::RT + C::MT) * CL * 32;
+  a.trs = (uint32_t)__cvta_generic_to_shared(tr);
+  a.prs = (uint32_t)__cvta_generic_to_shared(pr);
   HotCoef2 k;
   k.ry1 = pk(kc.ry1, kc.ry1); k.rx1 = pk(kc.rx1, kc.rx1); k.rz1 = pk(kc.rz1, kc.rz1); k.sdc = pk(kc.sdc, kc.sdc);
   k.amb = pk(kc.amb, kc.amb);
@@ -321,19 +385,15 @@ __global__ void __launch_bounds__(32 * NW, 1) hotspot_tb(const float* __restrict
     for (int j = 0; j < 3; ++j)
 #pragma unroll
       for (int g = 0; g < CL; ++g) W[i][j][g] = make_float4(0.f, 0.f, 0.f, 0.f);
-  // level-0 rows [rs, re) = [Y0 - H, Y1 + H); at step r level s computes row
-  // r - s, so steps r in [rs + 1, re) end with level H row Y1 - 1
-  const int rs = a.Y0 - H;
-  a.re = a.Y1 + H;
-  // prologue: rows rs .. rs + kTbAhead in flight (step r fetches r + kTbAhead)
+  // prologue: rows rs .. rs + kTbAhead in flight (the group at step r
+  // fetches r + kTbAhead ..)
 #pragma unroll
-  for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H, CL>(tr, pr, a, rs + q);
-  const int rb = rs + 1, rend = rb + SR + 2 * H - 1;
-  for (int r = rb; r < rend; r += 3) {
-    tb_step<H, CL, 0>(W, tr, pr, a, r, k);
-    if (r + 1 < rend) tb_step<H, CL, 1>(W, tr, pr, a, r + 1, k);
-    if (r + 2 < rend) tb_step<H, CL, 2>(W, tr, pr, a, r + 2, k);
-  }
+  for (int q = 0; q <= kTbAhead; ++q) tb_fetch<H, CL>(a, rs + q);
+  const int ngroups = (SR + 2 * H - 1 + 2) / 3;
+  if (__any_sync(0xffffffffu, a.wedge || a.eedge))
+    tb_run<H, CL, true>(W, tr, pr, a, rb, ngroups, k);
+  else
+    tb_run<H, CL, false>(W, tr, pr, a, rb, ngroups, k);
   cp_wait<0>();
 }
 
@@ -343,7 +403,7 @@ cudaError_t launch_tb_nw(const float* tin, const float* pw, float* tout, int64_t
   using C = TbCfg<H, CL>;
   if (rows + 16 >= (int64_t)INT32_MAX || cols >= (int64_t)INT32_MAX) return cudaErrorInvalidValue;
   const int64_t nwx = (cols + C::OW - 1) / C::OW;
-  const size_t smem = (size_t)NW * (C::RT + C::RP) * CL * 32 * sizeof(float4);
+  const size_t smem = (size_t)NW * C::ROWS * CL * 32 * sizeof(float4);
   static std::atomic<uint64_t> attr{0};
   static std::atomic<int> per_sm{0};   // resident CTAs per SM (registers bound it; same on every B200)
   cudaError_t e = once_per_device(attr, [&] {
