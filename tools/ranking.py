@@ -47,8 +47,12 @@ APPS = [
 # SM budgets per logical device (0 = the rest of the GPU).  HET-k (SURVEY
 # §8(f) f2): one fast device + m slow ones, the paper's GPU + CPU-worker mix
 # (P329: DP-Dep "uses all the CPU cores and the GPU" as equal workers).
+# PART-k: k equal green contexts with disjoint SMs (the GPU's remaining SMs
+# idle) — identical processors that, unlike HOMO-k, do not share SMs; only
+# HBM is still shared.
 PLATFORMS = {"HET-2": [0, 16], "HOMO-2": [0, 0], "HET-4": [0, 16, 16, 16], "HOMO-4": [0, 0, 0, 0],
-             "HET-8": [0, 8, 8, 8, 8, 8, 8, 8]}
+             "HET-8": [0, 8, 8, 8, 8, 8, 8, 8],
+             "PART-2": [72, 72], "PART-4": [32, 32, 32, 32], "PART-8": [16] * 8}
 
 
 def expected_order(cls, sync):
@@ -82,6 +86,9 @@ def emulation_note(budgets, cls, app_id):
         if cls == mm.MM_MK_DAG:
             notes.append("MK-DAG: a strategy that keeps the DAG on one device wins by construction here; "
                          "on separate GPUs it would leave the others idle")
+    elif len(set(budgets)) == 1 and app_id in MEM_BOUND:
+        notes.append("PART: equal SM partitions of one GPU share its HBM, so a memory-bound kernel on one "
+                     "device runs faster while the others idle (single-GPU artefact)")
     elif app_id in MEM_BOUND:
         notes.append("HET: SMs are partitioned (green contexts) but HBM bandwidth is shared, so memory-bound "
                      "kernels of the small devices steal bandwidth from the big one (single-GPU artefact)")
