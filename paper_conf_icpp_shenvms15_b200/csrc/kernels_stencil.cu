@@ -118,6 +118,7 @@ __global__ void __launch_bounds__(kThreads) hotspot_vec(const float* __restrict_
 // latency-bound on their level chains.  CTAs of 4 or 6 warps: 45.6 / 46.2 ms;
 // CTA barriers every 6-48 steps: slower.
 constexpr int kTbWarps = 12;                     // warps per CTA
+constexpr int kTbHeadGroups = 5;                 // 3-step groups at a strip's head with fewer levels (>= (2H - 1) / 3 for H <= 8)
 constexpr int kTbAhead = 3;                      // cp.async prefetch distance (rows, beyond a 3-step group)
 
 // Level-0 rings in shared memory, [row slot][group j][lane] so the lanes'
@@ -260,11 +261,13 @@ __device__ __forceinline__ void tb_fetch(TbArgs& a, int q) {
 // step is the grid's first or last row; CE = the warp holds the chip's first
 // or last column (both warp-uniform, so interior steps of interior warps run
 // without boundary selects).  tb = T row r, pb = P row r (ring bases).
-template <int H, int CL, int PH, bool EDGE, bool CE>
+// HEAD: only levels 1..smax (the strip's first steps, see tb_run).
+template <int H, int CL, int PH, bool EDGE, bool CE, bool HEAD = false>
 __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tb, const float4* pb,
-                                          const TbArgs& a, int r, const HotCoef2& k) {
+                                          const TbArgs& a, int r, const HotCoef2& k, int smax = H) {
 #pragma unroll
   for (int s = 1; s <= H; ++s) {
+    if (HEAD && s > smax) break;
     const int y = r - s;
     float4 cu[CL], up[CL], dn[CL], p[CL];
 #pragma unroll
@@ -309,9 +312,9 @@ __device__ __forceinline__ void tb_levels(float4 (&W)[H > 1 ? H - 1 : 1][3][CL],
 // no cp.async instructions (asm volatile, memory clobber) that would keep
 // ptxas from interleaving the steps' level chains (measured: 40.8 vs 41.6 ms
 // with a fetch + wait in every step).
-template <int H, int CL, int PH, bool CE>
+template <int H, int CL, int PH, bool CE, bool HEAD = false>
 __device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
-                                        TbArgs& a, int r, const HotCoef2& k) {
+                                        TbArgs& a, int r, const HotCoef2& k, int smax = H) {
   using C = TbCfg<H, CL>;
   if (PH == 0) {
     tb_fetch<H, CL>(a, r + kTbAhead);
@@ -321,7 +324,9 @@ __device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], c
   }
   const float4* tb = tr + ((r & (C::RT - 1)) + C::MT) * CL * 32;
   const float4* pb = pr + ((r & (C::RP - 1)) + C::MP) * CL * 32;
-  if ((unsigned)(r - H - 1) < (unsigned)a.eh)
+  if (HEAD)       // strip head: boundary selects always on (rare steps)
+    tb_levels<H, CL, PH, true, CE, true>(W, tb, pb, a, r, k, smax);
+  else if ((unsigned)(r - H - 1) < (unsigned)a.eh)
     tb_levels<H, CL, PH, false, CE>(W, tb, pb, a, r, k);
   else
     tb_levels<H, CL, PH, true, CE>(W, tb, pb, a, r, k);
@@ -333,7 +338,17 @@ __device__ __forceinline__ void tb_step(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], c
 template <int H, int CL, bool CE>
 __device__ __forceinline__ void tb_run(float4 (&W)[H > 1 ? H - 1 : 1][3][CL], const float4* tr, const float4* pr,
                                        TbArgs& a, int rb, int ngroups, const HotCoef2& k) {
-  for (int g = 0, r = rb; g < ngroups; ++g, r += 3) {
+  // The strip's first 2H - 2 steps (t = r - rb): level s computes row
+  // rb + t - s, which only feeds stored cells from t = 2s - 1 on (row
+  // >= Y0 - (H - s)), so step t runs levels 1 .. (t + 1) / 2; a skipped
+  // level's window keeps stale values that only reach rows never stored.
+  // Saves H^2 of the strip's (SR + 2H - 1) H level-rows (2.2 % at SR = 342).
+  for (int g = 0, r = rb; g < kTbHeadGroups; ++g, r += 3) {
+    tb_step<H, CL, 0, CE, true>(W, tr, pr, a, r, k, (3 * g + 1) / 2);
+    tb_step<H, CL, 1, CE, true>(W, tr, pr, a, r + 1, k, (3 * g + 2) / 2);
+    tb_step<H, CL, 2, CE, true>(W, tr, pr, a, r + 2, k, (3 * g + 3) / 2);
+  }
+  for (int g = kTbHeadGroups, r = rb + 3 * kTbHeadGroups; g < ngroups; ++g, r += 3) {
     tb_step<H, CL, 0, CE>(W, tr, pr, a, r, k);
     tb_step<H, CL, 1, CE>(W, tr, pr, a, r + 1, k);
     tb_step<H, CL, 2, CE>(W, tr, pr, a, r + 2, k);
