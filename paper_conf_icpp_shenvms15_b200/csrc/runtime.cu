@@ -1656,9 +1656,11 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     }
     t0 = std::chrono::steady_clock::now();
     CU_OK(set_dev(ctx, root));
-    CU_OK(cudaEventRecord(rt->t_start, rs));
+    // enqueue-only runs report no device time: no start/stop events around them
+    const bool ev = !(o && o->no_wait && !timing);
+    if (ev) CU_OK(cudaEventRecord(rt->t_start, rs));
     CU_OK(cudaGraphLaunch(rt->gexec, rs));
-    CU_OK(cudaEventRecord(rt->t_stop, rs));
+    if (ev) CU_OK(cudaEventRecord(rt->t_stop, rs));
     S->n_launches = rt->graph_launches;
     S->xfer_bytes = rt->graph_xfer;
     S->h2d_bytes = rt->graph_h2d;
@@ -1666,7 +1668,8 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     g_kernel_launches.fetch_add(rt->graph_launches, std::memory_order_relaxed);
   } else {
     CU_OK(set_dev(ctx, root));
-    CU_OK(cudaEventRecord(rt->t_start, rs));
+    const bool ev = !(o && o->no_wait && !timing);
+    if (ev) CU_OK(cudaEventRecord(rt->t_start, rs));
     const int64_t l0 = g_kernel_launches.load();
     for (int32_t rep = 0; rep < reps && !r; ++rep) {
       if (ctx->world == 1) r = issue_local(ctx, plan, buffers, o, timing, S);
@@ -1676,7 +1679,7 @@ mm_status mm_run(mm_ctx* ctx, mm_plan* plan_h, void* const* buffers, const mm_ru
     S->n_launches = g_kernel_launches.load() - l0;
     if (r) return r;
     CU_OK(set_dev(ctx, root));
-    CU_OK(cudaEventRecord(rt->t_stop, rs));
+    if (ev) CU_OK(cudaEventRecord(rt->t_stop, rs));
   }
   if (o && o->no_wait && !timing) {
     // enqueue only: every library stream of this run is joined into the root
