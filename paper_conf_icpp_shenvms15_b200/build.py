@@ -26,7 +26,7 @@ CUDA_INC = "/usr/local/cuda/include"
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
                      "-Xptxas", "-v", "--expt-relaxed-constexpr",
-                     "-I", INC, "-I", CSRC]
+                     "-I", INC, "-I", CSRC] + os.environ.get("MM_NVCC_EXTRA", "").split()   # dev experiments
 CXX_FLAGS = ["-O2", "-std=c++17", "-fPIC", "-Wall", "-Wextra", "-Wno-unused-parameter",
              "-I", INC, "-I", CSRC, "-I", CUDA_INC]
 
