@@ -117,3 +117,24 @@ def test_cholesky_single_tile(R, b, strategy):
         L = s.collect(plan, 0).reshape(b, b)
     assert np.array_equal(np.tril(L), L0)
     assert np.all(np.triu(L, 1) == 0)
+
+
+@pytest.mark.parametrize("shape", [(1, 4), (2, 8), (5, 12), (9, 1028), (17, 116)])
+@pytest.mark.parametrize("tb", [3, 8])
+@pytest.mark.parametrize("G", [1, 2])
+def test_hotspot_temporal_block_small_grids(R, shape, tb, G):
+    """Temporal blocks on grids shorter than the block's halo (rows < 2 tb),
+    one or two float4 columns, and widths just past one warp tile (116 = 112
+    output columns + 4): the strip head, the chip-edge warps and the grid's
+    first/last rows in one launch; bit-identical to the oracle."""
+    mm, runner = R
+    rows, cols = shape
+    iters = 2 * tb
+    t0, p = synthgen.hotspot(rows, cols)
+    ref = on.hotspot_run(t0, p, iters)
+    with runner.session(mm.MM_APP_HOTSPOT, [rows, cols, iters, 1, 1, tb], G=G) as s:
+        s.fill()
+        plan = s.plan(1, prof(mm, G, 1), chunks_per_dev=2)
+        s.run(plan)
+        got = s.collect(plan, 0).reshape(rows, cols)
+    assert np.array_equal(got, ref), (shape, tb, G)
